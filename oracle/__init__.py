@@ -1,0 +1,162 @@
+"""CPU oracle for CuSha's shard-processing path — TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s cpu_baseline /
+``--impl reference`` legs may import this package.  The product package
+(``paper_conf_hpdc_khorasanivgb14_b200``) never imports it and shares no code
+with it.  The arithmetic lives in ``oracle.c`` (plain single-threaded C, fp64
+for floating point); this file only marshals numpy arrays through ctypes.
+
+Parity pins for every function are in ``tests/test_oracle_*.py`` (no GPU).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "liboracle.so")
+_SRC = os.path.join(_HERE, "oracle.c")
+_lib = None
+
+INF = 0xFFFFFFFF
+OK, NOTCONV = 0, 1
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so: plain C11, single-threaded, -O2."""
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+        tmp = _SO + ".tmp%d" % os.getpid()
+        subprocess.check_call(["gcc", "-O2", "-shared", "-fPIC", "-std=c11", "-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, _SO)
+    return _SO
+
+
+def _L():
+    global _lib
+    if _lib is None:
+        build()
+        lib = ctypes.CDLL(_SO)
+        u64, u32, dbl, P = ctypes.c_uint64, ctypes.c_uint32, ctypes.c_double, ctypes.c_void_p
+        sig = {
+            "or_bfs": [u64, u64, P, P, u32, P],
+            "or_sssp": [u64, u64, P, P, P, u32, P],
+            "or_sswp": [u64, u64, P, P, P, u32, P],
+            "or_cc": [u64, u64, P, P, P],
+            "or_pagerank": [u64, u64, P, P, dbl, dbl, u64, P, P],
+            "or_nn": [u64, u64, P, P, P, P, dbl, u64, P, P],
+            "or_hs": [u64, u64, P, P, P, P, dbl, u64, P, P],
+            "or_cs": [u64, u64, P, P, P, P, P, dbl, u64, P, P],
+            "or_build_shards": [u64, u64, P, P, u32, P, P, P, P, P, P, P, P],
+        }
+        for name, args in sig.items():
+            f = getattr(lib, name)
+            f.argtypes = args
+            f.restype = ctypes.c_int
+        _lib = lib
+    return _lib
+
+
+def _p(a):
+    return None if a is None else a.ctypes.data_as(ctypes.c_void_p)
+
+
+def _u32(a):
+    return np.ascontiguousarray(a, dtype=np.uint32)
+
+
+def _f32(a):
+    return np.ascontiguousarray(a, dtype=np.float32)
+
+
+def _chk(rc, name, allow_notconv=False):
+    if rc < 0 or (rc == NOTCONV and not allow_notconv):
+        raise RuntimeError(f"oracle.{name} rc={rc}")
+    return rc
+
+
+def bfs(V, src, dst, source=0):
+    src, dst = _u32(src), _u32(dst)
+    out = np.empty(V, np.uint32)
+    _chk(_L().or_bfs(V, len(src), _p(src), _p(dst), source, _p(out)), "bfs")
+    return out
+
+
+def sssp(V, src, dst, weight, source=0):
+    src, dst, weight = _u32(src), _u32(dst), _u32(weight)
+    out = np.empty(V, np.uint32)
+    _chk(_L().or_sssp(V, len(src), _p(src), _p(dst), _p(weight), source, _p(out)), "sssp")
+    return out
+
+
+def sswp(V, src, dst, width, source=0):
+    src, dst, width = _u32(src), _u32(dst), _u32(width)
+    out = np.empty(V, np.uint32)
+    _chk(_L().or_sswp(V, len(src), _p(src), _p(dst), _p(width), source, _p(out)), "sswp")
+    return out
+
+
+def cc(V, src, dst):
+    src, dst = _u32(src), _u32(dst)
+    out = np.empty(V, np.uint32)
+    _chk(_L().or_cc(V, len(src), _p(src), _p(dst), _p(out)), "cc")
+    return out
+
+
+def pagerank(V, src, dst, damping=0.85, tol=1e-9, max_iters=100000):
+    """Returns (rank float64[V], sweeps)."""
+    src, dst = _u32(src), _u32(dst)
+    out = np.empty(V, np.float64)
+    it = ctypes.c_uint64(0)
+    _chk(_L().or_pagerank(V, len(src), _p(src), _p(dst), damping, tol, max_iters, _p(out), ctypes.byref(it)), "pagerank")
+    return out, it.value
+
+
+def nn(V, src, dst, weight, x0, tol=1e-9, max_iters=100000):
+    src, dst, weight, x0 = _u32(src), _u32(dst), _f32(weight), _f32(x0)
+    out = np.empty(V, np.float64)
+    it = ctypes.c_uint64(0)
+    _chk(_L().or_nn(V, len(src), _p(src), _p(dst), _p(weight), _p(x0), tol, max_iters, _p(out), ctypes.byref(it)), "nn")
+    return out, it.value
+
+
+def hs(V, src, dst, coeff, q0, tol=1e-9, max_iters=100000):
+    src, dst, coeff, q0 = _u32(src), _u32(dst), _f32(coeff), _f32(q0)
+    out = np.empty(V, np.float64)
+    it = ctypes.c_uint64(0)
+    _chk(_L().or_hs(V, len(src), _p(src), _p(dst), _p(coeff), _p(q0), tol, max_iters, _p(out), ctypes.byref(it)), "hs")
+    return out, it.value
+
+
+def cs(V, src, dst, G, v0, a0, tol=1e-9, max_iters=100000):
+    src, dst, G, v0, a0 = _u32(src), _u32(dst), _f32(G), _f32(v0), _f32(a0)
+    out = np.empty(V, np.float64)
+    it = ctypes.c_uint64(0)
+    _chk(_L().or_cs(V, len(src), _p(src), _p(dst), _p(G), _p(v0), _p(a0), tol, max_iters, _p(out), ctypes.byref(it)),
+         "cs")
+    return out, it.value
+
+
+def build_shards(V, src, dst, N):
+    """G-Shards + CW layout by definition. Returns a dict of numpy arrays."""
+    src, dst = _u32(src), _u32(dst)
+    E = len(src)
+    S = (V + N - 1) // N
+    r = dict(
+        S=S,
+        shard_off=np.empty(S + 1, np.uint64),
+        gs_src=np.empty(E, np.uint32),
+        gs_dst=np.empty(E, np.uint32),
+        gs_eid=np.empty(E, np.uint64),
+        win=np.empty((S + 1) * S, np.uint64),
+        cw_off=np.empty(S + 1, np.uint64),
+        cw_src=np.empty(E, np.uint32),
+        mapper=np.empty(E, np.uint64),
+    )
+    _chk(_L().or_build_shards(V, E, _p(src), _p(dst), N, _p(r["shard_off"]), _p(r["gs_src"]), _p(r["gs_dst"]),
+                              _p(r["gs_eid"]), _p(r["win"]), _p(r["cw_off"]), _p(r["cw_src"]), _p(r["mapper"])),
+         "build_shards")
+    r["win"] = r["win"].reshape(S + 1, S)
+    return r
