@@ -1,0 +1,239 @@
+/*
+ * cusha.h — C ABI of the B200-native CuSha shard-processing path.
+ *
+ * Paper: F. Khorasani, K. Vora, R. Gupta, L. N. Bhuyan, "CuSha: Vertex-Centric
+ * Graph Processing on GPUs", HPDC'14.  Citations "L<n>" are lines of the
+ * paper text with the section / figure / table they fall in.
+ *
+ * Problem statement (L45, §4): the user picks a
+ * vertex-centric algorithm (Table 3: a Vertex / StaticVertex / Edge
+ * type and init_compute / compute / update_condition); CuSha lays the graph
+ * out as G-Shards (§3.1) or Concatenated Windows (§3.2),
+ * chooses the shard size itself (L310), iterates the 4-stage shard pass
+ * (Fig. 5) until an iteration commits no update (L189), and returns
+ * the final vertex values (copied to the host only at the end, L457).  The
+ * eight Table-3 algorithms are compiled in; the ABI selects one by enum.
+ *
+ * Conventions for every entry point:
+ *  - Plain C types only.  Pointers documented "host" are ordinary host
+ *    memory; "device" pointers are CUDA device pointers on opts->device.
+ *  - Return value: CUSHA_OK (0) or a positive informational code on success,
+ *    a negative CUSHA_E* code on failure; cusha_last_error() then returns a
+ *    thread-local message.  No exception or longjmp crosses the ABI.
+ *  - The library never reads caller memory after a call returns.
+ *  - Thread safety: distinct graphs may be used from distinct threads; one
+ *    graph must not be used concurrently.
+ *  - Limits: |V| < 2^31, |E| < 2^32 - 2^26 (offsets are 32-bit), and
+ *    vertices_per_shard <= 65534 (16-bit local indices).
+ */
+#ifndef CUSHA_H
+#define CUSHA_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(__GNUC__)
+#define CUSHA_API __attribute__((visibility("default")))
+#else
+#define CUSHA_API
+#endif
+
+#define CUSHA_ABI_VERSION 1
+
+/* Return codes. */
+enum {
+  CUSHA_OK = 0,
+  CUSHA_NOT_CONVERGED = 1,   /* max_iters reached; values of the last iteration are retrievable */
+  CUSHA_EINVAL = -1,         /* bad argument (null pointer, id out of range, size mismatch, ...) */
+  CUSHA_ENOMEM = -2,         /* device or host allocation failed */
+  CUSHA_ECUDA = -3,          /* CUDA runtime error (message names the call) */
+  CUSHA_ENCCL = -4,          /* NCCL error (multi-GPU) */
+  CUSHA_EUNSUPPORTED = -5,   /* feature not available in this build / configuration */
+  CUSHA_ESTATE = -6          /* call out of order (e.g. get_values before any run) */
+};
+
+/* The eight benchmark algorithms of Table 3 (L314-325), in the table's order. */
+typedef enum {
+  CUSHA_BFS = 0,   /* Vertex {u32 Level};           L316 */
+  CUSHA_SSSP = 1,  /* Vertex {u32 Dist}, Edge {u32 Weight}; L317, Fig. 6 */
+  CUSHA_PR = 2,    /* Vertex {f32 Rank}, StaticVertex {u32 NbrsNum}; L318 */
+  CUSHA_CC = 3,    /* Vertex {u32 Cmpnent};         L319 */
+  CUSHA_SSWP = 4,  /* Vertex {u32 BWidth}, Edge {u32 Width}; L320 */
+  CUSHA_NN = 5,    /* Vertex {f32 x}, Edge {f32 Weight}; L321 */
+  CUSHA_HS = 6,    /* Vertex {f32 Q, f32 Q_new}, Edge {f32 coeff}; L322 */
+  CUSHA_CS = 7     /* Vertex {f32 V, f32 GsumOrA}, Edge {f32 G}; L323 */
+} cusha_algorithm;
+
+/* Graph representation (§3.1 G-Shards, §3.2 Concatenated Windows). */
+typedef enum { CUSHA_REPR_GSHARDS = 0, CUSHA_REPR_CW = 1 } cusha_repr;
+
+/* Where cusha_build_graph's src/dst/edge_values live. */
+typedef enum { CUSHA_INPUT_HOST = 0, CUSHA_INPUT_DEVICE = 1 } cusha_input_location;
+
+typedef struct {
+  cusha_repr repr;                 /* G-Shards or CW (default G-Shards)                        */
+  uint32_t vertices_per_shard;     /* |N|; 0 = the paper's rule (L310, cusha_shard_size)       */
+  uint32_t smem_bytes_per_vertex;  /* sizeof(Vertex) assumed by the |N| rule; 0 = 4 (L310)     */
+  int device;                      /* CUDA device ordinal                                      */
+  void* stream;                    /* cudaStream_t to run on; NULL = a library-owned stream    */
+  cusha_input_location input_location; /* host (copied in, timed as H2D) or device            */
+  /* Multi-GPU (destination-range partition): */
+  int world_size;                  /* 1 = single GPU (0 is treated as 1)                       */
+  int rank;                        /* this process's rank, 0..world_size-1                     */
+  const void* nccl_unique_id;      /* 128-byte ncclUniqueId shared by all ranks (world_size>1) */
+} cusha_build_opts;
+
+typedef struct cusha_graph cusha_graph;   /* opaque; owns all device memory it allocates */
+
+typedef struct {
+  uint32_t num_vertices;
+  uint64_t num_edges;
+  uint32_t vertices_per_shard;     /* |N| actually used                                        */
+  uint32_t num_shards;             /* |S| = ceil(|V| / |N|) (L173)                             */
+  uint32_t repr;                   /* cusha_repr                                               */
+  int32_t last_algorithm;          /* -1 before the first run                                  */
+  uint32_t iterations;             /* shard passes of the last run (incl. the converged one)   */
+  uint32_t converged;              /* 1 if the last run's final pass committed nothing         */
+  double build_ms;                 /* cusha_build_graph wall time on the stream (incl. H2D)    */
+  double h2d_ms;                   /* part of build_ms spent copying host inputs              */
+  double run_ms;                   /* last cusha_run: init + all shard passes (device events)  */
+  double loop_ms;                  /* last cusha_run: the shard passes only (device events)    */
+  uint64_t h2d_bytes;              /* bytes copied host->device by the build                   */
+  uint64_t device_bytes;           /* topology + value arrays resident on the device           */
+  uint64_t entries_padded;         /* shard entries incl. vector padding                       */
+  uint64_t stage2_bytes_per_iter;  /* algorithmic bytes stage 2 streams per iteration          */
+  uint64_t wb_bytes_all_active;    /* stage-4 algorithmic bytes if every shard is active       */
+  uint64_t algorithmic_bytes;      /* last run: sum over iterations of stage1..4 algorithmic bytes */
+  uint64_t edges_processed;        /* last run: iterations * |E|                                */
+  uint32_t device_loop;            /* 1 = the run looped on the device (CUDA-graph while node) */
+  int world_size, rank;
+} cusha_stats;
+
+/* ---------------------------------------------------------------- build */
+/*
+ * Build the G-Shards / CW representation of a directed graph (row a0).
+ *   num_vertices, num_edges  |V|, |E|.
+ *   src, dst                 edge endpoints, num_edges each, values < num_vertices
+ *                            (host or device per opts->input_location; caller-owned,
+ *                            read only during the call).  An edge u->v is stored in
+ *                            the shard that owns v (incoming edges, L119).
+ *   edge_values              nullable; num_edges raw 4-byte values: u32 Weight (SSSP),
+ *                            u32 Width (SSWP) or f32 bits (NN Weight, HS coeff, CS G).
+ *   opts                     nullable = defaults.
+ *   out                      receives the graph handle.
+ * Layout (L119-179): shard s owns vertices [s*|N|, (s+1)*|N|); its entries are
+ * sorted by (SrcIndex, DestIndex, input order) (Ordered L129; tie-break DESIGN.md
+ * R17); window W_ij (L155) and, for CW, CW_i and Mapper (L175) are derived from
+ * that order.  |N| = opts->vertices_per_shard or the L310 rule.  Duplicates and
+ * self-loops are kept as separate edges (R22).
+ * Errors: CUSHA_EINVAL (null src/dst/out with |E|>0, |V|=0, endpoint >= |V|,
+ * limits), CUSHA_ENOMEM, CUSHA_ECUDA.
+ */
+CUSHA_API int cusha_build_graph(uint32_t num_vertices, uint64_t num_edges, const uint32_t* src, const uint32_t* dst,
+                      const uint32_t* edge_values, const cusha_build_opts* opts, cusha_graph** out);
+
+/* Release every resource of g (NULL is ignored). */
+CUSHA_API void cusha_free_graph(cusha_graph* g);
+
+/*
+ * Initial vertex values for the next cusha_run of `alg` (host pointer, copied).
+ * Required for NN (f32 x0[|V|]), HS (f32 Q0[|V|]) and CS (f32 pairs
+ * {V0, GsumOrA0}[|V|]; GsumOrA0 != 0 marks an anchor, R15).  Optional for the
+ * others (overrides the Table-3 start state; e.g. to resume).  bytes must equal
+ * |V| * cusha_value_bytes(alg).  Errors: CUSHA_EINVAL.
+ */
+CUSHA_API int cusha_set_vertex_values(cusha_graph* g, cusha_algorithm alg, const void* init, size_t bytes);
+
+/* ------------------------------------------------------------------ run */
+/*
+ * Run `alg` to convergence (rows a1-a5): initialise VertexValues (Table 3
+ * start state, L327) and every SrcValue copy (R20), then repeat the shard
+ * pass (Fig. 5) until a pass commits no update (L189) or max_iters passes ran.
+ *   source     BFS/SSSP/SSWP start vertex (< |V|); ignored by the others.
+ *   max_iters  upper bound on shard passes (R23); 0 = do nothing.
+ * The iteration loop runs on the device (one CUDA-graph launch with a
+ * conditional while node); the host waits once at the end.
+ * Returns CUSHA_OK, CUSHA_NOT_CONVERGED, or CUSHA_EINVAL (bad source, NN/HS/CS
+ * without initial values, EdgeValue needed but absent) / CUSHA_ECUDA.
+ */
+CUSHA_API int cusha_run(cusha_algorithm alg, cusha_graph* g, uint32_t source, uint32_t max_iters);
+
+/*
+ * Copy the last run's VertexValues (|V| * cusha_value_bytes(alg) bytes) to
+ * `out` (host) / `dptr` (device).  Element types: u32 Level / Dist / Cmpnent /
+ * BWidth (INF = 0xFFFFFFFF, R1); f32 Rank / x; {f32 Q, f32 Q_new};
+ * {f32 V, f32 GsumOrA}.  out_bytes must be exactly that size.
+ * Errors: CUSHA_EINVAL (size), CUSHA_ESTATE (no run yet).
+ */
+CUSHA_API int cusha_get_values(const cusha_graph* g, void* out, size_t out_bytes);
+CUSHA_API int cusha_get_values_device(const cusha_graph* g, void* dptr, size_t out_bytes);
+
+/* Statistics of the graph and of its last run (host struct, filled). */
+CUSHA_API int cusha_get_stats(const cusha_graph* g, cusha_stats* s);
+
+/*
+ * Per-iteration trace of the last run (row f4 / Fig. 7): for i <
+ * min(iterations, cap): updated_vertices[i] (committed updates) and
+ * active_shards[i] (shards that ran stage 4).  Either pointer may be NULL.
+ * Returns the number of iterations written.
+ */
+CUSHA_API int cusha_get_trace(const cusha_graph* g, uint32_t* updated_vertices, uint32_t* active_shards, uint32_t cap);
+
+/* ------------------------------------------------------- layout export */
+/* Device arrays of the representation, copied to host for inspection/tests.
+ * Positions are "padded": each shard's (and each CW_i's) entries start at a
+ * multiple of 8 and are followed by filler entries up to the next multiple
+ * of 8.                                                */
+typedef enum {
+  CUSHA_LAYOUT_SHARD_OFFSETS = 0,   /* u32[|S|+1] first padded position of shard s          */
+  CUSHA_LAYOUT_SHARD_SIZES = 1,     /* u32[|S|]   real entries of shard s                   */
+  CUSHA_LAYOUT_SRC_INDEX = 2,       /* u32[P]     SrcIndex (global) per padded entry (GS)   */
+  CUSHA_LAYOUT_DEST_LOCAL = 3,      /* u16[P]     DestIndex - s*|N| (filler = |N|)         */
+  CUSHA_LAYOUT_EDGE_ID = 4,         /* u32[P]     input edge index (filler = 0xFFFFFFFF)    */
+  CUSHA_LAYOUT_WINDOWS = 5,         /* u32[(|S|+1)*|S|] win[i*|S|+j] = start of W_ij        */
+  CUSHA_LAYOUT_CW_OFFSETS = 6,      /* u32[|S|+1] first padded position of CW_i             */
+  CUSHA_LAYOUT_CW_SIZES = 7,        /* u32[|S|]   real entries of CW_i                      */
+  CUSHA_LAYOUT_CW_SRC_LOCAL = 8,    /* u16[Q]     SrcIndex - i*|N| per padded CW entry      */
+  CUSHA_LAYOUT_MAPPER = 9,          /* u32[Q]     padded shard position (filler = trash P)  */
+  CUSHA_LAYOUT_OUT_DEGREE = 10      /* u32[|V|]   out-degree (PR NbrsNum, L318)            */
+} cusha_layout_part;
+/* Returns the element count of `part` in *count (bytes = count * element size);
+ * copies it to `out` (host) when out != NULL and out_bytes is large enough.
+ * Parts not held by the representation return CUSHA_EUNSUPPORTED.          */
+CUSHA_API int cusha_get_layout(const cusha_graph* g, cusha_layout_part part, void* out, size_t out_bytes, uint64_t* count);
+
+/* ---------------------------------------------------------- host logic */
+/*
+ * The shard-size rule of L310 (§4 "Selecting shard size"), pure host code:
+ * |N|0 = the |N| making the average window |E||N|^2/|V|^2 (L173) equal 32
+ * (warp size), then snapped to the nearest of the sizes that use a whole
+ * share of the SM's shared memory, N_k = floor((smem_per_sm/k - reserved)/
+ * vertex_bytes) for k = 1..32 resident blocks, capped at 65534 and at |V|.
+ * smem_per_sm = 0 selects B200's 233472 bytes per SM with reserved_per_block =
+ * 1024 (the value passed is then ignored); otherwise both are taken as given
+ * (e.g. 49152 / 0 reproduces L310's 48 KB examples: 6K at 2 blocks, 3K at 4).
+ */
+CUSHA_API uint32_t cusha_shard_size(uint32_t num_vertices, uint64_t num_edges, uint32_t vertex_bytes, uint32_t smem_per_sm,
+                          uint32_t reserved_per_block);
+
+/* Bytes per vertex of cusha_get_values for alg (4 or 8), 0 if invalid. */
+CUSHA_API size_t cusha_value_bytes(cusha_algorithm alg);
+
+/* Thread-local message for the last failing call on this thread ("" if none). */
+CUSHA_API const char* cusha_last_error(void);
+
+/* CUSHA_ABI_VERSION of the loaded library. */
+CUSHA_API int cusha_abi_version(void);
+
+/* Multi-GPU helper: write a fresh 128-byte ncclUniqueId to out128 (rank 0
+ * calls this and broadcasts it, e.g. over torch.distributed). */
+CUSHA_API int cusha_nccl_unique_id(void* out128);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CUSHA_H */

@@ -105,12 +105,14 @@ def cc(V, src, dst):
     return out
 
 
-def pagerank(V, src, dst, damping=0.85, tol=1e-9, max_iters=100000):
-    """Returns (rank float64[V], sweeps)."""
+def pagerank(V, src, dst, damping=0.85, tol=1e-9, max_iters=100000, allow_notconv=False):
+    """Returns (rank float64[V], sweeps).  allow_notconv: stopping at max_iters
+    is not an error (used to time a bounded number of sweeps)."""
     src, dst = _u32(src), _u32(dst)
     out = np.empty(V, np.float64)
     it = ctypes.c_uint64(0)
-    _chk(_L().or_pagerank(V, len(src), _p(src), _p(dst), damping, tol, max_iters, _p(out), ctypes.byref(it)), "pagerank")
+    _chk(_L().or_pagerank(V, len(src), _p(src), _p(dst), damping, tol, max_iters, _p(out), ctypes.byref(it)),
+         "pagerank", allow_notconv=allow_notconv)
     return out, it.value
 
 

@@ -1,0 +1,421 @@
+// api.cu — the C ABI of include/cusha.h (row b) and the iteration driver (row a5).
+//
+// cusha_run replaces the paper's host loop (Fig. 5 lines 0-2 and 29; L189:
+// launch, cudaMemcpy(is_converged), decide) by ONE launch of a CUDA graph
+// whose body is the shard pass under a conditional while node; the shard
+// pass's last CTA decides whether the loop goes on (DESIGN.md "Iteration
+// control").  The host waits once, at the end.
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstring>
+#include <string>
+
+#include "algorithms.cuh"
+#include "graph.hpp"
+
+struct cusha_graph {
+  cusha::Graph g;
+  cudaGraphExec_t exec[cusha::kNumAlgs] = {};
+  bool exec_failed[cusha::kNumAlgs] = {};
+};
+
+namespace cusha {
+
+static thread_local std::string t_err;
+void set_error(const std::string& msg) { t_err = msg; }
+
+static int fail(int code, const std::string& msg) {
+  set_error(msg);
+  return code;
+}
+
+#define CKA(call)                                                                                  \
+  do {                                                                                             \
+    cudaError_t e_ = (call);                                                                       \
+    if (e_ != cudaSuccess) {                                                                       \
+      return fail(e_ == cudaErrorMemoryAllocation ? CUSHA_ENOMEM : CUSHA_ECUDA,                    \
+                  std::string(#call) + ": " + cudaGetErrorString(e_));                             \
+    }                                                                                              \
+  } while (0)
+
+static void free_graph_memory(Graph& g) {
+  void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcidx, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
+                  g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_srcvalue, g.d_vv, g.d_ctl, g.d_trace};
+  for (void* p : ptrs)
+    if (p) cudaFree(p);
+  for (void*& p : g.d_init)
+    if (p) { cudaFree(p); p = nullptr; }
+  if (g.h_ctl) cudaFreeHost(g.h_ctl);
+  if (g.ev0) cudaEventDestroy(g.ev0);
+  if (g.ev1) cudaEventDestroy(g.ev1);
+  if (g.evm) cudaEventDestroy(g.evm);
+  if (g.own_stream && g.stream) cudaStreamDestroy(g.stream);
+}
+
+static uint64_t device_bytes(const Graph& g) {
+  uint64_t b = 4ull * (g.S + 1) * 2 + 4ull * g.S * 2;  // offsets + counts
+  b += 2 * g.P + 4 * g.P;                               // dest + eid
+  if (g.has_ev) b += 4 * g.P;
+  if (g.d_srcidx) b += 4 * g.P;
+  if (g.d_win) b += 4ull * (g.S + 1) * g.S;
+  b += (2 + 4) * g.Q;                                   // CW
+  b += 4ull * g.V;                                      // outdeg
+  b += 4 * (g.P + 1) + 8ull * g.V;                      // SrcValue + VertexValues
+  return b;
+}
+
+}  // namespace cusha
+
+using namespace cusha;
+
+extern "C" {
+
+const char* cusha_last_error(void) { return t_err.c_str(); }
+int cusha_abi_version(void) { return CUSHA_ABI_VERSION; }
+
+size_t cusha_value_bytes(cusha_algorithm alg) {
+  if ((int)alg < 0 || (int)alg >= kNumAlgs) return 0;
+  return value_bytes((int)alg);
+}
+
+uint32_t cusha_shard_size(uint32_t V, uint64_t E, uint32_t vertex_bytes, uint32_t smem_per_sm,
+                          uint32_t reserved_per_block) {
+  // L310: |N| such that the average window |E||N|^2/|V|^2 (L173) is 32, then
+  // snapped to the nearest size that uses a whole share of the SM's shared memory.
+  if (V == 0) return 1;
+  if (vertex_bytes == 0) vertex_bytes = 4;
+  if (smem_per_sm == 0) {  // B200 defaults: 228 KB per SM, 1 KB reserved per resident CTA
+    smem_per_sm = 233472;
+    reserved_per_block = 1024;
+  }
+  double n0 = E ? (double)V * std::sqrt(32.0 / (double)E) : (double)V;
+  uint32_t best = 0;
+  double bestd = 1e300;
+  for (uint32_t k = 1; k <= 32; ++k) {
+    const int64_t q = (int64_t)(smem_per_sm / k) - (int64_t)reserved_per_block;
+    if (q <= 0) continue;
+    uint64_t nk = (uint64_t)q / vertex_bytes;
+    if (nk > 65534) nk = 65534;
+    if (nk == 0) continue;
+    const double d = std::fabs((double)nk - n0);
+    if (d < bestd) { bestd = d; best = (uint32_t)nk; }
+  }
+  if (best == 0) best = 1;
+  if (best > V) best = V;
+  return best;
+}
+
+int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_t* dst, const uint32_t* edge_values,
+                      const cusha_build_opts* opts, cusha_graph** out) {
+  if (!out) return fail(CUSHA_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (V == 0) return fail(CUSHA_EINVAL, "num_vertices must be > 0");
+  if (V >= (1u << 31)) return fail(CUSHA_EINVAL, "num_vertices must be < 2^31");
+  if (E >= 0xFFFFFFFFull - (1ull << 26)) return fail(CUSHA_EINVAL, "num_edges too large for 32-bit positions");
+  if (E && (!src || !dst)) return fail(CUSHA_EINVAL, "src/dst are NULL");
+  cusha_build_opts o{};
+  if (opts) o = *opts;
+  if (o.repr != CUSHA_REPR_GSHARDS && o.repr != CUSHA_REPR_CW) return fail(CUSHA_EINVAL, "bad repr");
+  if (o.world_size <= 0) o.world_size = 1;
+  if (o.world_size != 1) return fail(CUSHA_EUNSUPPORTED, "world_size > 1 requires cusha_build_graph_multi");
+  uint32_t N = o.vertices_per_shard ? o.vertices_per_shard : cusha_shard_size(V, E, o.smem_bytes_per_vertex, 0, 0);
+  if (N > 65534) return fail(CUSHA_EINVAL, "vertices_per_shard must be <= 65534");
+  if (N > V) N = V;
+
+  cusha_graph* h = new (std::nothrow) cusha_graph();
+  if (!h) return fail(CUSHA_ENOMEM, "host allocation");
+  Graph& g = h->g;
+  g.V = V; g.E = E; g.N = N; g.S = (V + N - 1) / N; g.repr = (int)o.repr; g.device = o.device;
+  auto bail = [&](int code) { free_graph_memory(g); delete h; return code; };
+  auto cu = [&](cudaError_t e, const char* what) -> int {
+    if (e == cudaSuccess) return 0;
+    set_error(std::string(what) + ": " + cudaGetErrorString(e));
+    return e == cudaErrorMemoryAllocation ? CUSHA_ENOMEM : CUSHA_ECUDA;
+  };
+  int rc;
+  if ((rc = cu(cudaSetDevice(o.device), "cudaSetDevice"))) return bail(rc);
+  if (o.stream) {
+    g.stream = (cudaStream_t)o.stream;
+  } else {
+    if ((rc = cu(cudaStreamCreateWithFlags(&g.stream, cudaStreamNonBlocking), "cudaStreamCreate"))) return bail(rc);
+    g.own_stream = true;
+  }
+  if ((rc = cu(cudaEventCreate(&g.ev0), "cudaEventCreate")) || (rc = cu(cudaEventCreate(&g.ev1), "cudaEventCreate")) ||
+      (rc = cu(cudaEventCreate(&g.evm), "cudaEventCreate")))
+    return bail(rc);
+  cudaEvent_t eh = nullptr;
+  if ((rc = cu(cudaEventCreate(&eh), "cudaEventCreate"))) return bail(rc);
+
+  auto t0 = std::chrono::steady_clock::now();
+  CKA(cudaEventRecord(g.ev0, g.stream));
+  const uint32_t *d_src = src, *d_dst = dst, *d_val = edge_values;
+  uint32_t* tmp = nullptr;
+  uint64_t h2d = 0;
+  if (o.input_location == CUSHA_INPUT_HOST && E) {
+    const uint64_t nvals = edge_values ? 3 : 2;
+    if ((rc = cu(cudaMalloc(&tmp, nvals * E * 4), "cudaMalloc(inputs)"))) { cudaEventDestroy(eh); return bail(rc); }
+    cudaMemcpyAsync(tmp, src, E * 4, cudaMemcpyHostToDevice, g.stream);
+    cudaMemcpyAsync(tmp + E, dst, E * 4, cudaMemcpyHostToDevice, g.stream);
+    if (edge_values) cudaMemcpyAsync(tmp + 2 * E, edge_values, E * 4, cudaMemcpyHostToDevice, g.stream);
+    d_src = tmp; d_dst = tmp + E; d_val = edge_values ? tmp + 2 * E : nullptr;
+    h2d = nvals * E * 4;
+  }
+  cudaEventRecord(eh, g.stream);
+  std::string err;
+  rc = build_layout(g, d_src, d_dst, d_val, err);
+  if (rc) {
+    if (tmp) cudaFree(tmp);
+    cudaEventDestroy(eh);
+    set_error("build: " + err);
+    return bail(rc);
+  }
+  if (tmp) cudaFree(tmp);
+  // per-run state: SrcValue (P entries + trash slot), VertexValues (8 B/vertex covers every Table-3 Vertex)
+  if ((rc = cu(cudaMalloc(&g.d_srcvalue, 4 * (g.P + 1)), "cudaMalloc(SrcValue)")) ||
+      (rc = cu(cudaMemsetAsync(g.d_srcvalue, 0, 4 * (g.P + 1), g.stream), "memset")) ||
+      (rc = cu(cudaMalloc(&g.d_vv, 8ull * V), "cudaMalloc(VertexValues)")) ||
+      (rc = cu(cudaMalloc(&g.d_ctl, sizeof(Ctl)), "cudaMalloc(ctl)")) ||
+      (rc = cu(cudaMallocHost(&g.h_ctl, sizeof(Ctl)), "cudaMallocHost(ctl)"))) {
+    cudaEventDestroy(eh);
+    return bail(rc);
+  }
+  CKA(cudaEventRecord(g.ev1, g.stream));
+  CKA(cudaEventSynchronize(g.ev1));
+  float ms = 0, ms_h2d = 0;
+  cudaEventElapsedTime(&ms, g.ev0, g.ev1);
+  cudaEventElapsedTime(&ms_h2d, g.ev0, eh);
+  cudaEventDestroy(eh);
+  (void)t0;
+  g.st.num_vertices = V;
+  g.st.num_edges = E;
+  g.st.vertices_per_shard = N;
+  g.st.num_shards = g.S;
+  g.st.repr = (uint32_t)g.repr;
+  g.st.last_algorithm = -1;
+  g.st.build_ms = ms;
+  g.st.h2d_ms = ms_h2d;
+  g.st.h2d_bytes = h2d;
+  g.st.device_bytes = device_bytes(g);
+  g.st.entries_padded = g.P;
+  g.st.world_size = 1;
+  g.st.rank = 0;
+  *out = h;
+  set_error("");
+  return CUSHA_OK;
+}
+
+void cusha_free_graph(cusha_graph* h) {
+  if (!h) return;
+  cudaSetDevice(h->g.device);
+  for (auto& e : h->exec)
+    if (e) cudaGraphExecDestroy(e);
+  free_graph_memory(h->g);
+  delete h;
+}
+
+int cusha_set_vertex_values(cusha_graph* h, cusha_algorithm alg, const void* init, size_t bytes) {
+  if (!h || !init) return fail(CUSHA_EINVAL, "null argument");
+  if ((int)alg < 0 || (int)alg >= kNumAlgs) return fail(CUSHA_EINVAL, "bad algorithm");
+  Graph& g = h->g;
+  const size_t want = (size_t)g.V * value_bytes((int)alg);
+  if (bytes != want) return fail(CUSHA_EINVAL, "bytes must be |V| * value_bytes(alg)");
+  CKA(cudaSetDevice(g.device));
+  if (!g.d_init[alg]) CKA(cudaMalloc(&g.d_init[alg], want));
+  CKA(cudaMemcpyAsync(g.d_init[alg], init, want, cudaMemcpyHostToDevice, g.stream));
+  CKA(cudaStreamSynchronize(g.stream));
+  return CUSHA_OK;
+}
+
+static int ensure_exec(cusha_graph* h, int alg) {
+  Graph& g = h->g;
+  if (h->exec[alg]) return CUSHA_OK;
+  const PassKernel& pk = pass_kernel(alg, g.repr);
+  const size_t smem = pk.smem_bytes(g.N);
+  if (smem > 227 * 1024)
+    return fail(CUSHA_EINVAL, "vertices_per_shard too large for this algorithm's shared-memory state");
+  CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  cudaGraph_t graph = nullptr;
+  CKA(cudaGraphCreate(&graph, 0));
+  cudaGraphConditionalHandle handle;
+  cudaError_t e = cudaGraphConditionalHandleCreate(&handle, graph, 1, cudaGraphCondAssignDefault);
+  if (e != cudaSuccess) { cudaGraphDestroy(graph); return fail(CUSHA_ECUDA, std::string("conditional handle: ") + cudaGetErrorString(e)); }
+  cudaGraphNodeParams cp = {};
+  cp.type = cudaGraphNodeTypeConditional;
+  cp.conditional.handle = handle;
+  cp.conditional.type = cudaGraphCondTypeWhile;
+  cp.conditional.size = 1;
+  cudaGraphNode_t cnode;
+  e = cudaGraphAddNode(&cnode, graph, nullptr, 0, &cp);
+  if (e != cudaSuccess) { cudaGraphDestroy(graph); return fail(CUSHA_ECUDA, std::string("conditional node: ") + cudaGetErrorString(e)); }
+  cudaGraph_t body = cp.conditional.phGraph_out[0];
+  KParams kp = make_params(g, 0);
+  kp.use_cond = 1;
+  kp.cond_handle = handle;
+  void* args[] = {&kp};
+  cudaKernelNodeParams knp = {};
+  knp.func = const_cast<void*>(pk.func);
+  knp.gridDim = dim3(g.S);
+  knp.blockDim = dim3(kThreads);
+  knp.sharedMemBytes = (unsigned)smem;
+  knp.kernelParams = args;
+  cudaGraphNode_t kn;
+  e = cudaGraphAddKernelNode(&kn, body, nullptr, 0, &knp);
+  if (e == cudaSuccess) e = cudaGraphInstantiate(&h->exec[alg], graph, 0);
+  cudaGraphDestroy(graph);
+  if (e != cudaSuccess) { h->exec[alg] = nullptr; return fail(CUSHA_ECUDA, std::string("graph: ") + cudaGetErrorString(e)); }
+  return CUSHA_OK;
+}
+
+int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max_iters) {
+  if (!h) return fail(CUSHA_EINVAL, "graph is NULL");
+  if ((int)alg < 0 || (int)alg >= kNumAlgs) return fail(CUSHA_EINVAL, "bad algorithm");
+  Graph& g = h->g;
+  const int a = (int)alg;
+  if ((a == kBFS || a == kSSSP || a == kSSWP) && source >= g.V) return fail(CUSHA_EINVAL, "source >= num_vertices");
+  if (alg_needs_edge_values(a) && !g.has_ev) return fail(CUSHA_EINVAL, "algorithm needs edge_values");
+  if (alg_needs_init(a) && !g.d_init[a]) return fail(CUSHA_EINVAL, "NN/HS/CS need cusha_set_vertex_values first");
+  CKA(cudaSetDevice(g.device));
+  // trace buffer sized to min(max_iters, 2^20)
+  const uint32_t want_cap = std::min<uint32_t>(std::max<uint32_t>(max_iters, 1), 1u << 20);
+  if (g.trace_cap < want_cap) {
+    if (g.d_trace) cudaFree(g.d_trace);
+    g.d_trace = nullptr;
+    g.trace_cap = 0;
+    CKA(cudaMalloc(&g.d_trace, sizeof(TraceRec) * (size_t)want_cap));
+    g.trace_cap = want_cap;
+    for (auto& e : h->exec)  // kernel params captured the old trace pointer
+      if (e) { cudaGraphExecDestroy(e); e = nullptr; }
+  }
+  int rc = ensure_exec(h, a);
+  if (rc) return rc;
+  CKA(cudaMemsetAsync(g.d_trace, 0, sizeof(TraceRec) * (size_t)g.trace_cap, g.stream));
+  CKA(cudaEventRecord(g.ev0, g.stream));
+  CKA(launch_reset_ctl(g.d_ctl, max_iters, g.stream));
+  CKA(launch_init(g, a, source, g.stream));
+  CKA(cudaEventRecord(g.evm, g.stream));
+  if (max_iters > 0) CKA(cudaGraphLaunch(h->exec[a], g.stream));
+  CKA(cudaEventRecord(g.ev1, g.stream));
+  CKA(cudaMemcpyAsync(g.h_ctl, g.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g.stream));
+  CKA(cudaStreamSynchronize(g.stream));
+  float ms = 0, lms = 0;
+  cudaEventElapsedTime(&ms, g.ev0, g.ev1);
+  cudaEventElapsedTime(&lms, g.evm, g.ev1);
+  const Ctl c = *g.h_ctl;
+  // statistics and algorithmic bytes
+  const uint64_t vb = value_bytes(a);
+  const uint64_t evb = alg_needs_edge_values(a) ? 4 : 0;
+  const uint32_t n = std::min(c.iter, g.trace_cap);
+  TraceRec* tr = new TraceRec[n ? n : 1];
+  CKA(cudaMemcpy(tr, g.d_trace, sizeof(TraceRec) * n, cudaMemcpyDeviceToHost));
+  uint64_t bytes = 0;
+  for (uint32_t i = 0; i < n; ++i) {
+    bytes += g.V * vb + (a == kPR ? 4ull * g.V : 0);                 // stages 1+3 reads
+    bytes += (uint64_t)tr[i].updated * vb;                            // stage 3 commits
+    bytes += g.E * (4 + 2 + evb);                                     // stage 2
+    if (g.repr == CUSHA_REPR_CW)
+      bytes += tr[i].wb_entries * 6 + tr[i].wb_stores * 4;            // SrcIndexCW + Mapper, SrcValue
+    else
+      bytes += tr[i].wb_entries * 4 + tr[i].wb_stores * 4 + (uint64_t)tr[i].active_shards * 8ull * g.S;
+  }
+  delete[] tr;
+  g.st.iterations = c.iter;
+  g.st.converged = c.converged;
+  g.st.run_ms = ms;
+  g.st.loop_ms = lms;
+  g.st.last_algorithm = a;
+  g.st.algorithmic_bytes = bytes;
+  g.st.edges_processed = (uint64_t)c.iter * g.E;
+  g.st.stage2_bytes_per_iter = g.E * (4 + 2 + evb);
+  g.st.wb_bytes_all_active = g.repr == CUSHA_REPR_CW ? g.E * 10 : g.E * 8;
+  g.st.device_loop = 1;
+  g.last_alg = a;
+  g.have_values = true;
+  return c.converged ? CUSHA_OK : CUSHA_NOT_CONVERGED;
+}
+
+int cusha_get_values(const cusha_graph* h, void* out, size_t out_bytes) {
+  if (!h || !out) return fail(CUSHA_EINVAL, "null argument");
+  const Graph& g = h->g;
+  if (!g.have_values) return fail(CUSHA_ESTATE, "no run yet");
+  const size_t want = (size_t)g.V * value_bytes(g.last_alg);
+  if (out_bytes != want) return fail(CUSHA_EINVAL, "out_bytes must be |V| * value_bytes(last algorithm)");
+  CKA(cudaSetDevice(g.device));
+  CKA(cudaMemcpyAsync(out, g.d_vv, want, cudaMemcpyDeviceToHost, g.stream));
+  CKA(cudaStreamSynchronize(g.stream));
+  return CUSHA_OK;
+}
+
+int cusha_get_values_device(const cusha_graph* h, void* dptr, size_t out_bytes) {
+  if (!h || !dptr) return fail(CUSHA_EINVAL, "null argument");
+  const Graph& g = h->g;
+  if (!g.have_values) return fail(CUSHA_ESTATE, "no run yet");
+  const size_t want = (size_t)g.V * value_bytes(g.last_alg);
+  if (out_bytes != want) return fail(CUSHA_EINVAL, "out_bytes must be |V| * value_bytes(last algorithm)");
+  CKA(cudaSetDevice(g.device));
+  CKA(cudaMemcpyAsync(dptr, g.d_vv, want, cudaMemcpyDeviceToDevice, g.stream));
+  CKA(cudaStreamSynchronize(g.stream));
+  return CUSHA_OK;
+}
+
+int cusha_get_stats(const cusha_graph* h, cusha_stats* s) {
+  if (!h || !s) return fail(CUSHA_EINVAL, "null argument");
+  *s = h->g.st;
+  return CUSHA_OK;
+}
+
+int cusha_get_trace(const cusha_graph* h, uint32_t* upd, uint32_t* act, uint32_t cap) {
+  if (!h) return fail(CUSHA_EINVAL, "null argument");
+  const Graph& g = h->g;
+  if (!g.have_values || !g.d_trace) return 0;
+  const uint32_t n = std::min(std::min(g.st.iterations, g.trace_cap), cap);
+  if (!n) return 0;
+  TraceRec* tr = new TraceRec[n];
+  cudaSetDevice(g.device);
+  if (cudaMemcpy(tr, g.d_trace, sizeof(TraceRec) * n, cudaMemcpyDeviceToHost) != cudaSuccess) {
+    delete[] tr;
+    return fail(CUSHA_ECUDA, "trace copy");
+  }
+  for (uint32_t i = 0; i < n; ++i) {
+    if (upd) upd[i] = tr[i].updated;
+    if (act) act[i] = tr[i].active_shards;
+  }
+  delete[] tr;
+  return (int)n;
+}
+
+int cusha_get_layout(const cusha_graph* h, cusha_layout_part part, void* out, size_t out_bytes, uint64_t* count) {
+  if (!h) return fail(CUSHA_EINVAL, "graph is NULL");
+  const Graph& g = h->g;
+  const void* src = nullptr;
+  uint64_t n = 0;
+  size_t es = 4;
+  switch (part) {
+    case CUSHA_LAYOUT_SHARD_OFFSETS: src = g.d_shard_off; n = (uint64_t)g.S + 1; break;
+    case CUSHA_LAYOUT_SHARD_SIZES: src = g.d_shard_cnt; n = g.S; break;
+    case CUSHA_LAYOUT_SRC_INDEX: src = g.d_srcidx; n = g.P; break;
+    case CUSHA_LAYOUT_DEST_LOCAL: src = g.d_dest; n = g.P; es = 2; break;
+    case CUSHA_LAYOUT_EDGE_ID: src = g.d_eid; n = g.P; break;
+    case CUSHA_LAYOUT_WINDOWS: src = g.d_win; n = ((uint64_t)g.S + 1) * g.S; break;
+    case CUSHA_LAYOUT_CW_OFFSETS: src = g.d_cw_off; n = (uint64_t)g.S + 1; break;
+    case CUSHA_LAYOUT_CW_SIZES: src = g.d_cw_cnt; n = g.S; break;
+    case CUSHA_LAYOUT_CW_SRC_LOCAL: src = g.d_cw_src; n = g.Q; es = 2; break;
+    case CUSHA_LAYOUT_MAPPER: src = g.d_mapper; n = g.Q; break;
+    case CUSHA_LAYOUT_OUT_DEGREE: src = g.d_outdeg; n = g.V; break;
+    default: return fail(CUSHA_EINVAL, "bad layout part");
+  }
+  if (!src) return fail(CUSHA_EUNSUPPORTED, "part not held by this representation");
+  if (count) *count = n;
+  if (!out) return CUSHA_OK;
+  if (out_bytes < n * es) return fail(CUSHA_EINVAL, "out_bytes too small");
+  CKA(cudaSetDevice(g.device));
+  CKA(cudaMemcpy(out, src, n * es, cudaMemcpyDeviceToHost));
+  return CUSHA_OK;
+}
+
+int cusha_nccl_unique_id(void* out128) {
+  (void)out128;
+  return fail(CUSHA_EUNSUPPORTED, "built without NCCL");
+}
+
+}  // extern "C"

@@ -1,0 +1,355 @@
+// builder.cu — row a0: G-Shards and Concatenated Windows built on the device.
+//
+// PAPER.md §3.1 L119-155 (G-Shards: Partitioned L128, Ordered L129, windows
+// W_ij L155) and §3.2 L175-179 (CW_i = SrcIndex of W_i0..W_i(p-1) in j order,
+// Mapper).  The paper builds on the host and copies the result over PCIe
+// (L457); here the edge list is copied once (12 B/edge) and the layout is
+// produced in HBM by radix sorts (CUB, a library primitive used at setup time
+// only) and a few scatter kernels.
+//
+// G-Shards order = lexicographic (shard(dst), src, dst, input index): one
+// stable radix sort of the packed key (shard(dst) | src | dst mod N) — the
+// input index tie-break (R17) comes from the sort's stability.  CW order =
+// stable sort of the G-Shards positions by source shard (positions inside one
+// source shard are already in (j, position) order, which is exactly W_i0,
+// W_i1, ... concatenated).
+#include <cub/cub.cuh>
+
+#include <string>
+
+#include "common.cuh"
+#include "graph.hpp"
+
+namespace cusha {
+
+namespace {
+
+int bits_for(uint64_t maxval) {  // bits needed to represent 0..maxval
+  int b = 0;
+  while (b < 64 && (1ull << b) <= maxval) ++b;
+  return b;
+}
+
+inline unsigned grid_for(uint64_t n, unsigned block = 256) {
+  uint64_t g = (n + block - 1) / block;
+  const uint64_t cap = 148ull * 64;
+  if (g > cap) g = cap;
+  return (unsigned)(g ? g : 1);
+}
+
+#define GRID_STRIDE(i, n) for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < (n); i += (uint64_t)gridDim.x * blockDim.x)
+
+__global__ void k_make_keys(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst, uint64_t E, uint32_t V,
+                            uint32_t N, int bn, int bsrc, uint64_t* keys, uint32_t* ids, uint32_t* bad) {
+  GRID_STRIDE(e, E) {
+    const uint32_t s = src[e], d = dst[e];
+    if (s >= V || d >= V) {
+      *bad = 1;
+      keys[e] = 0;
+    } else {
+      keys[e] = ((uint64_t)(d / N) << (bsrc + bn)) | ((uint64_t)s << bn) | (uint64_t)(d % N);
+    }
+    ids[e] = (uint32_t)e;
+  }
+}
+
+// start[t] = first sorted index whose (key >> shift) >= t, for t = 0..S
+__global__ void k_starts(const uint64_t* __restrict__ k, uint64_t E, int shift, uint64_t mask, uint32_t S,
+                         uint32_t* start) {
+  GRID_STRIDE(p, E + 1) {
+    const int64_t cur = p < E ? (int64_t)((k[p] >> shift) & mask) : (int64_t)S;
+    const int64_t prev = p == 0 ? -1 : (int64_t)((k[p - 1] >> shift) & mask);
+    for (int64_t t = prev + 1; t <= cur; ++t) start[t] = (uint32_t)p;
+  }
+}
+__global__ void k_starts32(const uint32_t* __restrict__ k, uint64_t E, uint32_t S, uint32_t* start) {
+  GRID_STRIDE(p, E + 1) {
+    const int64_t cur = p < E ? (int64_t)k[p] : (int64_t)S;
+    const int64_t prev = p == 0 ? -1 : (int64_t)k[p - 1];
+    for (int64_t t = prev + 1; t <= cur; ++t) start[t] = (uint32_t)p;
+  }
+}
+
+// cnt[s] = start[s+1]-start[s]; padded[s] = round up to kPad; padded[S] = 0
+__global__ void k_counts(const uint32_t* start, uint32_t S, uint32_t* cnt, uint64_t* padded) {
+  GRID_STRIDE(s, (uint64_t)S + 1) {
+    if (s < S) {
+      const uint32_t c = start[s + 1] - start[s];
+      cnt[s] = c;
+      padded[s] = (uint64_t)((c + kPad - 1) / kPad) * kPad;
+    } else {
+      padded[s] = 0;
+    }
+  }
+}
+__global__ void k_narrow(const uint64_t* in, uint64_t n, uint32_t* out) {
+  GRID_STRIDE(i, n) out[i] = (uint32_t)in[i];
+}
+
+// filler entries of every shard: DestIndex = N (trash slot), no edge
+__global__ void k_fill_shard_pads(const uint32_t* off, const uint32_t* cnt, uint32_t S, uint32_t N, uint16_t* dest,
+                                  uint32_t* srcidx, uint32_t* eid, uint32_t* ev) {
+  GRID_STRIDE(i, (uint64_t)S * kPad) {
+    const uint32_t s = (uint32_t)(i / kPad), r = (uint32_t)(i % kPad);
+    const uint32_t pos = off[s] + cnt[s] + r;
+    if (pos < off[s + 1]) {
+      dest[pos] = (uint16_t)N;
+      srcidx[pos] = 0;
+      eid[pos] = 0xFFFFFFFFu;
+      if (ev) ev[pos] = 0;
+    }
+  }
+}
+
+__global__ void k_scatter_gs(const uint64_t* __restrict__ keys, const uint32_t* __restrict__ ids, uint64_t E,
+                             const uint32_t* start, const uint32_t* off, int bn, int bsrc, const uint32_t* __restrict__ val,
+                             uint16_t* dest, uint32_t* srcidx, uint32_t* eid, uint32_t* ev, uint32_t* pos_of) {
+  const uint64_t mn = (1ull << bn) - 1, ms = (1ull << bsrc) - 1;
+  GRID_STRIDE(p, E) {
+    const uint64_t k = keys[p];
+    const uint32_t sh = (uint32_t)(k >> (bsrc + bn));
+    const uint32_t pp = off[sh] + (uint32_t)(p - start[sh]);
+    dest[pp] = (uint16_t)(k & mn);
+    srcidx[pp] = (uint32_t)((k >> bn) & ms);
+    const uint32_t id = ids[p];
+    eid[pp] = id;
+    if (ev) ev[pp] = val[id];
+    pos_of[p] = pp;
+  }
+}
+
+// window table: win[t*S + j] = first padded position of shard j with SrcIndex >= t*N (t = 0..S)
+__global__ void k_windows(const uint64_t* __restrict__ keys, uint64_t E, const uint32_t* start, const uint32_t* pos_of,
+                          uint32_t N, uint32_t S, int bn, int bsrc, uint32_t* win) {
+  const uint64_t ms = (1ull << bsrc) - 1;
+  GRID_STRIDE(p, E) {
+    const uint64_t k = keys[p];
+    const uint32_t j = (uint32_t)(k >> (bsrc + bn));
+    const int64_t i = (int64_t)(((k >> bn) & ms) / N);
+    const int64_t pi = (p == start[j]) ? -1 : (int64_t)(((keys[p - 1] >> bn) & ms) / N);
+    for (int64_t t = pi + 1; t <= i; ++t) win[(size_t)t * S + j] = pos_of[p];
+  }
+}
+__global__ void k_windows_tail(const uint64_t* __restrict__ keys, const uint32_t* start, const uint32_t* off,
+                               const uint32_t* cnt, uint32_t N, uint32_t S, int bn, int bsrc, uint32_t* win) {
+  const uint64_t ms = (1ull << bsrc) - 1;
+  GRID_STRIDE(j, (uint64_t)S) {
+    int64_t last = -1;
+    if (cnt[j]) last = (int64_t)(((keys[start[j + 1] - 1] >> bn) & ms) / N);
+    const uint32_t end = off[j] + cnt[j];
+    for (int64_t t = last + 1; t <= (int64_t)S; ++t) win[(size_t)t * S + j] = end;
+  }
+}
+
+__global__ void k_outdeg(const uint32_t* __restrict__ src, uint64_t E, uint32_t* outdeg) {
+  GRID_STRIDE(e, E) atomicAdd(&outdeg[src[e]], 1u);
+}
+
+// |CW_i| = sum of out-degrees over shard i's vertex range
+__global__ void k_cw_counts(const uint32_t* outdeg, uint32_t V, uint32_t N, uint32_t* cw_cnt) {
+  const uint32_t i = blockIdx.x;
+  const uint32_t b = i * N, e = min(V, b + N);
+  uint32_t acc = 0;
+  for (uint32_t v = b + threadIdx.x; v < e; v += blockDim.x) acc += outdeg[v];
+  typedef cub::BlockReduce<uint32_t, 256> BR;
+  __shared__ typename BR::TempStorage tmp;
+  acc = BR(tmp).Sum(acc);
+  if (threadIdx.x == 0) cw_cnt[i] = acc;
+}
+
+__global__ void k_src_shard(const uint64_t* __restrict__ keys, uint64_t E, uint32_t N, int bn, int bsrc, uint32_t* ks) {
+  const uint64_t ms = (1ull << bsrc) - 1;
+  GRID_STRIDE(p, E) ks[p] = (uint32_t)(((keys[p] >> bn) & ms) / N);
+}
+
+__global__ void k_scatter_cw(const uint32_t* __restrict__ ks, const uint32_t* __restrict__ pp, uint64_t E,
+                             const uint32_t* cstart, const uint32_t* coff, const uint32_t* srcidx, uint32_t N,
+                             uint16_t* cw_src, uint32_t* mapper) {
+  GRID_STRIDE(q, E) {
+    const uint32_t i = ks[q];
+    const uint32_t pk = coff[i] + (uint32_t)(q - cstart[i]);
+    const uint32_t pos = pp[q];
+    cw_src[pk] = (uint16_t)(srcidx[pos] - i * N);
+    mapper[pk] = pos;
+  }
+}
+__global__ void k_fill_cw_pads(const uint32_t* coff, const uint32_t* ccnt, uint32_t S, uint32_t trash, uint16_t* cw_src,
+                               uint32_t* mapper) {
+  GRID_STRIDE(i, (uint64_t)S * kPad) {
+    const uint32_t s = (uint32_t)(i / kPad), r = (uint32_t)(i % kPad);
+    const uint32_t pos = coff[s] + ccnt[s] + r;
+    if (pos < coff[s + 1]) {
+      cw_src[pos] = 0;
+      mapper[pos] = trash;
+    }
+  }
+}
+
+struct DevBuf {  // RAII temporary
+  void* p = nullptr;
+  ~DevBuf() { if (p) cudaFree(p); }
+};
+
+#define CK(call)                                                                     \
+  do {                                                                               \
+    cudaError_t e_ = (call);                                                         \
+    if (e_ != cudaSuccess) {                                                         \
+      err = std::string(#call) + ": " + cudaGetErrorString(e_);                      \
+      return e_ == cudaErrorMemoryAllocation ? CUSHA_ENOMEM : CUSHA_ECUDA;           \
+    }                                                                                \
+  } while (0)
+
+template <class T>
+cudaError_t dalloc(T** p, uint64_t n) {
+  return cudaMalloc(reinterpret_cast<void**>(p), (n ? n : 1) * sizeof(T));
+}
+
+}  // namespace
+
+int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const uint32_t* d_val, std::string& err) {
+  cudaStream_t st = g.stream;
+  const uint64_t E = g.E;
+  const uint32_t V = g.V, N = g.N, S = g.S;
+  const int bn = bits_for(N - 1) ? bits_for(N - 1) : 1, bsrc = bits_for(V - 1) ? bits_for(V - 1) : 1,
+            bsh = bits_for(S - 1);
+  const int total = bsh + bsrc + bn;
+  if (total > 64) { err = "key does not fit 64 bits"; return CUSHA_EINVAL; }
+
+  DevBuf keys, keys2, ids, ids2, bad, start, padded, temp, pos_of;
+  CK(dalloc((uint64_t**)&keys.p, E));
+  CK(dalloc((uint64_t**)&keys2.p, E));
+  CK(dalloc((uint32_t**)&ids.p, E));
+  CK(dalloc((uint32_t**)&ids2.p, E));
+  CK(dalloc((uint32_t**)&bad.p, 1));
+  CK(cudaMemsetAsync(bad.p, 0, 4, st));
+  if (E) k_make_keys<<<grid_for(E), 256, 0, st>>>(d_src, d_dst, E, V, N, bn, bsrc, (uint64_t*)keys.p, (uint32_t*)ids.p,
+                                                  (uint32_t*)bad.p);
+  CK(cudaGetLastError());
+  uint32_t h_bad = 0;
+  CK(cudaMemcpyAsync(&h_bad, bad.p, 4, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  if (h_bad) { err = "edge endpoint >= num_vertices"; return CUSHA_EINVAL; }
+
+  // ---- G-Shards order
+  cub::DoubleBuffer<uint64_t> kb((uint64_t*)keys.p, (uint64_t*)keys2.p);
+  cub::DoubleBuffer<uint32_t> vb((uint32_t*)ids.p, (uint32_t*)ids2.p);
+  size_t tbytes = 0;
+  if (E) {
+    CK(cub::DeviceRadixSort::SortPairs(nullptr, tbytes, kb, vb, (int64_t)E, 0, total, st));
+    CK(cudaMalloc(&temp.p, tbytes));
+    CK(cub::DeviceRadixSort::SortPairs(temp.p, tbytes, kb, vb, (int64_t)E, 0, total, st));
+  }
+  const uint64_t* K = kb.Current();
+  const uint32_t* I = vb.Current();
+
+  CK(dalloc((uint32_t**)&start.p, (uint64_t)S + 1));
+  CK(dalloc((uint64_t**)&padded.p, (uint64_t)S + 1));
+  CK(dalloc(&g.d_shard_cnt, S));
+  CK(dalloc(&g.d_shard_off, (uint64_t)S + 1));
+  k_starts<<<grid_for(E + 1), 256, 0, st>>>(K, E, bsrc + bn, ~0ull, S,
+                                            (uint32_t*)start.p);
+  k_counts<<<grid_for((uint64_t)S + 1), 256, 0, st>>>((uint32_t*)start.p, S, g.d_shard_cnt, (uint64_t*)padded.p);
+  CK(cudaGetLastError());
+  {
+    DevBuf t2, scan;
+    size_t b2 = 0;
+    CK(dalloc((uint64_t**)&scan.p, (uint64_t)S + 1));
+    CK(cub::DeviceScan::ExclusiveSum(nullptr, b2, (uint64_t*)padded.p, (uint64_t*)scan.p, (int64_t)S + 1, st));
+    CK(cudaMalloc(&t2.p, b2 ? b2 : 1));
+    CK(cub::DeviceScan::ExclusiveSum(t2.p, b2, (uint64_t*)padded.p, (uint64_t*)scan.p, (int64_t)S + 1, st));
+    uint64_t P = 0;
+    CK(cudaMemcpyAsync(&P, (uint64_t*)scan.p + S, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (P >= 0xFFFFFFF0ull) { err = "padded entry count exceeds 32-bit positions"; return CUSHA_EINVAL; }
+    g.P = P;
+    k_narrow<<<grid_for((uint64_t)S + 1), 256, 0, st>>>((uint64_t*)scan.p, (uint64_t)S + 1, g.d_shard_off);
+    CK(cudaGetLastError());
+  }
+  const uint64_t P = g.P;
+  CK(dalloc(&g.d_dest, P));
+  CK(dalloc(&g.d_srcidx, P));
+  CK(dalloc(&g.d_eid, P));
+  if (d_val) { CK(dalloc(&g.d_ev, P)); g.has_ev = true; }
+  CK(dalloc((uint32_t**)&pos_of.p, E));
+  k_fill_shard_pads<<<grid_for((uint64_t)S * kPad), 256, 0, st>>>(g.d_shard_off, g.d_shard_cnt, S, N, g.d_dest,
+                                                                   g.d_srcidx, g.d_eid, g.d_ev);
+  if (E)
+    k_scatter_gs<<<grid_for(E), 256, 0, st>>>(K, I, E, (uint32_t*)start.p, g.d_shard_off, bn, bsrc, d_val, g.d_dest,
+                                              g.d_srcidx, g.d_eid, g.d_ev, (uint32_t*)pos_of.p);
+  CK(cudaGetLastError());
+
+  // ---- window table W_ij (both representations keep it; GS stage 4 reads it)
+  CK(dalloc(&g.d_win, ((uint64_t)S + 1) * S));
+  if (E)
+    k_windows<<<grid_for(E), 256, 0, st>>>(K, E, (uint32_t*)start.p, (uint32_t*)pos_of.p, N, S, bn, bsrc, g.d_win);
+  k_windows_tail<<<grid_for(S), 256, 0, st>>>(K, (uint32_t*)start.p, g.d_shard_off, g.d_shard_cnt, N, S, bn, bsrc,
+                                              g.d_win);
+  CK(cudaGetLastError());
+
+  // ---- out-degrees (PR NbrsNum, L318) and |CW_i|
+  CK(dalloc(&g.d_outdeg, V));
+  CK(cudaMemsetAsync(g.d_outdeg, 0, (size_t)V * 4, st));
+  if (E) k_outdeg<<<grid_for(E), 256, 0, st>>>(d_src, E, g.d_outdeg);
+  CK(dalloc(&g.d_cw_cnt, S));
+  k_cw_counts<<<S, 256, 0, st>>>(g.d_outdeg, V, N, g.d_cw_cnt);
+  CK(cudaGetLastError());
+
+  // ---- Concatenated Windows + Mapper (§3.2)
+  if (g.repr == CUSHA_REPR_CW) {
+    // reuse the key buffers: ks (u32) in keys.Alternate, positions in ids.Alternate
+    uint32_t* ks = reinterpret_cast<uint32_t*>(kb.Alternate());
+    uint32_t* ks2 = ks + E;
+    const int bks = bits_for(S - 1) ? bits_for(S - 1) : 1;
+    if (E) k_src_shard<<<grid_for(E), 256, 0, st>>>(K, E, N, bn, bsrc, ks);
+    CK(cudaGetLastError());
+    cub::DoubleBuffer<uint32_t> kk(ks, ks2);
+    cub::DoubleBuffer<uint32_t> pv((uint32_t*)pos_of.p, vb.Alternate());
+    if (E) {
+      size_t b3 = 0;
+      CK(cub::DeviceRadixSort::SortPairs(nullptr, b3, kk, pv, (int64_t)E, 0, bks, st));
+      if (b3 > tbytes) {
+        cudaFree(temp.p);
+        temp.p = nullptr;
+        CK(cudaMalloc(&temp.p, b3));
+        tbytes = b3;
+      }
+      CK(cub::DeviceRadixSort::SortPairs(temp.p, b3, kk, pv, (int64_t)E, 0, bks, st));
+    }
+    DevBuf cstart, cpad, cscan, t4;
+    CK(dalloc((uint32_t**)&cstart.p, (uint64_t)S + 1));
+    CK(dalloc((uint64_t**)&cpad.p, (uint64_t)S + 1));
+    CK(dalloc((uint64_t**)&cscan.p, (uint64_t)S + 1));
+    k_starts32<<<grid_for(E + 1), 256, 0, st>>>(kk.Current(), E, S, (uint32_t*)cstart.p);
+    DevBuf ccnt;
+    CK(dalloc((uint32_t**)&ccnt.p, S));
+    k_counts<<<grid_for((uint64_t)S + 1), 256, 0, st>>>((uint32_t*)cstart.p, S, (uint32_t*)ccnt.p, (uint64_t*)cpad.p);
+    CK(cudaGetLastError());
+    size_t b4 = 0;
+    CK(cub::DeviceScan::ExclusiveSum(nullptr, b4, (uint64_t*)cpad.p, (uint64_t*)cscan.p, (int64_t)S + 1, st));
+    CK(cudaMalloc(&t4.p, b4 ? b4 : 1));
+    CK(cub::DeviceScan::ExclusiveSum(t4.p, b4, (uint64_t*)cpad.p, (uint64_t*)cscan.p, (int64_t)S + 1, st));
+    uint64_t Q = 0;
+    CK(cudaMemcpyAsync(&Q, (uint64_t*)cscan.p + S, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (Q >= 0xFFFFFFF0ull) { err = "padded CW entry count exceeds 32-bit positions"; return CUSHA_EINVAL; }
+    g.Q = Q;
+    CK(dalloc(&g.d_cw_off, (uint64_t)S + 1));
+    k_narrow<<<grid_for((uint64_t)S + 1), 256, 0, st>>>((uint64_t*)cscan.p, (uint64_t)S + 1, g.d_cw_off);
+    CK(dalloc(&g.d_cw_src, Q));
+    CK(dalloc(&g.d_mapper, Q));
+    k_fill_cw_pads<<<grid_for((uint64_t)S * kPad), 256, 0, st>>>(g.d_cw_off, (uint32_t*)ccnt.p, S, (uint32_t)P,
+                                                                  g.d_cw_src, g.d_mapper);
+    if (E)
+      k_scatter_cw<<<grid_for(E), 256, 0, st>>>(kk.Current(), pv.Current(), E, (uint32_t*)cstart.p, g.d_cw_off,
+                                                g.d_srcidx, N, g.d_cw_src, g.d_mapper);
+    CK(cudaGetLastError());
+    CK(cudaStreamSynchronize(st));
+    // CW keeps the 3-tuple shards + SrcIndexCW + Mapper (L175): no per-entry global SrcIndex
+    cudaFree(g.d_srcidx);
+    g.d_srcidx = nullptr;
+  }
+  CK(cudaStreamSynchronize(st));
+  return CUSHA_OK;
+}
+
+}  // namespace cusha

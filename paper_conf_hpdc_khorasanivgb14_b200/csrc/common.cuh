@@ -1,0 +1,55 @@
+// common.cuh — device helpers shared by the CuSha kernels (product path only).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace cusha {
+
+constexpr uint32_t kInf = 0xFFFFFFFFu;   // DESIGN.md R1 (Table 3 "INF")
+constexpr uint32_t kPad = 8;             // entries per vector chunk: shards / CW_i padded to multiples of 8
+constexpr int kThreads = 512;            // threads per shard CTA (tools/microbench: 512 > 256 for ATOMS)
+
+// ---------------------------------------------------------------- loads
+// SrcValue is written by other CTAs' stage 4 during the same launch (the
+// asynchronous model of L45), so it is read with ld.global.cg (L2, never a
+// possibly stale L1 line and never the non-coherent path).  Topology arrays
+// are read-only for the whole run: non-coherent, no L1 allocation.
+__device__ __forceinline__ uint4 ld_cg_v4(const void* p) {
+  uint4 r;
+  asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ uint4 ld_stream_v4(const void* p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ uint32_t ld_ro(const uint32_t* p) { return __ldg(p); }
+__device__ __forceinline__ void st_u32(uint32_t* p, uint32_t v) {
+  asm volatile("st.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// --------------------------------------------------- 64-bit fixed point
+// Float sums of Table 3 (PR, NN, HS, CS) are accumulated in shared memory as
+// 64-bit two's-complement fixed point with 32 fraction bits, using native
+// 32-bit ATOMS.ADD on a lo word and carrying into a hi word (f32 shared
+// atomicAdd is a CAS loop on sm_100a; u32 add is native).  Integer addition
+// is associative, so the sum is independent of the atomic order
+// (R11: frozen inputs give frozen sums, so PR terminates).
+__device__ __forceinline__ uint64_t f2fix(float x) {
+  return (uint64_t)__float2ll_rn(x * 4294967296.0f);
+}
+__device__ __forceinline__ float fix2f(uint32_t lo, uint32_t hi) {
+  long long v = (long long)(((uint64_t)hi << 32) | lo);
+  return ldexpf(__ll2float_rn(v), -32);
+}
+__device__ __forceinline__ void fix_add(uint32_t* lo, uint32_t* hi, uint64_t F) {
+  uint32_t l = (uint32_t)F, h = (uint32_t)(F >> 32);
+  uint32_t old = atomicAdd(lo, l);
+  h += (old + l < old) ? 1u : 0u;  // carry out of the low word
+  if (h) atomicAdd(hi, h);
+}
+
+}  // namespace cusha

@@ -1,0 +1,112 @@
+// graph.hpp — internal (non-ABI) declarations shared by the library's .cu files.
+#pragma once
+#include <cstddef>
+#include <cstdint>
+#include <string>
+#include <cuda_runtime.h>
+
+#include "../../include/cusha.h"
+
+namespace cusha {
+
+// Iteration control word block (row a5), one per graph, device resident.
+struct Ctl {
+  uint32_t iter;       // shard passes completed in this run
+  uint32_t changed;    // set by any CTA whose stage 3 committed an update (is_converged = false, L255)
+  uint32_t ctas_done;  // arrival counter; the last CTA closes the iteration
+  uint32_t max_iters;
+  uint32_t converged;  // 1 once a pass committed nothing
+  uint32_t pad[3];
+};
+
+// Per-iteration trace (row f4; also the source of algorithmic byte counts).
+struct TraceRec {
+  uint32_t updated;          // vertices committed in stage 3
+  uint32_t active_shards;    // shards that ran stage 4
+  unsigned long long wb_entries;  // CW / window entries visited by stage 4
+  unsigned long long wb_stores;   // SrcValue words actually stored by stage 4
+};
+
+// Everything a shard-pass launch needs (passed by value).
+struct KParams {
+  uint32_t V, N, S, source;
+  const uint32_t* shard_off;   // S+1 padded start positions
+  const uint16_t* dest;        // P local DestIndex (filler = N)
+  const uint32_t* ev;          // P EdgeValue or null
+  uint32_t* srcvalue;          // P+1 (slot P = trash for CW filler)
+  const uint32_t* srcidx;      // GS: P SrcIndex
+  const uint32_t* win;         // GS: (S+1)*S window starts
+  const uint32_t* cw_off;      // CW: S+1 padded CW_i starts
+  const uint32_t* cw_cnt;      // S real |CW_i| (both reprs; = entries stage 4 of shard i visits)
+  const uint16_t* cw_src;      // CW: Q local SrcIndex
+  const uint32_t* mapper;      // CW: Q padded shard positions
+  void* vv;                    // VertexValues
+  const uint32_t* outdeg;      // V out-degrees (PR NbrsNum)
+  Ctl* ctl;
+  TraceRec* trace;
+  uint32_t trace_cap;
+  int use_cond;
+  unsigned long long cond_handle;
+};
+
+struct PassKernel {
+  const void* func;       // __global__ shard_pass<Alg, Repr>
+  uint32_t words;         // shared 32-bit words per vertex (local state)
+  bool wb_array;          // separate write-back value array in shared memory
+  bool monotone;          // changed-bit array in shared memory
+  size_t smem_bytes(uint32_t N) const;
+};
+
+struct Graph {
+  // topology
+  uint32_t V = 0, N = 0, S = 0;
+  uint64_t E = 0, P = 0, Q = 0;
+  int repr = 0, device = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  bool has_ev = false;
+  uint32_t* d_shard_off = nullptr;  // S+1
+  uint32_t* d_shard_cnt = nullptr;  // S
+  uint16_t* d_dest = nullptr;       // P
+  uint32_t* d_srcidx = nullptr;     // P (GS)
+  uint32_t* d_eid = nullptr;        // P
+  uint32_t* d_ev = nullptr;         // P (if has_ev)
+  uint32_t* d_win = nullptr;        // (S+1)*S (GS)
+  uint32_t* d_cw_off = nullptr;     // S+1
+  uint32_t* d_cw_cnt = nullptr;     // S
+  uint16_t* d_cw_src = nullptr;     // Q (CW)
+  uint32_t* d_mapper = nullptr;     // Q (CW)
+  uint32_t* d_outdeg = nullptr;     // V
+  // per-run state
+  uint32_t* d_srcvalue = nullptr;   // P+1
+  void* d_vv = nullptr;             // V * 8 bytes
+  void* d_init[8] = {};             // user initial values per algorithm
+  Ctl* d_ctl = nullptr;
+  TraceRec* d_trace = nullptr;
+  uint32_t trace_cap = 0;
+  Ctl* h_ctl = nullptr;             // pinned mirror
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr, evm = nullptr;
+  // multi-GPU
+  int world_size = 1, rank = 0;
+  // stats
+  cusha_stats st{};
+  int last_alg = -1;
+  bool have_values = false;
+};
+
+// kernels.cu
+const PassKernel& pass_kernel(int alg, int repr);
+cudaError_t launch_init(const Graph& g, int alg, uint32_t source, cudaStream_t s);
+cudaError_t launch_reset_ctl(Ctl* ctl, uint32_t max_iters, cudaStream_t s);
+KParams make_params(const Graph& g, uint32_t source);
+size_t value_bytes(int alg);
+bool alg_needs_edge_values(int alg);
+bool alg_needs_init(int alg);
+
+// builder.cu
+int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const uint32_t* d_val, std::string& err);
+
+// api.cu
+void set_error(const std::string& msg);
+
+}  // namespace cusha
