@@ -217,7 +217,7 @@ def bench_cusha(args):
         ev = torch.from_numpy(wl.edge_u32.view(np.int32)).to(f"cuda:{dev}")
     torch.cuda.synchronize()
     g = cusha.build_graph(wl.V, src_d, dst_d, edge_values=ev, repr=repr_, vertices_per_shard=args.N, device=dev,
-                          stream=stream.cuda_stream)
+                          stream=stream.cuda_stream, host_loop=args.host_loop)
     st0 = cusha.get_stats(g)
     log(f"[bench] built {repr_} |N|={st0['vertices_per_shard']} |S|={st0['num_shards']} in {st0['build_ms']:.1f} ms")
     del src_d, dst_d, ev
@@ -325,6 +325,7 @@ def main():
     ap.add_argument("--N", type=int, default=0, help="vertices per shard (0 = L310 rule)")
     ap.add_argument("--cache-dir", default=None)
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--host-loop", action="store_true", help="host-launched passes (for ncu); default: device loop")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0)

@@ -81,6 +81,10 @@ typedef struct {
   int device;                      /* CUDA device ordinal                                      */
   void* stream;                    /* cudaStream_t to run on; NULL = a library-owned stream    */
   cusha_input_location input_location; /* host (copied in, timed as H2D) or device            */
+  int host_loop;                   /* 0 = loop on the device (CUDA-graph while node, default);
+                                      1 = host launches passes in chunks of 8 (for profilers that
+                                      cannot see kernels inside conditional graphs); passes past
+                                      convergence exit at once, so results are identical      */
   /* Multi-GPU (destination-range partition): */
   int world_size;                  /* 1 = single GPU (0 is treated as 1)                       */
   int rank;                        /* this process's rank, 0..world_size-1                     */
@@ -191,7 +195,7 @@ CUSHA_API int cusha_get_trace(const cusha_graph* g, uint32_t* updated_vertices, 
 typedef enum {
   CUSHA_LAYOUT_SHARD_OFFSETS = 0,   /* u32[|S|+1] first padded position of shard s          */
   CUSHA_LAYOUT_SHARD_SIZES = 1,     /* u32[|S|]   real entries of shard s                   */
-  CUSHA_LAYOUT_SRC_INDEX = 2,       /* u32[P]     SrcIndex (global) per padded entry (GS)   */
+  CUSHA_LAYOUT_SRC_INDEX = 2,       /* u16[P]     SrcIndex - i*|N| (i = source shard; GS)    */
   CUSHA_LAYOUT_DEST_LOCAL = 3,      /* u16[P]     DestIndex - s*|N| (filler = |N|)         */
   CUSHA_LAYOUT_EDGE_ID = 4,         /* u32[P]     input edge index (filler = 0xFFFFFFFF)    */
   CUSHA_LAYOUT_WINDOWS = 5,         /* u32[(|S|+1)*|S|] win[i*|S|+j] = start of W_ij        */

@@ -40,7 +40,7 @@ static int fail(int code, const std::string& msg) {
   } while (0)
 
 static void free_graph_memory(Graph& g) {
-  void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcidx, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
+  void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcloc, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
                   g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_srcvalue, g.d_vv, g.d_ctl, g.d_trace};
   for (void* p : ptrs)
     if (p) cudaFree(p);
@@ -57,7 +57,7 @@ static uint64_t device_bytes(const Graph& g) {
   uint64_t b = 4ull * (g.S + 1) * 2 + 4ull * g.S * 2;  // offsets + counts
   b += 2 * g.P + 4 * g.P;                               // dest + eid
   if (g.has_ev) b += 4 * g.P;
-  if (g.d_srcidx) b += 4 * g.P;
+  if (g.d_srcloc) b += 2 * g.P;
   if (g.d_win) b += 4ull * (g.S + 1) * g.S;
   b += (2 + 4) * g.Q;                                   // CW
   b += 4ull * g.V;                                      // outdeg
@@ -127,6 +127,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   if (!h) return fail(CUSHA_ENOMEM, "host allocation");
   Graph& g = h->g;
   g.V = V; g.E = E; g.N = N; g.S = (V + N - 1) / N; g.repr = (int)o.repr; g.device = o.device;
+  g.host_loop = o.host_loop != 0;
   auto bail = [&](int code) { free_graph_memory(g); delete h; return code; };
   auto cu = [&](cudaError_t e, const char* what) -> int {
     if (e == cudaSuccess) return 0;
@@ -235,6 +236,7 @@ static int ensure_exec(cusha_graph* h, int alg) {
   if (smem > 227 * 1024)
     return fail(CUSHA_EINVAL, "vertices_per_shard too large for this algorithm's shared-memory state");
   CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared));
   cudaGraph_t graph = nullptr;
   CKA(cudaGraphCreate(&graph, 0));
   cudaGraphConditionalHandle handle;
@@ -256,7 +258,7 @@ static int ensure_exec(cusha_graph* h, int alg) {
   cudaKernelNodeParams knp = {};
   knp.func = const_cast<void*>(pk.func);
   knp.gridDim = dim3(g.S);
-  knp.blockDim = dim3(kThreads);
+  knp.blockDim = dim3(pk.threads);
   knp.sharedMemBytes = (unsigned)smem;
   knp.kernelParams = args;
   cudaGraphNode_t kn;
@@ -287,14 +289,37 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     for (auto& e : h->exec)  // kernel params captured the old trace pointer
       if (e) { cudaGraphExecDestroy(e); e = nullptr; }
   }
-  int rc = ensure_exec(h, a);
-  if (rc) return rc;
+  const PassKernel& pk = pass_kernel(a, g.repr);
+  const size_t smem = pk.smem_bytes(g.N);
+  int rc = CUSHA_OK;
+  if (g.host_loop) {
+    if (smem > 227 * 1024)
+      return fail(CUSHA_EINVAL, "vertices_per_shard too large for this algorithm's shared-memory state");
+    CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared));
+  } else {
+    rc = ensure_exec(h, a);
+    if (rc) return rc;
+  }
   CKA(cudaMemsetAsync(g.d_trace, 0, sizeof(TraceRec) * (size_t)g.trace_cap, g.stream));
   CKA(cudaEventRecord(g.ev0, g.stream));
   CKA(launch_reset_ctl(g.d_ctl, max_iters, g.stream));
   CKA(launch_init(g, a, source, g.stream));
   CKA(cudaEventRecord(g.evm, g.stream));
-  if (max_iters > 0) CKA(cudaGraphLaunch(h->exec[a], g.stream));
+  if (max_iters > 0 && !g.host_loop) CKA(cudaGraphLaunch(h->exec[a], g.stream));
+  if (max_iters > 0 && g.host_loop) {
+    // passes launched by the host in chunks; a pass that finds the run
+    // converged (or at max_iters) exits at once, so over-launching is exact
+    KParams kp = make_params(g, source);
+    void* args[] = {&kp};
+    for (;;) {
+      for (int k = 0; k < 8; ++k)
+        CKA(cudaLaunchKernel(pk.func, dim3(g.S), dim3(pk.threads), args, smem, g.stream));
+      CKA(cudaMemcpyAsync(g.h_ctl, g.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g.stream));
+      CKA(cudaStreamSynchronize(g.stream));
+      if (g.h_ctl->converged || g.h_ctl->iter >= max_iters) break;
+    }
+  }
   CKA(cudaEventRecord(g.ev1, g.stream));
   CKA(cudaMemcpyAsync(g.h_ctl, g.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g.stream));
   CKA(cudaStreamSynchronize(g.stream));
@@ -328,7 +353,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   g.st.edges_processed = (uint64_t)c.iter * g.E;
   g.st.stage2_bytes_per_iter = g.E * (4 + 2 + evb);
   g.st.wb_bytes_all_active = g.repr == CUSHA_REPR_CW ? g.E * 10 : g.E * 8;
-  g.st.device_loop = 1;
+  g.st.device_loop = g.host_loop ? 0 : 1;
   g.last_alg = a;
   g.have_values = true;
   return c.converged ? CUSHA_OK : CUSHA_NOT_CONVERGED;
@@ -393,7 +418,7 @@ int cusha_get_layout(const cusha_graph* h, cusha_layout_part part, void* out, si
   switch (part) {
     case CUSHA_LAYOUT_SHARD_OFFSETS: src = g.d_shard_off; n = (uint64_t)g.S + 1; break;
     case CUSHA_LAYOUT_SHARD_SIZES: src = g.d_shard_cnt; n = g.S; break;
-    case CUSHA_LAYOUT_SRC_INDEX: src = g.d_srcidx; n = g.P; break;
+    case CUSHA_LAYOUT_SRC_INDEX: src = g.d_srcloc; n = g.P; es = 2; break;
     case CUSHA_LAYOUT_DEST_LOCAL: src = g.d_dest; n = g.P; es = 2; break;
     case CUSHA_LAYOUT_EDGE_ID: src = g.d_eid; n = g.P; break;
     case CUSHA_LAYOUT_WINDOWS: src = g.d_win; n = ((uint64_t)g.S + 1) * g.S; break;

@@ -88,7 +88,7 @@ __global__ void k_narrow(const uint64_t* in, uint64_t n, uint32_t* out) {
 
 // filler entries of every shard: DestIndex = N (trash slot), no edge
 __global__ void k_fill_shard_pads(const uint32_t* off, const uint32_t* cnt, uint32_t S, uint32_t N, uint16_t* dest,
-                                  uint32_t* srcidx, uint32_t* eid, uint32_t* ev) {
+                                  uint16_t* srcidx, uint32_t* eid, uint32_t* ev) {
   GRID_STRIDE(i, (uint64_t)S * kPad) {
     const uint32_t s = (uint32_t)(i / kPad), r = (uint32_t)(i % kPad);
     const uint32_t pos = off[s] + cnt[s] + r;
@@ -103,14 +103,15 @@ __global__ void k_fill_shard_pads(const uint32_t* off, const uint32_t* cnt, uint
 
 __global__ void k_scatter_gs(const uint64_t* __restrict__ keys, const uint32_t* __restrict__ ids, uint64_t E,
                              const uint32_t* start, const uint32_t* off, int bn, int bsrc, const uint32_t* __restrict__ val,
-                             uint16_t* dest, uint32_t* srcidx, uint32_t* eid, uint32_t* ev, uint32_t* pos_of) {
+                             uint32_t N, uint16_t* dest, uint16_t* srcidx, uint32_t* eid, uint32_t* ev,
+                             uint32_t* pos_of) {
   const uint64_t mn = (1ull << bn) - 1, ms = (1ull << bsrc) - 1;
   GRID_STRIDE(p, E) {
     const uint64_t k = keys[p];
     const uint32_t sh = (uint32_t)(k >> (bsrc + bn));
     const uint32_t pp = off[sh] + (uint32_t)(p - start[sh]);
     dest[pp] = (uint16_t)(k & mn);
-    srcidx[pp] = (uint32_t)((k >> bn) & ms);
+    srcidx[pp] = (uint16_t)(((k >> bn) & ms) % N);  // SrcIndex local to its source shard
     const uint32_t id = ids[p];
     eid[pp] = id;
     if (ev) ev[pp] = val[id];
@@ -163,13 +164,14 @@ __global__ void k_src_shard(const uint64_t* __restrict__ keys, uint64_t E, uint3
 }
 
 __global__ void k_scatter_cw(const uint32_t* __restrict__ ks, const uint32_t* __restrict__ pp, uint64_t E,
-                             const uint32_t* cstart, const uint32_t* coff, const uint32_t* srcidx, uint32_t N,
+                             const uint32_t* cstart, const uint32_t* coff, const uint16_t* srcidx, uint32_t N,
                              uint16_t* cw_src, uint32_t* mapper) {
   GRID_STRIDE(q, E) {
     const uint32_t i = ks[q];
     const uint32_t pk = coff[i] + (uint32_t)(q - cstart[i]);
     const uint32_t pos = pp[q];
-    cw_src[pk] = (uint16_t)(srcidx[pos] - i * N);
+    (void)N;
+    cw_src[pk] = srcidx[pos];  // already SrcIndex - i*N
     mapper[pk] = pos;
   }
 }
@@ -267,15 +269,15 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   }
   const uint64_t P = g.P;
   CK(dalloc(&g.d_dest, P));
-  CK(dalloc(&g.d_srcidx, P));
+  CK(dalloc(&g.d_srcloc, P));
   CK(dalloc(&g.d_eid, P));
   if (d_val) { CK(dalloc(&g.d_ev, P)); g.has_ev = true; }
   CK(dalloc((uint32_t**)&pos_of.p, E));
   k_fill_shard_pads<<<grid_for((uint64_t)S * kPad), 256, 0, st>>>(g.d_shard_off, g.d_shard_cnt, S, N, g.d_dest,
-                                                                   g.d_srcidx, g.d_eid, g.d_ev);
+                                                                   g.d_srcloc, g.d_eid, g.d_ev);
   if (E)
-    k_scatter_gs<<<grid_for(E), 256, 0, st>>>(K, I, E, (uint32_t*)start.p, g.d_shard_off, bn, bsrc, d_val, g.d_dest,
-                                              g.d_srcidx, g.d_eid, g.d_ev, (uint32_t*)pos_of.p);
+    k_scatter_gs<<<grid_for(E), 256, 0, st>>>(K, I, E, (uint32_t*)start.p, g.d_shard_off, bn, bsrc, d_val, N, g.d_dest,
+                                              g.d_srcloc, g.d_eid, g.d_ev, (uint32_t*)pos_of.p);
   CK(cudaGetLastError());
 
   // ---- window table W_ij (both representations keep it; GS stage 4 reads it)
@@ -341,12 +343,12 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
                                                                   g.d_cw_src, g.d_mapper);
     if (E)
       k_scatter_cw<<<grid_for(E), 256, 0, st>>>(kk.Current(), pv.Current(), E, (uint32_t*)cstart.p, g.d_cw_off,
-                                                g.d_srcidx, N, g.d_cw_src, g.d_mapper);
+                                                g.d_srcloc, N, g.d_cw_src, g.d_mapper);
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(st));
-    // CW keeps the 3-tuple shards + SrcIndexCW + Mapper (L175): no per-entry global SrcIndex
-    cudaFree(g.d_srcidx);
-    g.d_srcidx = nullptr;
+    // CW keeps the 3-tuple shards + SrcIndexCW + Mapper (L175): no per-entry SrcIndex in shard order
+    cudaFree(g.d_srcloc);
+    g.d_srcloc = nullptr;
   }
   CK(cudaStreamSynchronize(st));
   return CUSHA_OK;

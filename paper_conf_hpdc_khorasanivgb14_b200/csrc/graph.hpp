@@ -34,7 +34,7 @@ struct KParams {
   const uint16_t* dest;        // P local DestIndex (filler = N)
   const uint32_t* ev;          // P EdgeValue or null
   uint32_t* srcvalue;          // P+1 (slot P = trash for CW filler)
-  const uint32_t* srcidx;      // GS: P SrcIndex
+  const uint16_t* srcloc;      // GS: P SrcIndex - (source shard)*N
   const uint32_t* win;         // GS: (S+1)*S window starts
   const uint32_t* cw_off;      // CW: S+1 padded CW_i starts
   const uint32_t* cw_cnt;      // S real |CW_i| (both reprs; = entries stage 4 of shard i visits)
@@ -54,6 +54,8 @@ struct PassKernel {
   uint32_t words;         // shared 32-bit words per vertex (local state)
   bool wb_array;          // separate write-back value array in shared memory
   bool monotone;          // changed-bit array in shared memory
+  uint32_t ring_bytes;    // TMA tile ring
+  uint32_t threads;       // CTA size (producer warp + consumer warps)
   size_t smem_bytes(uint32_t N) const;
 };
 
@@ -68,7 +70,7 @@ struct Graph {
   uint32_t* d_shard_off = nullptr;  // S+1
   uint32_t* d_shard_cnt = nullptr;  // S
   uint16_t* d_dest = nullptr;       // P
-  uint32_t* d_srcidx = nullptr;     // P (GS)
+  uint16_t* d_srcloc = nullptr;     // P (GS): SrcIndex local to its source shard
   uint32_t* d_eid = nullptr;        // P
   uint32_t* d_ev = nullptr;         // P (if has_ev)
   uint32_t* d_win = nullptr;        // (S+1)*S (GS)
@@ -92,6 +94,7 @@ struct Graph {
   cusha_stats st{};
   int last_alg = -1;
   bool have_values = false;
+  bool host_loop = false;
 };
 
 // kernels.cu

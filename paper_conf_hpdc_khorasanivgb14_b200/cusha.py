@@ -27,7 +27,7 @@ EINVAL, ENOMEM, ECUDA, ENCCL, EUNSUPPORTED, ESTATE = -1, -2, -3, -4, -5, -6
 INF = 0xFFFFFFFF
 
 LAYOUT = {
-    "shard_offsets": (0, np.uint32), "shard_sizes": (1, np.uint32), "src_index": (2, np.uint32),
+    "shard_offsets": (0, np.uint32), "shard_sizes": (1, np.uint32), "src_index": (2, np.uint16),
     "dest_local": (3, np.uint16), "edge_id": (4, np.uint32), "windows": (5, np.uint32),
     "cw_offsets": (6, np.uint32), "cw_sizes": (7, np.uint32), "cw_src_local": (8, np.uint16),
     "mapper": (9, np.uint32), "out_degree": (10, np.uint32),
@@ -42,6 +42,7 @@ class BuildOpts(ctypes.Structure):
         ("device", ctypes.c_int),
         ("stream", ctypes.c_void_p),
         ("input_location", ctypes.c_int),
+        ("host_loop", ctypes.c_int),
         ("world_size", ctypes.c_int),
         ("rank", ctypes.c_int),
         ("nccl_unique_id", ctypes.c_void_p),
@@ -169,7 +170,8 @@ class Graph:
 
 
 def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertices_per_shard: int = 0,
-                smem_bytes_per_vertex: int = 0, device: int = 0, stream: Optional[int] = None) -> Graph:
+                smem_bytes_per_vertex: int = 0, device: int = 0, stream: Optional[int] = None,
+                host_loop: bool = False) -> Graph:
     """cusha_build_graph.  src/dst/edge_values: numpy (host, copied in) or CUDA tensors (device)."""
     on_dev = _is_device(src)
     if not on_dev:
@@ -188,6 +190,7 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
     o.device = device
     o.stream = stream
     o.input_location = INPUT_DEVICE if on_dev else INPUT_HOST
+    o.host_loop = int(host_loop)
     o.world_size = 1
     h = ctypes.c_void_p()
     _check(lib().cusha_build_graph(num_vertices, len(src), _ptr(src), _ptr(dst), _ptr(edge_values),

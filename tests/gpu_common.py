@@ -12,8 +12,9 @@ EPS = 1e-5      # TOLERANCE of Table 3 (R9)
 D = 0.85
 
 
-def gpu_run(alg, V, src, dst, ev=None, repr="gs", N=0, source=0, init=None, max_iters=1 << 20, expect_converged=True):
-    with cusha.build_graph(V, src, dst, edge_values=ev, repr=repr, vertices_per_shard=N) as g:
+def gpu_run(alg, V, src, dst, ev=None, repr="gs", N=0, source=0, init=None, max_iters=1 << 20, expect_converged=True,
+            host_loop=False):
+    with cusha.build_graph(V, src, dst, edge_values=ev, repr=repr, vertices_per_shard=N, host_loop=host_loop) as g:
         if init is not None:
             cusha.set_vertex_values(g, alg, init)
         rc = cusha.run(alg, g, source=source, max_iters=max_iters)

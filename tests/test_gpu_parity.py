@@ -194,7 +194,7 @@ def test_layout_matches_oracle(repr, V, E, N):
     to_unpadded = np.full(int(off[-1]) + 1, -1, np.int64)
     to_unpadded[real] = np.arange(len(real))
     if repr == "gs":
-        np.testing.assert_array_equal(srcidx[real], ref["gs_src"])
+        np.testing.assert_array_equal(srcidx[real].astype(np.int64), ref["gs_src"].astype(np.int64) % N)
     else:
         creal = np.concatenate([np.arange(cw_off[i], cw_off[i] + cw_cnt[i]) for i in range(S)]) if E else np.zeros(0, np.int64)
         np.testing.assert_array_equal(to_unpadded[mapper[creal]], ref["mapper"].astype(np.int64))
@@ -258,3 +258,18 @@ def test_trace_matches_bfs_levels():
     lv = oracle.bfs(V, s, d, 0)
     assert len(upd) == st["iterations"] and upd[-1] == 0 and act[-1] == 0
     assert upd.sum() >= (lv != cusha.INF).sum() - 1
+
+
+@pytest.mark.parametrize("repr", REPRS)
+def test_host_loop_mode_same_results(c1, repr):
+    """host_loop=1 (profiler mode: host-launched passes that early-exit once
+    converged) reaches the same values and the same pass count semantics."""
+    V, s, d, w = c1
+    got, st = gpu_run("sssp", V, s, d, ev=w, repr=repr, N=128, host_loop=True)
+    np.testing.assert_array_equal(got, oracle.sssp(V, s, d, w, 0))
+    assert st["device_loop"] == 0 and st["converged"] == 1
+    x_star, _ = oracle.pagerank(V, s, d, tol=1e-9)
+    got, st = gpu_run("pr", V, s, d, repr=repr, N=128, host_loop=True)
+    pr_check(got, x_star)
+    got, st = gpu_run("bfs", V, s, d, repr=repr, N=128, host_loop=True, max_iters=3, expect_converged=False)
+    assert st["iterations"] == 3 and st["converged"] == 0
