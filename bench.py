@@ -197,6 +197,8 @@ def bench_reference(args):
 def bench_cusha(args):
     import torch
     from paper_conf_hpdc_khorasanivgb14_b200 import cusha
+    if args.lib:  # tuning experiments: a variant build of libcusha.so
+        cusha.LIB_PATH = os.path.abspath(args.lib)
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -326,6 +328,7 @@ def main():
     ap.add_argument("--cache-dir", default=None)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--host-loop", action="store_true", help="host-launched passes (for ncu); default: device loop")
+    ap.add_argument("--lib", default=None, help="alternative libcusha.so (tuning variants)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0)

@@ -41,17 +41,20 @@ def _stale(target: str, deps) -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    os.makedirs(OBJDIR, exist_ok=True)
+def build(force: bool = False, verbose: bool = False, defines=(), out: str = OUT) -> str:
+    """defines / out: tuning experiments build variants (e.g. -DCUSHA_STAGES=4) to another .so."""
+    objdir = OBJDIR if not defines else os.path.join(OBJDIR, "variant_" + "_".join(d.replace("=", "") for d in defines))
+    os.makedirs(objdir, exist_ok=True)
     hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [os.path.join(ROOT, "include", "cusha.h")]
     objs = []
     jobs = []
     for s in SOURCES:
         src = os.path.join(CSRC, s)
-        obj = os.path.join(OBJDIR, s + ".o")
+        obj = os.path.join(objdir, s + ".o")
         objs.append(obj)
         if force or _stale(obj, [src] + hdrs):
-            cmd = [nvcc(), *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]
+            cmd = [nvcc(), *NVCC_FLAGS, *["-D" + d for d in defines], "-I", os.path.join(ROOT, "include"), "-c", src,
+                   "-o", obj]
             jobs.append((s, cmd))
 
     def run(job):
@@ -65,18 +68,21 @@ def build(force: bool = False, verbose: bool = False) -> str:
         for name, log in ex.map(run, jobs):
             if verbose:
                 print(f"== {name}\n{log}")
-            with open(os.path.join(OBJDIR, name + ".ptxas.txt"), "w") as f:
+            with open(os.path.join(objdir, name + ".ptxas.txt"), "w") as f:
                 f.write(log)
-    if force or jobs or not os.path.exists(OUT):
-        tmp = OUT + ".tmp%d" % os.getpid()
+    if force or jobs or not os.path.exists(out):
+        tmp = out + ".tmp%d" % os.getpid()
         cmd = [nvcc(), "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", tmp, *objs,
                "-Xcompiler", "-fPIC", "-cudart", "static"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stderr}")
-        os.replace(tmp, OUT)
-    return OUT
+        os.replace(tmp, out)
+    return out
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    defs = [a[2:] for a in sys.argv[1:] if a.startswith("-D")]
+    outs = [a[6:] for a in sys.argv[1:] if a.startswith("--out=")]
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, defines=defs,
+                out=outs[0] if outs else OUT))

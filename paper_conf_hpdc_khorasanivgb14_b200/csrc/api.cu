@@ -41,7 +41,8 @@ static int fail(int code, const std::string& msg) {
 
 static void free_graph_memory(Graph& g) {
   void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcloc, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
-                  g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_srcvalue, g.d_vv, g.d_ctl, g.d_trace};
+                  g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_srcvalue, g.d_vv, g.d_ctl, g.d_trace,
+                  g.d_active};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (void*& p : g.d_init)
@@ -228,6 +229,19 @@ int cusha_set_vertex_values(cusha_graph* h, cusha_algorithm alg, const void* ini
   return CUSHA_OK;
 }
 
+// Persistent grid of the shard pass: as many CTAs as fit on the device at
+// once (occupancy x SMs), never more than there are shards.
+static uint32_t pass_grid(const Graph& g, const PassKernel& pk, size_t smem) {
+  if (!pk.persistent) return std::max<uint32_t>(g.S, 1);
+  int sms = 148, per_sm = 1;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g.device);
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, pk.func, (int)pk.threads, smem) != cudaSuccess ||
+      per_sm < 1)
+    per_sm = 1;
+  const uint64_t gsz = (uint64_t)sms * (uint64_t)per_sm;
+  return (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(gsz, g.S));
+}
+
 static int ensure_exec(cusha_graph* h, int alg) {
   Graph& g = h->g;
   if (h->exec[alg]) return CUSHA_OK;
@@ -257,7 +271,7 @@ static int ensure_exec(cusha_graph* h, int alg) {
   void* args[] = {&kp};
   cudaKernelNodeParams knp = {};
   knp.func = const_cast<void*>(pk.func);
-  knp.gridDim = dim3(g.S);
+  knp.gridDim = dim3(pass_grid(g, pk, smem));
   knp.blockDim = dim3(pk.threads);
   knp.sharedMemBytes = (unsigned)smem;
   knp.kernelParams = args;
@@ -314,7 +328,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     void* args[] = {&kp};
     for (;;) {
       for (int k = 0; k < 8; ++k)
-        CKA(cudaLaunchKernel(pk.func, dim3(g.S), dim3(pk.threads), args, smem, g.stream));
+        CKA(cudaLaunchKernel(pk.func, dim3(pass_grid(g, pk, smem)), dim3(pk.threads), args, smem, g.stream));
       CKA(cudaMemcpyAsync(g.h_ctl, g.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g.stream));
       CKA(cudaStreamSynchronize(g.stream));
       if (g.h_ctl->converged || g.h_ctl->iter >= max_iters) break;

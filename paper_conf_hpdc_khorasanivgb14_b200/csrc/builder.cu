@@ -296,6 +296,8 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   k_cw_counts<<<S, 256, 0, st>>>(g.d_outdeg, V, N, g.d_cw_cnt);
   CK(cudaGetLastError());
 
+  CK(dalloc(&g.d_active, S));  // stage-4 prefetch predictor of the shard pass
+
   // ---- Concatenated Windows + Mapper (§3.2)
   if (g.repr == CUSHA_REPR_CW) {
     // reuse the key buffers: ks (u32) in keys.Alternate, positions in ids.Alternate

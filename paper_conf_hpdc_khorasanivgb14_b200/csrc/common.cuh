@@ -63,6 +63,20 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
                : "memory");
 }
 
+// named barrier over `count` threads; returns the OR of pred over them
+__device__ __forceinline__ int bar_sync_or(uint32_t id, uint32_t count, int pred) {
+  int r;
+  asm volatile(
+      "{\n .reg .pred p, q;\n setp.ne.s32 p, %1, 0;\n bar.red.or.pred q, %2, %3, p;\n selp.s32 %0, 1, 0, q;\n}\n"
+      : "=r"(r)
+      : "r"(pred), "r"(id), "r"(count)
+      : "memory");
+  return r;
+}
+__device__ __forceinline__ void bar_sync(uint32_t id, uint32_t count) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
+}
+
 // --------------------------------------------------- 64-bit fixed point
 // Float sums of Table 3 (PR, NN, HS, CS) are accumulated in shared memory as
 // 64-bit two's-complement fixed point with 32 fraction bits, using native
@@ -70,8 +84,12 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 // atomicAdd is a CAS loop on sm_100a; u32 add is native).  Integer addition
 // is associative, so the sum is independent of the atomic order
 // (R11: frozen inputs give frozen sums, so PR terminates).
+// x * 2^32 (exact power-of-two scaling) truncated toward zero to a 64-bit
+// two's-complement integer (F2I.S64).  Exact for |x| < 2^31; larger
+// magnitudes saturate (never reached: DESIGN.md R11).  (An integer-shift
+// version was measured slower on B200: tools/tune.)
 __device__ __forceinline__ uint64_t f2fix(float x) {
-  return (uint64_t)__float2ll_rn(x * 4294967296.0f);
+  return (uint64_t)__float2ll_rz(x * 4294967296.0f);
 }
 __device__ __forceinline__ float fix2f(uint32_t lo, uint32_t hi) {
   long long v = (long long)(((uint64_t)hi << 32) | lo);

@@ -16,7 +16,8 @@ struct Ctl {
   uint32_t ctas_done;  // arrival counter; the last CTA closes the iteration
   uint32_t max_iters;
   uint32_t converged;  // 1 once a pass committed nothing
-  uint32_t pad[3];
+  uint32_t next_shard; // dynamic shard queue of the persistent pass
+  uint32_t pad[2];
 };
 
 // Per-iteration trace (row f4; also the source of algorithmic byte counts).
@@ -38,6 +39,7 @@ struct KParams {
   const uint32_t* win;         // GS: (S+1)*S window starts
   const uint32_t* cw_off;      // CW: S+1 padded CW_i starts
   const uint32_t* cw_cnt;      // S real |CW_i| (both reprs; = entries stage 4 of shard i visits)
+  uint8_t* active;             // S: shard ran stage 4 in the previous pass (stage-4 prefetch predictor)
   const uint16_t* cw_src;      // CW: Q local SrcIndex
   const uint32_t* mapper;      // CW: Q padded shard positions
   void* vv;                    // VertexValues
@@ -56,6 +58,7 @@ struct PassKernel {
   bool monotone;          // changed-bit array in shared memory
   uint32_t ring_bytes;    // TMA tile ring
   uint32_t threads;       // CTA size (producer warp + consumer warps)
+  bool persistent;        // grid = resident CTAs pulling shards from a queue (else one CTA per shard)
   size_t smem_bytes(uint32_t N) const;
 };
 
@@ -76,6 +79,8 @@ struct Graph {
   uint32_t* d_win = nullptr;        // (S+1)*S (GS)
   uint32_t* d_cw_off = nullptr;     // S+1
   uint32_t* d_cw_cnt = nullptr;     // S
+  uint8_t* d_active = nullptr;      // S: stage-4 prefetch predictor
+  uint32_t grid = 0;                // persistent CTAs of the shard pass
   uint16_t* d_cw_src = nullptr;     // Q (CW)
   uint32_t* d_mapper = nullptr;     // Q (CW)
   uint32_t* d_outdeg = nullptr;     // V

@@ -1,18 +1,23 @@
 // kernels.cu — the shard pass (rows a1-a5) and its initialisation kernels.
 //
-// One launch = one CuSha iteration (Fig. 5): one CTA per shard
-// (L191), four stages separated by block barriers, and the global
-// convergence flag (L189, L255).  The iteration loop itself stays on the
+// One launch = one CuSha iteration (Fig. 5): every shard runs the
+// four stages once (L191), then the global convergence flag decides whether
+// another iteration follows (L189, L255).  The iteration loop stays on the
 // device: the last CTA to finish closes the iteration and sets the CUDA-graph
 // while-condition, instead of the paper's
 // per-iteration cudaMemcpy of is_converged (L189).
 //
-// B200 structure of a CTA: one producer warp drives the TMA engine
-// (cp.async.bulk) to stream the shard's entry arrays — and, in stage 4, the
-// CW_s index arrays — through a ring of kStages shared-memory tiles guarded
-// by mbarriers; eight consumer warps reduce from / scatter out of the ring.
-// The memory system thus sees kStages tiles in flight per CTA regardless of
-// how long the consumers' shared-memory atomics take.
+// B200 structure: a persistent grid (a few CTAs per
+// SM).  In each CTA one producer thread takes shards from a global queue in
+// shard order and streams, with the TMA engine (cp.async.bulk), every tile
+// the CTA will consume — the shard's entries for stage 2 and, for CW, the
+// CW_s index arrays for stage 4 — through a ring of shared-memory slots
+// guarded by mbarriers, running ahead across stage and shard boundaries.
+// Eight consumer warps run the paper's stages on one shard at a time
+// (local_vertices in shared memory, as in Fig. 5), taking tiles from the
+// ring.  Stage-4 tiles are prefetched when the shard was active in the
+// previous pass (a misprediction only costs bandwidth: an unpredicted active
+// shard reads its index arrays directly, a predicted inactive one drops them).
 #include <cstdio>
 
 #include "algorithms.cuh"
@@ -21,11 +26,36 @@
 namespace cusha {
 
 constexpr uint32_t kFull = 0xFFFFFFFFu;
-constexpr uint32_t kConsumerWarps = 8;
+// tuning constants (tools/tune: variants are built with -DCUSHA_*)
+#ifndef CUSHA_CONSUMER_WARPS
+#define CUSHA_CONSUMER_WARPS 8
+#endif
+#ifndef CUSHA_STAGES
+#define CUSHA_STAGES 4
+#endif
+#ifndef CUSHA_TILE
+#define CUSHA_TILE 1024
+#endif
+#ifndef CUSHA_PERSISTENT
+#define CUSHA_PERSISTENT 1
+#endif
+#ifndef CUSHA_MIN_BLOCKS
+#define CUSHA_MIN_BLOCKS 2
+#endif
+constexpr bool kPersistent = CUSHA_PERSISTENT != 0;  // grid = resident CTAs (queue) vs one CTA per shard
+#ifndef CUSHA_VB
+#define CUSHA_VB 8
+#endif
+#ifndef CUSHA_SPEC
+#define CUSHA_SPEC 1
+#endif
+constexpr uint32_t kVB = CUSHA_VB;                   // vertex loads in flight per thread in stages 1 and 3
+constexpr uint32_t kConsumerWarps = CUSHA_CONSUMER_WARPS;
 constexpr uint32_t kConsumers = kConsumerWarps * 32;
 constexpr uint32_t kPassThreads = kConsumers + 32;  // + 1 producer warp
-constexpr uint32_t kTile = 1024;                    // entries per ring slot
-constexpr uint32_t kStages = 4;                     // ring depth
+constexpr uint32_t kTile = CUSHA_TILE;              // entries per ring slot
+constexpr uint32_t kStages = CUSHA_STAGES;          // ring depth
+constexpr uint32_t kConsumerBar = 1;                // named barrier of the consumer warps
 
 // ring slot: stage 2 = SrcValue (4T) | DestIndex (2T) | EdgeValue (4T);
 //            stage 4 = SrcIndexCW (2T) | Mapper (4T)
@@ -33,6 +63,12 @@ template <class A>
 constexpr uint32_t slot_bytes() {
   return kTile * (6 + (A::kEdge ? 4 : 0));
 }
+
+enum : uint32_t { kDescStage2 = 0, kDescStage4 = 1, kDescDone = 2 };
+enum : uint32_t { kFlagLast = 1, kFlagSpec4 = 2 };
+struct __align__(16) TileDesc {
+  uint32_t shard, kind, n, flags;  // flags: kFlagLast = last tile of this stage; kFlagSpec4 (on a shard's
+};                                 // first tile) = stage-4 tiles of this shard follow its stage-2 tiles
 
 // ------------------------------------------------------------ stage 2 body
 template <class A>
@@ -122,66 +158,134 @@ __device__ __forceinline__ void gs_walk(const KParams& p, uint32_t s, uint32_t l
   }
 }
 
+// ------------------------------------------------------------ producer
+// Per shard: its stage-2 tiles, then — for CW — its stage-4 tiles, either
+// right away (shard predicted active: prefetch overlaps stage 3) or once the
+// consumers' stage 3 has decided values_updated (decide_bar / s_any).
 template <class A, int REPR>
-__global__ void __launch_bounds__(kPassThreads, 2) shard_pass(const KParams p) {
+__device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDesc* desc, uint64_t* full_bar,
+                                         uint64_t* empty_bar, uint64_t* decide_bar, const volatile int* s_any) {
+  constexpr uint32_t SLOT = slot_bytes<A>();
+  uint32_t slot = 0, ph = 0, dph = 0;
+  auto push = [&](uint32_t shard, uint32_t kind, uint32_t n, uint32_t flags, const void* g0, uint32_t b0,
+                  const void* g1, uint32_t o1, uint32_t b1, const void* g2, uint32_t o2, uint32_t b2) {
+    mbar_wait(&empty_bar[slot], ph ^ 1);
+    desc[slot] = TileDesc{shard, kind, n, flags};
+    uint8_t* buf = ring + slot * SLOT;
+    const uint32_t bytes = b0 + b1 + b2;
+    if (bytes) {
+      mbar_expect_tx(&full_bar[slot], bytes);
+      if (b0) bulk_g2s(buf, g0, b0, &full_bar[slot]);
+      if (b1) bulk_g2s(buf + o1, g1, b1, &full_bar[slot]);
+      if (b2) bulk_g2s(buf + o2, g2, b2, &full_bar[slot]);
+    } else {
+      mbar_arrive(&full_bar[slot]);
+    }
+    if (++slot == kStages) { slot = 0; ph ^= 1; }
+  };
+  for (uint32_t round = 0;; ++round) {
+    // persistent grid: shards from the global queue; otherwise CTA b runs shard b only
+    const uint32_t s = kPersistent ? atomicAdd(&p.ctl->next_shard, 1u) : (round == 0 ? blockIdx.x : p.S);
+    if (s >= p.S) {
+      push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
+      return;
+    }
+    const bool spec = CUSHA_SPEC && REPR == CUSHA_REPR_CW && p.active[s];
+    const uint32_t b = p.shard_off[s], e = p.shard_off[s + 1];
+    if (b == e) push(s, kDescStage2, 0, kFlagLast | (spec ? kFlagSpec4 : 0u), nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
+    for (uint32_t t0 = b; t0 < e; t0 += kTile) {
+      const uint32_t n = min(kTile, e - t0);
+      const uint32_t flags = (t0 + n >= e ? kFlagLast : 0u) | (t0 == b && spec ? kFlagSpec4 : 0u);
+      push(s, kDescStage2, n, flags, p.srcvalue + t0, n * 4, p.dest + t0, 4 * kTile, n * 2,
+           A::kEdge ? (const void*)(p.ev + t0) : nullptr, 6 * kTile, A::kEdge ? n * 4 : 0u);
+    }
+    bool send4 = spec;
+    if (REPR == CUSHA_REPR_CW && !spec) {
+      mbar_wait(decide_bar, dph);  // consumers finished stage 3 of shard s
+      dph ^= 1;
+      send4 = *s_any != 0;
+    }
+    if (send4) {
+      const uint32_t kb = p.cw_off[s], ke = p.cw_off[s + 1];
+      if (kb == ke) push(s, kDescStage4, 0, kFlagLast, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
+      for (uint32_t k0 = kb; k0 < ke; k0 += kTile) {
+        const uint32_t n = min(kTile, ke - k0);
+        push(s, kDescStage4, n, k0 + n >= ke ? kFlagLast : 0u, p.cw_src + k0, n * 2, p.mapper + k0, 2 * kTile,
+             n * 4, nullptr, 0, 0);
+      }
+    }
+  }
+}
+
+template <class A, int REPR>
+__global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(const KParams p) {
   extern __shared__ __align__(128) uint8_t dyn[];
   constexpr uint32_t SLOT = slot_bytes<A>();
   uint8_t* const ring = dyn;
   uint32_t* const sm = reinterpret_cast<uint32_t*>(dyn + kStages * SLOT);
-  __shared__ uint64_t full_bar[kStages], empty_bar[kStages];
+  __shared__ uint64_t full_bar[kStages], empty_bar[kStages], decide_bar;
+  __shared__ TileDesc desc[kStages];
   __shared__ uint32_t s_upd;
+  __shared__ int s_any;
   __shared__ unsigned long long s_stores;
   using V_t = typename A::Value;
   const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
-  const uint32_t s = blockIdx.x, N = p.N, st = N + 1;
-  const uint32_t off = s * N;
-  const uint32_t nv = min(N, p.V - off);
-  V_t* vv = reinterpret_cast<V_t*>(p.vv) + off;
-  uint32_t* aux = sm + A::kWords * st;  // write-back values (float algs) or changed bits (integer algs)
+  const uint32_t N = p.N, st = N + 1;
+  uint32_t* const aux = sm + A::kWords * st;  // write-back values (float algs) or changed bits (integer algs)
   const uint32_t it = *reinterpret_cast<volatile uint32_t*>(&p.ctl->iter);
   // a pass launched after the run converged / hit max_iters is a no-op (host-loop mode)
   if (*reinterpret_cast<volatile uint32_t*>(&p.ctl->converged) || it >= p.ctl->max_iters) return;
   if (tid == 0) {
-    s_upd = 0;
-    s_stores = 0;
     for (uint32_t i = 0; i < kStages; ++i) {
-      mbar_init(&full_bar[i], 1);                // the producer's arrive.expect_tx
+      mbar_init(&full_bar[i], 1);                // the producer's arrive(.expect_tx)
       mbar_init(&empty_bar[i], kConsumerWarps);  // one arrive per consumer warp
     }
+    mbar_init(&decide_bar, 1);  // stage-3 decision of a non-prefetched CW shard
     mbar_fence_init();
   }
-
-  // ---- stage 1: local_vertices <- init_compute(VertexValues) (Fig. 5 lines 8-10, L267)
-  for (uint32_t v = tid; v < nv; v += kPassThreads) A::init(sm, st, v, vv[v]);
-  if (tid == 0) A::init(sm, st, N, V_t{});  // trash slot for filler entries
   __syncthreads();
 
-  // ring position: the producer lane and every consumer thread walk the same tile sequence
-  uint32_t slot = 0, ph = 0;
-  const uint32_t ct = tid - 32;  // consumer thread index (warps 1..8)
+  if (warp == 0) {
+    if (lane == 0) producer<A, REPR>(p, ring, desc, full_bar, empty_bar, &decide_bar, &s_any);
+  } else {
+    const uint32_t ct = tid - 32, cwarp = warp - 1;  // consumer thread / warp index
+    uint32_t slot = 0, ph = 0;
+    for (;;) {
+      mbar_wait(&full_bar[slot], ph);
+      TileDesc d = desc[slot];
+      if (d.kind == kDescDone) break;
+      const uint32_t s = d.shard;
+      const bool spec4 = d.flags & kFlagSpec4;
+      const uint32_t off = s * N;
+      const uint32_t nv = min(N, p.V - off);
+      V_t* vv = reinterpret_cast<V_t*>(p.vv) + off;
 
-  // ---- stage 2: stream the shard's entries, compute() into shared memory (lines 12-13, L269)
-  {
-    const uint32_t b = p.shard_off[s], e = p.shard_off[s + 1];
-    if (warp == 0) {
-      if (lane == 0) {
-        for (uint32_t t0 = b; t0 < e; t0 += kTile) {
-          const uint32_t n = min(kTile, e - t0);
-          mbar_wait(&empty_bar[slot], ph ^ 1);
-          uint8_t* buf = ring + slot * SLOT;
-          mbar_expect_tx(&full_bar[slot], n * (A::kEdge ? 10u : 6u));
-          bulk_g2s(buf, p.srcvalue + t0, n * 4, &full_bar[slot]);
-          bulk_g2s(buf + 4 * kTile, p.dest + t0, n * 2, &full_bar[slot]);
-          if (A::kEdge) bulk_g2s(buf + 6 * kTile, p.ev + t0, n * 4, &full_bar[slot]);
-          if (++slot == kStages) { slot = 0; ph ^= 1; }
+      // ---- stage 1: local_vertices <- init_compute(VertexValues) (Fig. 5 lines 8-10, L267)
+      // (kVB loads in flight per thread before any is used)
+      for (uint32_t base = 0; base < nv; base += kVB * kConsumers) {
+        V_t x[kVB];
+#pragma unroll
+        for (uint32_t u = 0; u < kVB; ++u) {
+          const uint32_t v = base + u * kConsumers + ct;
+          if (v < nv) x[u] = vv[v];
+        }
+#pragma unroll
+        for (uint32_t u = 0; u < kVB; ++u) {
+          const uint32_t v = base + u * kConsumers + ct;
+          if (v < nv) A::init(sm, st, v, x[u]);
         }
       }
-    } else {
-      for (uint32_t t0 = b; t0 < e; t0 += kTile) {
-        const uint32_t n = min(kTile, e - t0);
-        mbar_wait(&full_bar[slot], ph);
+      if (ct == 0) {
+        A::init(sm, st, N, V_t{});  // trash slot for filler entries
+        s_upd = 0;
+        s_stores = 0;
+      }
+      bar_sync(kConsumerBar, kConsumers);
+
+      // ---- stage 2: the shard's entries from the ring, compute() into shared memory (lines 12-13, L269)
+      for (;;) {
         const uint8_t* buf = ring + slot * SLOT;
-        for (uint32_t i = ct * 4; i < n; i += kConsumers * 4) {
+        for (uint32_t i = ct * 4; i < d.n; i += kConsumers * 4) {
           const uint4 sv = *reinterpret_cast<const uint4*>(buf + 4 * i);
           const uint2 dd = *reinterpret_cast<const uint2*>(buf + 4 * kTile + 2 * i);
           uint4 ev = make_uint4(0, 0, 0, 0);
@@ -191,95 +295,109 @@ __global__ void __launch_bounds__(kPassThreads, 2) shard_pass(const KParams p) {
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty_bar[slot]);
         if (++slot == kStages) { slot = 0; ph ^= 1; }
+        if (d.flags & kFlagLast) break;
+        mbar_wait(&full_bar[slot], ph);
+        d = desc[slot];
+      }
+      bar_sync(kConsumerBar, kConsumers);
+
+      // ---- stage 3: update_condition, commit to VertexValues, values_updated (lines 15-20, L271)
+      uint32_t my_upd = 0;
+      for (uint32_t base = 0; base < nv; base += kVB * kConsumers) {
+        V_t x[kVB];
+        uint32_t od[kVB];
+#pragma unroll
+        for (uint32_t u = 0; u < kVB; ++u) {
+          const uint32_t v = base + u * kConsumers + ct;
+          od[u] = 0;
+          if (v < nv) {
+            x[u] = vv[v];
+            if (A::kOutDeg) od[u] = __ldg(p.outdeg + off + v);
+          }
+        }
+#pragma unroll
+        for (uint32_t u = 0; u < kVB; ++u) {
+          const uint32_t v = base + u * kConsumers + ct;
+          bool up = false;
+          if (v < nv) {
+            V_t out;
+            uint32_t wbv = 0;
+            up = A::update(sm, st, v, x[u], &out, &wbv, od[u]);
+            if (up) vv[v] = out;
+            if (!A::kMonotone) aux[v] = wbv;
+          }
+          const uint32_t m = __ballot_sync(kFull, up);
+          if (lane == 0 && m) atomicAdd(&s_upd, (uint32_t)__popc(m));
+          const uint32_t w0 = base + u * kConsumers + cwarp * 32;
+          if (A::kMonotone && lane == 0 && w0 < nv) aux[w0 >> 5] = m;
+          my_upd |= up ? 1u : 0u;
+        }
+      }
+      const int any = bar_sync_or(kConsumerBar, kConsumers, (int)my_upd);
+
+      // ---- stage 4: write-back into every shard's window (lines 23-26, L308)
+      uint32_t stores = 0;
+      if (REPR == CUSHA_REPR_CW) {
+        // thread per CW_s entry: SrcValue[Mapper[k]] = local[SrcIndex[k]] (L177, Fig. 4b);
+        // consecutive threads take consecutive entries, so the stores of one
+        // window (consecutive Mapper targets) coalesce into whole sectors
+        const uint32_t trash = p.shard_off[p.S];
+        if (!spec4 && ct == 0) {  // tell the producer whether CW_s's tiles are needed
+          s_any = any;
+          mbar_arrive(&decide_bar);
+        }
+        if (spec4 || any) {
+          for (;;) {
+            mbar_wait(&full_bar[slot], ph);
+            d = desc[slot];
+            if (any) {
+              const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
+              const uint32_t* M = reinterpret_cast<const uint32_t*>(ring + slot * SLOT + 2 * kTile);
+              for (uint32_t i = ct; i < d.n; i += kConsumers) {
+                const uint32_t m = M[i];
+                uint32_t val;
+                if (m != trash && wb_get<A>(sm, aux, L[i], val)) { st_u32(p.srcvalue + m, val); ++stores; }
+              }
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty_bar[slot]);
+            if (++slot == kStages) { slot = 0; ph ^= 1; }
+            if (d.flags & kFlagLast) break;
+          }
+        }
+      } else if (any) {
+        // G-Shards: windows W_sj of every shard j (L151, Fig. 3c), walked a
+        // batch of 32 windows per warp with one entry per lane (gs_walk)
+        gs_walk(p, s, lane, cwarp, kConsumerWarps, [&](uint32_t e, uint32_t l) {
+          uint32_t val;
+          if (wb_get<A>(sm, aux, l, val)) { st_u32(p.srcvalue + e, val); ++stores; }
+        });
+      }
+#pragma unroll
+      for (int o = 16; o; o >>= 1) stores += __shfl_xor_sync(kFull, stores, o);
+      if (lane == 0 && stores) atomicAdd(&s_stores, (unsigned long long)stores);
+      bar_sync(kConsumerBar, kConsumers);
+
+      // ---- per-shard bookkeeping: convergence flag (line 26), predictor, trace
+      if (ct == 0) {
+        p.active[s] = any ? 1 : 0;
+        if (any) {
+          *reinterpret_cast<volatile uint32_t*>(&p.ctl->changed) = 1u;
+          if (it < p.trace_cap) {
+            TraceRec* t = p.trace + it;
+            atomicAdd(&t->updated, s_upd);
+            atomicAdd(&t->active_shards, 1u);
+            atomicAdd(&t->wb_entries, (unsigned long long)p.cw_cnt[s]);
+            atomicAdd(&t->wb_stores, s_stores);
+          }
+        }
       }
     }
   }
   __syncthreads();
 
-  // ---- stage 3: update_condition, commit to VertexValues, values_updated (lines 15-20, L271)
-  uint32_t my_upd = 0;
-  for (uint32_t base = 0; base < nv; base += kPassThreads) {
-    const uint32_t v = base + tid;
-    bool u = false;
-    if (v < nv) {
-      V_t out;
-      uint32_t wbv = 0;
-      const uint32_t od = A::kOutDeg ? __ldg(p.outdeg + off + v) : 0u;
-      u = A::update(sm, st, v, vv[v], &out, &wbv, od);
-      if (u) vv[v] = out;
-      if (!A::kMonotone) aux[v] = wbv;
-    }
-    const uint32_t m = __ballot_sync(kFull, u);
-    if (lane == 0 && m) atomicAdd(&s_upd, (uint32_t)__popc(m));
-    if (A::kMonotone && lane == 0 && base + warp * 32 < nv) aux[(base >> 5) + warp] = m;
-    my_upd |= u ? 1u : 0u;
-  }
-  const int any = __syncthreads_or((int)my_upd);
-
-  // ---- stage 4: write-back into every shard's window (lines 23-26, L308)
-  if (any) {
-    uint32_t stores = 0;
-    if (REPR == CUSHA_REPR_CW) {
-      // thread per CW_s entry: SrcValue[Mapper[k]] = local[SrcIndex[k]] (L177,
-      // Fig. 4b).  CW_s's index arrays stream through the ring; consecutive
-      // consumer threads take consecutive entries, so the stores of one window
-      // (consecutive Mapper targets) coalesce into whole sectors.
-      const uint32_t kb = p.cw_off[s], ke = p.cw_off[s + 1];
-      const uint32_t trash = p.shard_off[p.S];
-      if (warp == 0) {
-        if (lane == 0) {
-          for (uint32_t k0 = kb; k0 < ke; k0 += kTile) {
-            const uint32_t n = min(kTile, ke - k0);
-            mbar_wait(&empty_bar[slot], ph ^ 1);
-            uint8_t* buf = ring + slot * SLOT;
-            mbar_expect_tx(&full_bar[slot], n * 6u);
-            bulk_g2s(buf, p.cw_src + k0, n * 2, &full_bar[slot]);
-            bulk_g2s(buf + 2 * kTile, p.mapper + k0, n * 4, &full_bar[slot]);
-            if (++slot == kStages) { slot = 0; ph ^= 1; }
-          }
-        }
-      } else {
-        for (uint32_t k0 = kb; k0 < ke; k0 += kTile) {
-          const uint32_t n = min(kTile, ke - k0);
-          mbar_wait(&full_bar[slot], ph);
-          const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
-          const uint32_t* M = reinterpret_cast<const uint32_t*>(ring + slot * SLOT + 2 * kTile);
-          for (uint32_t i = ct; i < n; i += kConsumers) {
-            const uint32_t m = M[i];
-            uint32_t val;
-            if (m != trash && wb_get<A>(sm, aux, L[i], val)) { st_u32(p.srcvalue + m, val); ++stores; }
-          }
-          __syncwarp();
-          if (lane == 0) mbar_arrive(&empty_bar[slot]);
-          if (++slot == kStages) { slot = 0; ph ^= 1; }
-        }
-      }
-    } else if (warp > 0) {
-      // G-Shards: windows W_sj of every shard j (L151, Fig. 3c), walked a
-      // batch of 32 windows per warp with one entry per lane (gs_walk)
-      gs_walk(p, s, lane, warp - 1, kConsumerWarps, [&](uint32_t e, uint32_t l) {
-        uint32_t val;
-        if (wb_get<A>(sm, aux, l, val)) { st_u32(p.srcvalue + e, val); ++stores; }
-      });
-    }
-#pragma unroll
-    for (int o = 16; o; o >>= 1) stores += __shfl_xor_sync(kFull, stores, o);
-    if (lane == 0 && stores) atomicAdd(&s_stores, (unsigned long long)stores);
-    __syncthreads();
-  }
-
-  // ---- convergence flag and iteration close (line 26 "is_converged = false"; L189)
+  // ---- iteration close (L189): the last CTA to finish decides whether another pass follows
   if (tid == 0) {
-    if (any) {
-      *reinterpret_cast<volatile uint32_t*>(&p.ctl->changed) = 1u;
-      if (it < p.trace_cap) {
-        TraceRec* t = p.trace + it;
-        atomicAdd(&t->updated, s_upd);
-        atomicAdd(&t->active_shards, 1u);
-        atomicAdd(&t->wb_entries, (unsigned long long)p.cw_cnt[s]);
-        atomicAdd(&t->wb_stores, s_stores);
-      }
-    }
     __threadfence();
     const uint32_t t = atomicAdd(&p.ctl->ctas_done, 1u);
     if (t == gridDim.x - 1) {
@@ -289,6 +407,7 @@ __global__ void __launch_bounds__(kPassThreads, 2) shard_pass(const KParams p) {
       p.ctl->iter = nit;
       p.ctl->changed = 0;
       p.ctl->ctas_done = 0;
+      p.ctl->next_shard = 0;
       p.ctl->converged = changed ? 0u : 1u;
       __threadfence();
       if (p.use_cond) cudaGraphSetConditional(p.cond_handle, (changed && nit < p.ctl->max_iters) ? 1u : 0u);
@@ -297,7 +416,8 @@ __global__ void __launch_bounds__(kPassThreads, 2) shard_pass(const KParams p) {
 }
 
 // ------------------------------------------------------------ init kernels
-// VertexValues <- Table-3 start state (L327) or the user's initial values.
+// VertexValues <- Table-3 start state (L327) or the user's initial values;
+// every shard predicted active for the first pass.
 template <class A>
 __global__ void init_vertex_values(const KParams p, const void* user) {
   using V_t = typename A::Value;
@@ -305,6 +425,8 @@ __global__ void init_vertex_values(const KParams p, const void* user) {
   const V_t* u = reinterpret_cast<const V_t*>(user);
   for (size_t v = blockIdx.x * (size_t)blockDim.x + threadIdx.x; v < p.V; v += (size_t)gridDim.x * blockDim.x)
     vv[v] = u ? u[v] : A::start((uint32_t)v, p.source);
+  for (size_t s = blockIdx.x * (size_t)blockDim.x + threadIdx.x; s < p.S; s += (size_t)gridDim.x * blockDim.x)
+    p.active[s] = 1;
 }
 
 // SrcValue[e] <- VertexValues[SrcIndex[e]] for every entry (R20: a full
@@ -338,6 +460,7 @@ __global__ void reset_ctl(Ctl* ctl, uint32_t max_iters) {
   ctl->ctas_done = 0;
   ctl->max_iters = max_iters;
   ctl->converged = 0;
+  ctl->next_shard = 0;
 }
 
 // -------------------------------------------------------------- dispatch
@@ -357,6 +480,7 @@ static PassKernel make_pk() {
   k.monotone = A::kMonotone;
   k.ring_bytes = kStages * slot_bytes<A>();
   k.threads = kPassThreads;
+  k.persistent = kPersistent;
   return k;
 }
 
@@ -378,7 +502,7 @@ KParams make_params(const Graph& g, uint32_t source) {
   KParams p{};
   p.V = g.V; p.N = g.N; p.S = g.S; p.source = source;
   p.shard_off = g.d_shard_off; p.dest = g.d_dest; p.ev = g.d_ev; p.srcvalue = g.d_srcvalue;
-  p.srcloc = g.d_srcloc; p.win = g.d_win; p.cw_off = g.d_cw_off; p.cw_cnt = g.d_cw_cnt;
+  p.srcloc = g.d_srcloc; p.win = g.d_win; p.cw_off = g.d_cw_off; p.cw_cnt = g.d_cw_cnt; p.active = g.d_active;
   p.cw_src = g.d_cw_src; p.mapper = g.d_mapper; p.vv = g.d_vv; p.outdeg = g.d_outdeg;
   p.ctl = g.d_ctl; p.trace = g.d_trace; p.trace_cap = g.trace_cap;
   p.use_cond = 0; p.cond_handle = 0;
