@@ -27,7 +27,7 @@ import numpy as np  # noqa: E402
 
 # workload -> (algorithm, representation, source, description)
 WORKLOADS = {
-    "C1": ("bfs", "gs", 0, "BFS from 0 on R-MAT 4,096 V / 32,768 E"),
+    "C1": ("bfs", "gs", 0, "BFS from 0 on R-MAT 4,096 V / 32,768 E, |N| = 128 (SURVEY §8(a) override)"),
     "C2": ("pr", "cw", 0, "PageRank (d=0.85, eps=1e-5) on LiveJournal-shaped R-MAT 4,847,571 V / 68,993,773 E, CW"),
     "C3": ("sssp", "cw", 0, "SSSP on RoadNet-CA-shaped mesh 1,971,281 V / 5,533,214 E, CW"),
     "C3gs": ("sssp", "gs", 0, "SSSP on RoadNet-CA-shaped mesh 1,971,281 V / 5,533,214 E, G-Shards"),
@@ -65,7 +65,7 @@ class ClockSampler:
     def __enter__(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                          "--format=csv,noheader,nounits", "-lms", "20"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
         except FileNotFoundError:
             self.proc = None
@@ -208,6 +208,8 @@ def bench_cusha(args):
     torch.cuda.set_device(local)
     dev = local
     alg, repr_, source, desc = WORKLOADS[args.workload]
+    if args.N == 0 and args.workload == "C1":
+        args.N = 128  # the L310 rule gives 3 shards at this size
     if args.repr:
         repr_ = args.repr
     wl = load_graph(args.workload, args.cache_dir)

@@ -27,14 +27,16 @@ namespace cusha {
 
 constexpr uint32_t kFull = 0xFFFFFFFFu;
 // tuning constants (tools/tune: variants are built with -DCUSHA_*)
+// (measured on C2 PageRank: bytes in flight per SM
+// decide; 2 CTAs/SM x 3 slots x 24 KB beat deeper rings at 1 CTA/SM)
 #ifndef CUSHA_CONSUMER_WARPS
-#define CUSHA_CONSUMER_WARPS 8
+#define CUSHA_CONSUMER_WARPS 16
 #endif
 #ifndef CUSHA_STAGES
-#define CUSHA_STAGES 4
+#define CUSHA_STAGES 3
 #endif
 #ifndef CUSHA_TILE
-#define CUSHA_TILE 1024
+#define CUSHA_TILE 4096  // entries per slot without EdgeValue (24 KB); halved with EdgeValue (20 KB)
 #endif
 #ifndef CUSHA_PERSISTENT
 #define CUSHA_PERSISTENT 1
@@ -53,7 +55,11 @@ constexpr uint32_t kVB = CUSHA_VB;                   // vertex loads in flight p
 constexpr uint32_t kConsumerWarps = CUSHA_CONSUMER_WARPS;
 constexpr uint32_t kConsumers = kConsumerWarps * 32;
 constexpr uint32_t kPassThreads = kConsumers + 32;  // + 1 producer warp
-constexpr uint32_t kTile = CUSHA_TILE;              // entries per ring slot
+// entries per ring slot
+template <class A>
+constexpr uint32_t tile_of() {
+  return A::kEdge ? CUSHA_TILE / 2 : CUSHA_TILE;
+}
 constexpr uint32_t kStages = CUSHA_STAGES;          // ring depth
 constexpr uint32_t kConsumerBar = 1;                // named barrier of the consumer warps
 
@@ -61,7 +67,7 @@ constexpr uint32_t kConsumerBar = 1;                // named barrier of the cons
 //            stage 4 = SrcIndexCW (2T) | Mapper (4T)
 template <class A>
 constexpr uint32_t slot_bytes() {
-  return kTile * (6 + (A::kEdge ? 4 : 0));
+  return tile_of<A>() * (6 + (A::kEdge ? 4 : 0));
 }
 
 enum : uint32_t { kDescStage2 = 0, kDescStage4 = 1, kDescDone = 2 };
@@ -166,6 +172,7 @@ template <class A, int REPR>
 __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDesc* desc, uint64_t* full_bar,
                                          uint64_t* empty_bar, uint64_t* decide_bar, const volatile int* s_any) {
   constexpr uint32_t SLOT = slot_bytes<A>();
+  constexpr uint32_t kTile = tile_of<A>();
   uint32_t slot = 0, ph = 0, dph = 0;
   auto push = [&](uint32_t shard, uint32_t kind, uint32_t n, uint32_t flags, const void* g0, uint32_t b0,
                   const void* g1, uint32_t o1, uint32_t b1, const void* g2, uint32_t o2, uint32_t b2) {
@@ -221,6 +228,7 @@ template <class A, int REPR>
 __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(const KParams p) {
   extern __shared__ __align__(128) uint8_t dyn[];
   constexpr uint32_t SLOT = slot_bytes<A>();
+  constexpr uint32_t kTile = tile_of<A>();
   uint8_t* const ring = dyn;
   uint32_t* const sm = reinterpret_cast<uint32_t*>(dyn + kStages * SLOT);
   __shared__ uint64_t full_bar[kStages], empty_bar[kStages], decide_bar;
