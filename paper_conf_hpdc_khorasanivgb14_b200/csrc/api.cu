@@ -43,15 +43,31 @@ static void free_graph_memory(Graph& g) {
   void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcloc, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
                   g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_srcvalue, g.d_vv, g.d_ctl, g.d_trace,
                   g.d_active};
+  // device memory is stream-ordered (cudaMallocAsync on g.stream): released to
+  // the retained pool without unmapping or a device-wide synchronisation
   for (void* p : ptrs)
-    if (p) cudaFree(p);
+    if (p) cudaFreeAsync(p, g.stream);
   for (void*& p : g.d_init)
-    if (p) { cudaFree(p); p = nullptr; }
-  if (g.h_ctl) cudaFreeHost(g.h_ctl);
+    if (p) { cudaFreeAsync(p, g.stream); p = nullptr; }
+  delete g.h_ctl;
+  g.h_ctl = nullptr;
   if (g.ev0) cudaEventDestroy(g.ev0);
   if (g.ev1) cudaEventDestroy(g.ev1);
   if (g.evm) cudaEventDestroy(g.evm);
-  if (g.own_stream && g.stream) cudaStreamDestroy(g.stream);
+  if (g.own_stream && g.stream) {
+    cudaStreamSynchronize(g.stream);
+    cudaStreamDestroy(g.stream);
+  }
+}
+
+// Keep freed device memory in the default pool so that repeated builds (the
+// e2e path) reuse it instead of mapping HBM again.
+static void retain_pool(int device) {
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+    uint64_t keep = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+  }
 }
 
 static uint64_t device_bytes(const Graph& g) {
@@ -137,6 +153,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   };
   int rc;
   if ((rc = cu(cudaSetDevice(o.device), "cudaSetDevice"))) return bail(rc);
+  retain_pool(o.device);
   if (o.stream) {
     g.stream = (cudaStream_t)o.stream;
   } else {
@@ -156,7 +173,10 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   uint64_t h2d = 0;
   if (o.input_location == CUSHA_INPUT_HOST && E) {
     const uint64_t nvals = edge_values ? 3 : 2;
-    if ((rc = cu(cudaMalloc(&tmp, nvals * E * 4), "cudaMalloc(inputs)"))) { cudaEventDestroy(eh); return bail(rc); }
+    if ((rc = cu(cudaMallocAsync(&tmp, nvals * E * 4, g.stream), "cudaMallocAsync(inputs)"))) {
+      cudaEventDestroy(eh);
+      return bail(rc);
+    }
     cudaMemcpyAsync(tmp, src, E * 4, cudaMemcpyHostToDevice, g.stream);
     cudaMemcpyAsync(tmp + E, dst, E * 4, cudaMemcpyHostToDevice, g.stream);
     if (edge_values) cudaMemcpyAsync(tmp + 2 * E, edge_values, E * 4, cudaMemcpyHostToDevice, g.stream);
@@ -167,18 +187,19 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   std::string err;
   rc = build_layout(g, d_src, d_dst, d_val, err);
   if (rc) {
-    if (tmp) cudaFree(tmp);
+    if (tmp) cudaFreeAsync(tmp, g.stream);
     cudaEventDestroy(eh);
     set_error("build: " + err);
     return bail(rc);
   }
-  if (tmp) cudaFree(tmp);
+  if (tmp) cudaFreeAsync(tmp, g.stream);
   // per-run state: SrcValue (P entries + trash slot), VertexValues (8 B/vertex covers every Table-3 Vertex)
-  if ((rc = cu(cudaMalloc(&g.d_srcvalue, 4 * (g.P + 1)), "cudaMalloc(SrcValue)")) ||
+  g.h_ctl = new (std::nothrow) Ctl();
+  if ((rc = cu(cudaMallocAsync(&g.d_srcvalue, 4 * (g.P + 1), g.stream), "cudaMallocAsync(SrcValue)")) ||
       (rc = cu(cudaMemsetAsync(g.d_srcvalue, 0, 4 * (g.P + 1), g.stream), "memset")) ||
-      (rc = cu(cudaMalloc(&g.d_vv, 8ull * V), "cudaMalloc(VertexValues)")) ||
-      (rc = cu(cudaMalloc(&g.d_ctl, sizeof(Ctl)), "cudaMalloc(ctl)")) ||
-      (rc = cu(cudaMallocHost(&g.h_ctl, sizeof(Ctl)), "cudaMallocHost(ctl)"))) {
+      (rc = cu(cudaMallocAsync(&g.d_vv, 8ull * V, g.stream), "cudaMallocAsync(VertexValues)")) ||
+      (rc = cu(cudaMallocAsync(&g.d_ctl, sizeof(Ctl), g.stream), "cudaMallocAsync(ctl)")) ||
+      (rc = g.h_ctl ? 0 : CUSHA_ENOMEM)) {
     cudaEventDestroy(eh);
     return bail(rc);
   }
@@ -223,7 +244,7 @@ int cusha_set_vertex_values(cusha_graph* h, cusha_algorithm alg, const void* ini
   const size_t want = (size_t)g.V * value_bytes((int)alg);
   if (bytes != want) return fail(CUSHA_EINVAL, "bytes must be |V| * value_bytes(alg)");
   CKA(cudaSetDevice(g.device));
-  if (!g.d_init[alg]) CKA(cudaMalloc(&g.d_init[alg], want));
+  if (!g.d_init[alg]) CKA(cudaMallocAsync(&g.d_init[alg], want, g.stream));
   CKA(cudaMemcpyAsync(g.d_init[alg], init, want, cudaMemcpyHostToDevice, g.stream));
   CKA(cudaStreamSynchronize(g.stream));
   return CUSHA_OK;
@@ -295,10 +316,10 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   // trace buffer sized to min(max_iters, 2^20)
   const uint32_t want_cap = std::min<uint32_t>(std::max<uint32_t>(max_iters, 1), 1u << 20);
   if (g.trace_cap < want_cap) {
-    if (g.d_trace) cudaFree(g.d_trace);
+    if (g.d_trace) cudaFreeAsync(g.d_trace, g.stream);
     g.d_trace = nullptr;
     g.trace_cap = 0;
-    CKA(cudaMalloc(&g.d_trace, sizeof(TraceRec) * (size_t)want_cap));
+    CKA(cudaMallocAsync(&g.d_trace, sizeof(TraceRec) * (size_t)want_cap, g.stream));
     g.trace_cap = want_cap;
     for (auto& e : h->exec)  // kernel params captured the old trace pointer
       if (e) { cudaGraphExecDestroy(e); e = nullptr; }

@@ -15,6 +15,9 @@
 // W_i1, ... concatenated).
 #include <cub/cub.cuh>
 
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <string>
 
 #include "common.cuh"
@@ -187,9 +190,30 @@ __global__ void k_fill_cw_pads(const uint32_t* coff, const uint32_t* ccnt, uint3
   }
 }
 
+// Build temporaries are stream-ordered allocations on the graph's stream
+// (cudaMallocAsync from the device pool, which cusha_build_graph sets to
+// retain freed memory): repeated builds neither map nor unmap HBM.
+thread_local cudaStream_t t_alloc_stream = nullptr;
 struct DevBuf {  // RAII temporary
   void* p = nullptr;
-  ~DevBuf() { if (p) cudaFree(p); }
+  ~DevBuf() { if (p) cudaFreeAsync(p, t_alloc_stream); }
+};
+
+// Diagnostics only: CUSHA_DEBUG_BUILD=1 prints the wall time of each build
+// phase (synchronising at every mark, so it perturbs what it measures).
+struct PhaseTimer {
+  bool on = std::getenv("CUSHA_DEBUG_BUILD") != nullptr;
+  cudaStream_t st;
+  std::chrono::steady_clock::time_point t = std::chrono::steady_clock::now();
+  explicit PhaseTimer(cudaStream_t s) : st(s) {}
+  void mark(const char* what) {
+    if (!on) return;
+    cudaStreamSynchronize(st);
+    const auto n = std::chrono::steady_clock::now();
+    std::fprintf(stderr, "[cusha build] %-28s %9.3f ms\n", what,
+                 std::chrono::duration<double, std::milli>(n - t).count());
+    t = n;
+  }
 };
 
 #define CK(call)                                                                     \
@@ -203,7 +227,7 @@ struct DevBuf {  // RAII temporary
 
 template <class T>
 cudaError_t dalloc(T** p, uint64_t n) {
-  return cudaMalloc(reinterpret_cast<void**>(p), (n ? n : 1) * sizeof(T));
+  return cudaMallocAsync(reinterpret_cast<void**>(p), (n ? n : 1) * sizeof(T), t_alloc_stream);
 }
 
 }  // namespace
@@ -216,12 +240,15 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
             bsh = bits_for(S - 1);
   const int total = bsh + bsrc + bn;
   if (total > 64) { err = "key does not fit 64 bits"; return CUSHA_EINVAL; }
+  PhaseTimer pt(st);
+  t_alloc_stream = st;
 
   DevBuf keys, keys2, ids, ids2, bad, start, padded, temp, pos_of;
   CK(dalloc((uint64_t**)&keys.p, E));
   CK(dalloc((uint64_t**)&keys2.p, E));
   CK(dalloc((uint32_t**)&ids.p, E));
   CK(dalloc((uint32_t**)&ids2.p, E));
+  pt.mark("alloc keys/ids");
   CK(dalloc((uint32_t**)&bad.p, 1));
   CK(cudaMemsetAsync(bad.p, 0, 4, st));
   if (E) k_make_keys<<<grid_for(E), 256, 0, st>>>(d_src, d_dst, E, V, N, bn, bsrc, (uint64_t*)keys.p, (uint32_t*)ids.p,
@@ -231,6 +258,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   CK(cudaMemcpyAsync(&h_bad, bad.p, 4, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   if (h_bad) { err = "edge endpoint >= num_vertices"; return CUSHA_EINVAL; }
+  pt.mark("keys + validate");
 
   // ---- G-Shards order
   cub::DoubleBuffer<uint64_t> kb((uint64_t*)keys.p, (uint64_t*)keys2.p);
@@ -238,9 +266,10 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   size_t tbytes = 0;
   if (E) {
     CK(cub::DeviceRadixSort::SortPairs(nullptr, tbytes, kb, vb, (int64_t)E, 0, total, st));
-    CK(cudaMalloc(&temp.p, tbytes));
+    CK(cudaMallocAsync(&temp.p, tbytes, st));
     CK(cub::DeviceRadixSort::SortPairs(temp.p, tbytes, kb, vb, (int64_t)E, 0, total, st));
   }
+  pt.mark("G-Shards sort");
   const uint64_t* K = kb.Current();
   const uint32_t* I = vb.Current();
 
@@ -257,7 +286,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
     size_t b2 = 0;
     CK(dalloc((uint64_t**)&scan.p, (uint64_t)S + 1));
     CK(cub::DeviceScan::ExclusiveSum(nullptr, b2, (uint64_t*)padded.p, (uint64_t*)scan.p, (int64_t)S + 1, st));
-    CK(cudaMalloc(&t2.p, b2 ? b2 : 1));
+    CK(cudaMallocAsync(&t2.p, b2 ? b2 : 1, st));
     CK(cub::DeviceScan::ExclusiveSum(t2.p, b2, (uint64_t*)padded.p, (uint64_t*)scan.p, (int64_t)S + 1, st));
     uint64_t P = 0;
     CK(cudaMemcpyAsync(&P, (uint64_t*)scan.p + S, 8, cudaMemcpyDeviceToHost, st));
@@ -273,6 +302,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   CK(dalloc(&g.d_eid, P));
   if (d_val) { CK(dalloc(&g.d_ev, P)); g.has_ev = true; }
   CK(dalloc((uint32_t**)&pos_of.p, E));
+  pt.mark("offsets + alloc shard arrays");
   k_fill_shard_pads<<<grid_for((uint64_t)S * kPad), 256, 0, st>>>(g.d_shard_off, g.d_shard_cnt, S, N, g.d_dest,
                                                                    g.d_srcloc, g.d_eid, g.d_ev);
   if (E)
@@ -281,6 +311,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   CK(cudaGetLastError());
 
   // ---- window table W_ij (both representations keep it; GS stage 4 reads it)
+  pt.mark("scatter shards");
   CK(dalloc(&g.d_win, ((uint64_t)S + 1) * S));
   if (E)
     k_windows<<<grid_for(E), 256, 0, st>>>(K, E, (uint32_t*)start.p, (uint32_t*)pos_of.p, N, S, bn, bsrc, g.d_win);
@@ -289,6 +320,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   CK(cudaGetLastError());
 
   // ---- out-degrees (PR NbrsNum, L318) and |CW_i|
+  pt.mark("window table");
   CK(dalloc(&g.d_outdeg, V));
   CK(cudaMemsetAsync(g.d_outdeg, 0, (size_t)V * 4, st));
   if (E) k_outdeg<<<grid_for(E), 256, 0, st>>>(d_src, E, g.d_outdeg);
@@ -299,6 +331,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   CK(dalloc(&g.d_active, S));  // stage-4 prefetch predictor of the shard pass
 
   // ---- Concatenated Windows + Mapper (§3.2)
+  pt.mark("outdeg + cw counts");
   if (g.repr == CUSHA_REPR_CW) {
     // reuse the key buffers: ks (u32) in keys.Alternate, positions in ids.Alternate
     uint32_t* ks = reinterpret_cast<uint32_t*>(kb.Alternate());
@@ -312,13 +345,14 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
       size_t b3 = 0;
       CK(cub::DeviceRadixSort::SortPairs(nullptr, b3, kk, pv, (int64_t)E, 0, bks, st));
       if (b3 > tbytes) {
-        cudaFree(temp.p);
+        cudaFreeAsync(temp.p, st);
         temp.p = nullptr;
-        CK(cudaMalloc(&temp.p, b3));
+        CK(cudaMallocAsync(&temp.p, b3, st));
         tbytes = b3;
       }
       CK(cub::DeviceRadixSort::SortPairs(temp.p, b3, kk, pv, (int64_t)E, 0, bks, st));
     }
+    pt.mark("CW sort");
     DevBuf cstart, cpad, cscan, t4;
     CK(dalloc((uint32_t**)&cstart.p, (uint64_t)S + 1));
     CK(dalloc((uint64_t**)&cpad.p, (uint64_t)S + 1));
@@ -330,7 +364,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
     CK(cudaGetLastError());
     size_t b4 = 0;
     CK(cub::DeviceScan::ExclusiveSum(nullptr, b4, (uint64_t*)cpad.p, (uint64_t*)cscan.p, (int64_t)S + 1, st));
-    CK(cudaMalloc(&t4.p, b4 ? b4 : 1));
+    CK(cudaMallocAsync(&t4.p, b4 ? b4 : 1, st));
     CK(cub::DeviceScan::ExclusiveSum(t4.p, b4, (uint64_t*)cpad.p, (uint64_t*)cscan.p, (int64_t)S + 1, st));
     uint64_t Q = 0;
     CK(cudaMemcpyAsync(&Q, (uint64_t*)cscan.p + S, 8, cudaMemcpyDeviceToHost, st));
@@ -349,9 +383,10 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(st));
     // CW keeps the 3-tuple shards + SrcIndexCW + Mapper (L175): no per-entry SrcIndex in shard order
-    cudaFree(g.d_srcloc);
+    cudaFreeAsync(g.d_srcloc, st);
     g.d_srcloc = nullptr;
   }
+  pt.mark("CW offsets + scatter");
   CK(cudaStreamSynchronize(st));
   return CUSHA_OK;
 }
