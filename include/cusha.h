@@ -85,10 +85,23 @@ typedef struct {
                                       1 = host launches passes in chunks of 8 (for profilers that
                                       cannot see kernels inside conditional graphs); passes past
                                       convergence exit at once, so results are identical      */
-  /* Multi-GPU (destination-range partition): */
-  int world_size;                  /* 1 = single GPU (0 is treated as 1)                       */
-  int rank;                        /* this process's rank, 0..world_size-1                     */
-  const void* nccl_unique_id;      /* 128-byte ncclUniqueId shared by all ranks (world_size>1) */
+  /* Destination-range partition (row e; north_star (4)).  With
+   * world_size = G > 1 the shards are split into G contiguous ranges of
+   * near-equal work (cusha_partition_shards); partition r owns the vertices
+   * of its shards.  Within a partition the pass is asynchronous (L45); across
+   * partitions it is BSP: after each pass every partition's write-back values
+   * are exchanged and the windows fed by other partitions are refreshed.
+   * CW representation only.
+   *   nccl_unique_id != NULL: one process per GPU; every rank passes the full
+   *     edge list, its rank and the same 128-byte ncclUniqueId
+   *     (cusha_nccl_unique_id on rank 0, broadcast by the caller); the
+   *     exchange is NCCL broadcasts over NVLink.
+   *   nccl_unique_id == NULL: all G partitions run in this process on one
+   *     device and exchange through device memory (the same kernels; used to
+   *     test the partitioned algorithm on one GPU).                            */
+  int world_size;                  /* 1 = single partition (0 is treated as 1)                  */
+  int rank;                        /* this process's rank, 0..world_size-1 (NCCL mode)          */
+  const void* nccl_unique_id;      /* 128-byte ncclUniqueId, or NULL (see above)                */
 } cusha_build_opts;
 
 typedef struct cusha_graph cusha_graph;   /* opaque; owns all device memory it allocates */
@@ -234,8 +247,20 @@ CUSHA_API const char* cusha_last_error(void);
 CUSHA_API int cusha_abi_version(void);
 
 /* Multi-GPU helper: write a fresh 128-byte ncclUniqueId to out128 (rank 0
- * calls this and broadcasts it, e.g. over torch.distributed). */
+ * calls this and broadcasts it, e.g. over torch.distributed).  NCCL
+ * (libnccl.so.2) is loaded at run time; CUSHA_EUNSUPPORTED if absent. */
 CUSHA_API int cusha_nccl_unique_id(void* out128);
+
+/* Host logic of the destination-range partition (pure host, no device):
+ * split shards 0..num_shards-1 into `parts` contiguous ranges of near-equal
+ * total work[s] (cusha_build_graph uses stage-2 + stage-4 entries per shard).
+ * bounds[parts+1] receives 0 = b0 <= b1 <= ... <= b_parts = num_shards; range
+ * q = [b_q, b_{q+1}).  Deterministic: every rank computes the same bounds. */
+CUSHA_API int cusha_partition_shards(uint32_t num_shards, const uint64_t* work, uint32_t parts, uint32_t* bounds);
+
+/* The partition a graph was built with: writes G+1 bounds (G = 1 for an
+ * unpartitioned graph) to bounds (host, cap entries); returns G. */
+CUSHA_API int cusha_get_partition(const cusha_graph* g, uint32_t* bounds, uint32_t cap);
 
 #ifdef __cplusplus
 }

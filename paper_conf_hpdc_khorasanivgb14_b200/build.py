@@ -15,7 +15,19 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 OUT = os.path.join(HERE, "libcusha.so")
 OBJDIR = os.path.join(HERE, "build")
-SOURCES = ["api.cu", "builder.cu", "kernels.cu"]
+SOURCES = ["api.cu", "builder.cu", "kernels.cu", "nccl.cu"]
+
+
+def nccl_include() -> str:
+    """nccl.h only (the library is dlopen'ed at run time): torch's NCCL wheel, else the system."""
+    try:
+        import nvidia.nccl  # noqa: F401
+        d = os.path.join(list(nvidia.nccl.__path__)[0], "include")
+        if os.path.exists(os.path.join(d, "nccl.h")):
+            return d
+    except Exception:
+        pass
+    return "/usr/include"
 HEADERS = ["common.cuh", "algorithms.cuh", "graph.hpp"]
 
 NVCC_FLAGS = [
@@ -53,8 +65,8 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str = OUT
         obj = os.path.join(objdir, s + ".o")
         objs.append(obj)
         if force or _stale(obj, [src] + hdrs):
-            cmd = [nvcc(), *NVCC_FLAGS, *["-D" + d for d in defines], "-I", os.path.join(ROOT, "include"), "-c", src,
-                   "-o", obj]
+            cmd = [nvcc(), *NVCC_FLAGS, *["-D" + d for d in defines], "-I", os.path.join(ROOT, "include"),
+                   "-I", nccl_include(), "-c", src, "-o", obj]
             jobs.append((s, cmd))
 
     def run(job):
@@ -73,7 +85,7 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str = OUT
     if force or jobs or not os.path.exists(out):
         tmp = out + ".tmp%d" % os.getpid()
         cmd = [nvcc(), "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", tmp, *objs,
-               "-Xcompiler", "-fPIC", "-cudart", "static"]
+               "-Xcompiler", "-fPIC", "-cudart", "static", "-ldl"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stderr}")

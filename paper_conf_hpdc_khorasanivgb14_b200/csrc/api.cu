@@ -42,7 +42,8 @@ static int fail(int code, const std::string& msg) {
 static void free_graph_memory(Graph& g) {
   void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcloc, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
                   g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_srcvalue, g.d_vv, g.d_ctl, g.d_trace,
-                  g.d_active};
+                  g.d_active, g.d_bounds, g.d_owner, g.d_cwp, g.d_gathered};
+  nccl_destroy(g);
   // device memory is stream-ordered (cudaMallocAsync on g.stream): released to
   // the retained pool without unmapping or a device-wide synchronisation
   for (void* p : ptrs)
@@ -135,7 +136,11 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   if (opts) o = *opts;
   if (o.repr != CUSHA_REPR_GSHARDS && o.repr != CUSHA_REPR_CW) return fail(CUSHA_EINVAL, "bad repr");
   if (o.world_size <= 0) o.world_size = 1;
-  if (o.world_size != 1) return fail(CUSHA_EUNSUPPORTED, "world_size > 1 requires cusha_build_graph_multi");
+  if (o.world_size > 64) return fail(CUSHA_EINVAL, "world_size must be <= 64");
+  if (o.world_size > 1 && o.repr != CUSHA_REPR_CW)
+    return fail(CUSHA_EUNSUPPORTED, "the partitioned (multi-GPU) mode uses the CW representation");
+  if (o.world_size > 1 && o.nccl_unique_id && (o.rank < 0 || o.rank >= o.world_size))
+    return fail(CUSHA_EINVAL, "rank out of range");
   uint32_t N = o.vertices_per_shard ? o.vertices_per_shard : cusha_shard_size(V, E, o.smem_bytes_per_vertex, 0, 0);
   if (N > 65534) return fail(CUSHA_EINVAL, "vertices_per_shard must be <= 65534");
   if (N > V) N = V;
@@ -145,6 +150,14 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   Graph& g = h->g;
   g.V = V; g.E = E; g.N = N; g.S = (V + N - 1) / N; g.repr = (int)o.repr; g.device = o.device;
   g.host_loop = o.host_loop != 0;
+  g.world_size = o.world_size;
+  g.rank = o.world_size > 1 && o.nccl_unique_id ? o.rank : 0;
+  g.simulate = o.world_size > 1 && !o.nccl_unique_id;
+  g.G = std::min<uint32_t>((uint32_t)o.world_size, g.S);  // never more partitions than shards
+  if (!g.simulate && g.G != (uint32_t)o.world_size) {
+    delete h;
+    return fail(CUSHA_EINVAL, "world_size exceeds the number of shards");
+  }
   auto bail = [&](int code) { free_graph_memory(g); delete h; return code; };
   auto cu = [&](cudaError_t e, const char* what) -> int {
     if (e == cudaSuccess) return 0;
@@ -193,6 +206,15 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
     return bail(rc);
   }
   if (tmp) cudaFreeAsync(tmp, g.stream);
+  if (g.G > 1) {  // destination-range partition (row e)
+    rc = build_partition(g, err);
+    if (!rc && !g.simulate) rc = nccl_init(g, o.nccl_unique_id, err);
+    if (rc) {
+      cudaEventDestroy(eh);
+      set_error("partition: " + err);
+      return bail(rc);
+    }
+  }
   // per-run state: SrcValue (P entries + trash slot), VertexValues (8 B/vertex covers every Table-3 Vertex)
   g.h_ctl = new (std::nothrow) Ctl();
   if ((rc = cu(cudaMallocAsync(&g.d_srcvalue, 4 * (g.P + 1), g.stream), "cudaMallocAsync(SrcValue)")) ||
@@ -221,8 +243,8 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   g.st.h2d_bytes = h2d;
   g.st.device_bytes = device_bytes(g);
   g.st.entries_padded = g.P;
-  g.st.world_size = 1;
-  g.st.rank = 0;
+  g.st.world_size = g.world_size;
+  g.st.rank = g.rank;
   *out = h;
   set_error("");
   return CUSHA_OK;
@@ -253,14 +275,16 @@ int cusha_set_vertex_values(cusha_graph* h, cusha_algorithm alg, const void* ini
 // Persistent grid of the shard pass: as many CTAs as fit on the device at
 // once (occupancy x SMs), never more than there are shards.
 static uint32_t pass_grid(const Graph& g, const PassKernel& pk, size_t smem) {
-  if (!pk.persistent) return std::max<uint32_t>(g.S, 1);
+  // shards this process runs: its partition (multi-GPU) or all of them
+  const uint32_t mine = g.G > 1 && !g.simulate ? g.h_bounds[g.rank + 1] - g.h_bounds[g.rank] : g.S;
+  if (!pk.persistent) return std::max<uint32_t>(mine, 1);
   int sms = 148, per_sm = 1;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g.device);
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, pk.func, (int)pk.threads, smem) != cudaSuccess ||
       per_sm < 1)
     per_sm = 1;
   const uint64_t gsz = (uint64_t)sms * (uint64_t)per_sm;
-  return (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(gsz, g.S));
+  return (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(gsz, mine));
 }
 
 static int ensure_exec(cusha_graph* h, int alg) {
@@ -327,7 +351,8 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   const PassKernel& pk = pass_kernel(a, g.repr);
   const size_t smem = pk.smem_bytes(g.N);
   int rc = CUSHA_OK;
-  if (g.host_loop) {
+  const bool host_loop = g.host_loop || g.G > 1;  // the partitioned mode exchanges between passes
+  if (host_loop) {
     if (smem > 227 * 1024)
       return fail(CUSHA_EINVAL, "vertices_per_shard too large for this algorithm's shared-memory state");
     CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -341,19 +366,32 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   CKA(launch_reset_ctl(g.d_ctl, max_iters, g.stream));
   CKA(launch_init(g, a, source, g.stream));
   CKA(cudaEventRecord(g.evm, g.stream));
-  if (max_iters > 0 && !g.host_loop) CKA(cudaGraphLaunch(h->exec[a], g.stream));
-  if (max_iters > 0 && g.host_loop) {
+  if (max_iters > 0 && !host_loop) CKA(cudaGraphLaunch(h->exec[a], g.stream));
+  if (max_iters > 0 && host_loop) {
     // passes launched by the host in chunks; a pass that finds the run
-    // converged (or at max_iters) exits at once, so over-launching is exact
+    // converged (or at max_iters) exits at once, so over-launching is exact.
+    // Partitioned: pass -> exchange (NCCL, multi-GPU) -> refresh of remote
+    // windows + global convergence; every rank takes the same decisions
+    // from the same exchanged data, so all issue the same collectives.
     KParams kp = make_params(g, source);
     void* args[] = {&kp};
+    const dim3 grid(pass_grid(g, pk, smem));
+    const int chunk = g.G > 1 && !g.simulate ? 1 : 8;
+    std::string err;
     for (;;) {
-      for (int k = 0; k < 8; ++k)
-        CKA(cudaLaunchKernel(pk.func, dim3(pass_grid(g, pk, smem)), dim3(pk.threads), args, smem, g.stream));
+      for (int k = 0; k < chunk; ++k) {
+        CKA(cudaLaunchKernel(pk.func, grid, dim3(pk.threads), args, smem, g.stream));
+        if (g.G > 1) {
+          if (!g.simulate && (rc = nccl_exchange(g, 0, false, err))) return fail(rc, "exchange: " + err);
+          CKA(launch_refresh(g, g.stream));
+        }
+      }
       CKA(cudaMemcpyAsync(g.h_ctl, g.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g.stream));
       CKA(cudaStreamSynchronize(g.stream));
       if (g.h_ctl->converged || g.h_ctl->iter >= max_iters) break;
     }
+    if (g.G > 1 && !g.simulate && (rc = nccl_exchange(g, (uint32_t)value_bytes(a), true, err)))
+      return fail(rc, "final exchange: " + err);
   }
   CKA(cudaEventRecord(g.ev1, g.stream));
   CKA(cudaMemcpyAsync(g.h_ctl, g.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g.stream));
@@ -474,8 +512,30 @@ int cusha_get_layout(const cusha_graph* h, cusha_layout_part part, void* out, si
 }
 
 int cusha_nccl_unique_id(void* out128) {
-  (void)out128;
-  return fail(CUSHA_EUNSUPPORTED, "built without NCCL");
+  if (!out128) return fail(CUSHA_EINVAL, "out128 is NULL");
+  std::string err;
+  const int rc = nccl_unique_id(out128, err);
+  return rc ? fail(rc, err) : CUSHA_OK;
+}
+
+int cusha_partition_shards(uint32_t num_shards, const uint64_t* work, uint32_t parts, uint32_t* bounds) {
+  if (!work || !bounds || parts == 0) return fail(CUSHA_EINVAL, "null argument or parts == 0");
+  partition_bounds(num_shards, work, parts, bounds);
+  return CUSHA_OK;
+}
+
+int cusha_get_partition(const cusha_graph* h, uint32_t* bounds, uint32_t cap) {
+  if (!h || !bounds) return fail(CUSHA_EINVAL, "null argument");
+  const Graph& g = h->g;
+  if (g.G <= 1) {
+    if (cap < 2) return fail(CUSHA_EINVAL, "cap too small");
+    bounds[0] = 0;
+    bounds[1] = g.S;
+    return 1;
+  }
+  if (cap < g.G + 1) return fail(CUSHA_EINVAL, "cap too small");
+  for (uint32_t q = 0; q <= g.G; ++q) bounds[q] = g.h_bounds[q];
+  return (int)g.G;
 }
 
 }  // extern "C"

@@ -391,4 +391,70 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   return CUSHA_OK;
 }
 
+// ------------------------------------------------ destination-range partition
+// Contiguous shard ranges (= destination-vertex ranges, the Partitioned
+// property) with near-equal work: bounds[q] = first shard whose work
+// prefix reaches q/G of the total.
+void partition_bounds(uint32_t S, const uint64_t* work, uint32_t G, uint32_t* bounds) {
+  uint64_t total = 0;
+  for (uint32_t s = 0; s < S; ++s) total += work[s];
+  bounds[0] = 0;
+  uint64_t pre = 0;
+  uint32_t s = 0;
+  for (uint32_t q = 1; q < G; ++q) {
+    const long double target = (long double)total * q / G;
+    while (s < S && (long double)pre + (long double)work[s] / 2 < target) pre += work[s++];
+    bounds[q] = s;
+  }
+  bounds[G] = S;
+}
+
+namespace {
+// cwp[i][q] = first CW_i position whose Mapper target lies in partition q:
+// CW_i lists W_i0, W_i1, ... in shard order (L175), so that is cw_off[i] plus
+// the sizes of W_ij for j < bounds[q].
+__global__ void k_cwp(const uint32_t* __restrict__ win, const uint32_t* cw_off, const uint32_t* cw_cnt,
+                      const uint32_t* bounds, uint32_t S, uint32_t G, uint32_t* cwp) {
+  GRID_STRIDE(t, (uint64_t)S * (G + 1)) {
+    const uint32_t i = (uint32_t)(t / (G + 1)), q = (uint32_t)(t % (G + 1));
+    uint32_t acc = 0;
+    if (q == G) {
+      acc = cw_cnt[i];
+    } else {
+      const uint32_t* r0 = win + (size_t)i * S;
+      const uint32_t* r1 = r0 + S;
+      for (uint32_t j = 0; j < bounds[q]; ++j) acc += r1[j] - r0[j];
+    }
+    cwp[t] = cw_off[i] + acc;
+  }
+}
+}  // namespace
+
+int build_partition(Graph& g, std::string& err) {
+  cudaStream_t st = g.stream;
+  t_alloc_stream = st;
+  const uint32_t S = g.S, G = g.G;
+  std::vector<uint32_t> cnt(S), ccnt(S);
+  CK(cudaMemcpyAsync(cnt.data(), g.d_shard_cnt, 4ull * S, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(ccnt.data(), g.d_cw_cnt, 4ull * S, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  std::vector<uint64_t> work(S);
+  for (uint32_t s = 0; s < S; ++s) work[s] = (uint64_t)cnt[s] + ccnt[s];  // stage-2 + stage-4 entries
+  g.h_bounds.assign(G + 1, 0);
+  partition_bounds(S, work.data(), G, g.h_bounds.data());
+  std::vector<uint8_t> owner(S);
+  for (uint32_t q = 0; q < G; ++q)
+    for (uint32_t s = g.h_bounds[q]; s < g.h_bounds[q + 1]; ++s) owner[s] = (uint8_t)q;
+  CK(dalloc(&g.d_bounds, G + 1));
+  CK(dalloc(&g.d_owner, S));
+  CK(dalloc(&g.d_cwp, (uint64_t)S * (G + 1)));
+  CK(dalloc(&g.d_gathered, g.V));
+  CK(cudaMemcpyAsync(g.d_bounds, g.h_bounds.data(), 4ull * (G + 1), cudaMemcpyHostToDevice, st));
+  CK(cudaMemcpyAsync(g.d_owner, owner.data(), S, cudaMemcpyHostToDevice, st));
+  k_cwp<<<grid_for((uint64_t)S * (G + 1)), 256, 0, st>>>(g.d_win, g.d_cw_off, g.d_cw_cnt, g.d_bounds, S, G, g.d_cwp);
+  CK(cudaGetLastError());
+  CK(cudaStreamSynchronize(st));
+  return CUSHA_OK;
+}
+
 }  // namespace cusha

@@ -3,6 +3,7 @@
 #include <cstddef>
 #include <cstdint>
 #include <string>
+#include <vector>
 #include <cuda_runtime.h>
 
 #include "../../include/cusha.h"
@@ -11,13 +12,14 @@ namespace cusha {
 
 // Iteration control word block (row a5), one per graph, device resident.
 struct Ctl {
-  uint32_t iter;       // shard passes completed in this run
-  uint32_t changed;    // set by any CTA whose stage 3 committed an update (is_converged = false, L255)
-  uint32_t ctas_done;  // arrival counter; the last CTA closes the iteration
+  uint32_t iter;        // shard passes completed in this run
+  uint32_t changed;     // set by any CTA whose stage 3 committed an update (is_converged = false, L255)
+  uint32_t ctas_done;   // arrival counter; the last CTA closes the iteration
   uint32_t max_iters;
-  uint32_t converged;  // 1 once a pass committed nothing
-  uint32_t next_shard; // dynamic shard queue of the persistent pass
-  uint32_t pad[2];
+  uint32_t converged;   // 1 once a pass committed nothing
+  uint32_t next_shard;  // dynamic shard queue of the persistent pass
+  uint32_t gchanged;    // partitioned mode: some shard of any partition was active (refresh kernel)
+  uint32_t rctas_done;  // partitioned mode: refresh-kernel arrival counter
 };
 
 // Per-iteration trace (row f4; also the source of algorithmic byte counts).
@@ -39,7 +41,7 @@ struct KParams {
   const uint32_t* win;         // GS: (S+1)*S window starts
   const uint32_t* cw_off;      // CW: S+1 padded CW_i starts
   const uint32_t* cw_cnt;      // S real |CW_i| (both reprs; = entries stage 4 of shard i visits)
-  uint8_t* active;             // S: shard ran stage 4 in the previous pass (stage-4 prefetch predictor)
+  uint8_t* active;             // S: shard ran stage 4 in the last pass (stage-4 prefetch predictor; exchanged)
   const uint16_t* cw_src;      // CW: Q local SrcIndex
   const uint32_t* mapper;      // CW: Q padded shard positions
   void* vv;                    // VertexValues
@@ -49,6 +51,13 @@ struct KParams {
   uint32_t trace_cap;
   int use_cond;
   unsigned long long cond_handle;
+  // destination-range partition (row e); G = 1: single partition
+  uint32_t G;                  // partitions
+  int part;                    // partition this launch processes (-1: all, the single-process simulation)
+  const uint32_t* bounds;      // G+1 shard bounds of the partitions
+  const uint8_t* owner;        // S: partition owning shard s
+  const uint32_t* cwp;         // S*(G+1): CW_i entries whose targets lie in partition p = [cwp[i][p], cwp[i][p+1])
+  uint32_t* gathered;          // V: write-back value of every vertex after its last pass (exchanged)
 };
 
 struct PassKernel {
@@ -80,7 +89,6 @@ struct Graph {
   uint32_t* d_cw_off = nullptr;     // S+1
   uint32_t* d_cw_cnt = nullptr;     // S
   uint8_t* d_active = nullptr;      // S: stage-4 prefetch predictor
-  uint32_t grid = 0;                // persistent CTAs of the shard pass
   uint16_t* d_cw_src = nullptr;     // Q (CW)
   uint32_t* d_mapper = nullptr;     // Q (CW)
   uint32_t* d_outdeg = nullptr;     // V
@@ -91,10 +99,18 @@ struct Graph {
   Ctl* d_ctl = nullptr;
   TraceRec* d_trace = nullptr;
   uint32_t trace_cap = 0;
-  Ctl* h_ctl = nullptr;             // pinned mirror
+  Ctl* h_ctl = nullptr;             // host mirror
   cudaEvent_t ev0 = nullptr, ev1 = nullptr, evm = nullptr;
-  // multi-GPU
+  // destination-range partition (row e)
   int world_size = 1, rank = 0;
+  bool simulate = false;            // all partitions in this process, exchange through device memory
+  uint32_t G = 1;
+  std::vector<uint32_t> h_bounds;   // G+1 shard bounds
+  uint32_t* d_bounds = nullptr;
+  uint8_t* d_owner = nullptr;       // S
+  uint32_t* d_cwp = nullptr;        // S*(G+1)
+  uint32_t* d_gathered = nullptr;   // V
+  void* nccl_comm = nullptr;        // ncclComm_t (real multi-GPU)
   // stats
   cusha_stats st{};
   int last_alg = -1;
@@ -106,6 +122,7 @@ struct Graph {
 const PassKernel& pass_kernel(int alg, int repr);
 cudaError_t launch_init(const Graph& g, int alg, uint32_t source, cudaStream_t s);
 cudaError_t launch_reset_ctl(Ctl* ctl, uint32_t max_iters, cudaStream_t s);
+cudaError_t launch_refresh(const Graph& g, cudaStream_t s);
 KParams make_params(const Graph& g, uint32_t source);
 size_t value_bytes(int alg);
 bool alg_needs_edge_values(int alg);
@@ -113,8 +130,16 @@ bool alg_needs_init(int alg);
 
 // builder.cu
 int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const uint32_t* d_val, std::string& err);
+int build_partition(Graph& g, std::string& err);  // bounds, owner, cwp, gathered (G > 1)
+void partition_bounds(uint32_t S, const uint64_t* work, uint32_t G, uint32_t* bounds);
 
 // api.cu
 void set_error(const std::string& msg);
+
+// nccl.cpp (loaded at run time; no link-time NCCL dependency)
+int nccl_unique_id(void* out128, std::string& err);
+int nccl_init(Graph& g, const void* id128, std::string& err);
+int nccl_exchange(Graph& g, uint32_t value_bytes_vv, bool final_values, std::string& err);
+void nccl_destroy(Graph& g);
 
 }  // namespace cusha

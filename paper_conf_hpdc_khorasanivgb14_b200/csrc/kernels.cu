@@ -72,9 +72,12 @@ constexpr uint32_t slot_bytes() {
 
 enum : uint32_t { kDescStage2 = 0, kDescStage4 = 1, kDescDone = 2 };
 enum : uint32_t { kFlagLast = 1, kFlagSpec4 = 2 };
+// flags: kFlagLast = last tile of this stage; kFlagSpec4 (on a shard's first
+// tile) = stage-4 tiles of this shard follow its stage-2 tiles.  n = entries
+// copied into the slot; [lo, hi) = the entries the consumers use.
 struct __align__(16) TileDesc {
-  uint32_t shard, kind, n, flags;  // flags: kFlagLast = last tile of this stage; kFlagSpec4 (on a shard's
-};                                 // first tile) = stage-4 tiles of this shard follow its stage-2 tiles
+  uint32_t shard, kind, n, flags, lo, hi, pad0, pad1;
+};
 
 // ------------------------------------------------------------ stage 2 body
 template <class A>
@@ -175,9 +178,10 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
   constexpr uint32_t kTile = tile_of<A>();
   uint32_t slot = 0, ph = 0, dph = 0;
   auto push = [&](uint32_t shard, uint32_t kind, uint32_t n, uint32_t flags, const void* g0, uint32_t b0,
-                  const void* g1, uint32_t o1, uint32_t b1, const void* g2, uint32_t o2, uint32_t b2) {
+                  const void* g1, uint32_t o1, uint32_t b1, const void* g2, uint32_t o2, uint32_t b2,
+                  uint32_t lo = 0, uint32_t hi = 0xFFFFFFFFu) {
     mbar_wait(&empty_bar[slot], ph ^ 1);
-    desc[slot] = TileDesc{shard, kind, n, flags};
+    desc[slot] = TileDesc{shard, kind, n, flags, lo, hi == 0xFFFFFFFFu ? n : hi, 0, 0};
     uint8_t* buf = ring + slot * SLOT;
     const uint32_t bytes = b0 + b1 + b2;
     if (bytes) {
@@ -190,10 +194,12 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     }
     if (++slot == kStages) { slot = 0; ph ^= 1; }
   };
+  // shards of this launch: one partition's range (multi-GPU) or all of them
+  const uint32_t q_lo = p.part >= 0 ? p.bounds[p.part] : 0u, q_hi = p.part >= 0 ? p.bounds[p.part + 1] : p.S;
   for (uint32_t round = 0;; ++round) {
-    // persistent grid: shards from the global queue; otherwise CTA b runs shard b only
-    const uint32_t s = kPersistent ? atomicAdd(&p.ctl->next_shard, 1u) : (round == 0 ? blockIdx.x : p.S);
-    if (s >= p.S) {
+    // persistent grid: shards from the global queue; otherwise CTA b runs shard q_lo + b only
+    const uint32_t s = q_lo + (kPersistent ? atomicAdd(&p.ctl->next_shard, 1u) : (round == 0 ? blockIdx.x : q_hi));
+    if (s >= q_hi) {
       push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
       return;
     }
@@ -213,13 +219,27 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
       send4 = *s_any != 0;
     }
     if (send4) {
-      const uint32_t kb = p.cw_off[s], ke = p.cw_off[s + 1];
-      if (kb == ke) push(s, kDescStage4, 0, kFlagLast, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
-      for (uint32_t k0 = kb; k0 < ke; k0 += kTile) {
-        const uint32_t n = min(kTile, ke - k0);
-        push(s, kDescStage4, n, k0 + n >= ke ? kFlagLast : 0u, p.cw_src + k0, n * 2, p.mapper + k0, 2 * kTile,
-             n * 4, nullptr, 0, 0);
+      // CW_s entries whose targets lie in the shard's own partition: all of
+      // CW_s on one GPU; with G partitions the other windows are refreshed
+      // after the exchange.  Tiles are 8-entry aligned for TMA; [lo, hi)
+      // marks the valid part of each tile.
+      uint32_t a, b2;
+      if (p.G > 1) {
+        const uint32_t o = p.owner[s];
+        a = p.cwp[(size_t)s * (p.G + 1) + o];
+        b2 = p.cwp[(size_t)s * (p.G + 1) + o + 1];
+      } else {
+        a = p.cw_off[s];
+        b2 = a + p.cw_cnt[s];
       }
+      const uint32_t kb = a & ~7u, ke = (b2 + 7u) & ~7u;
+      if (a >= b2) push(s, kDescStage4, 0, kFlagLast, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
+      else
+        for (uint32_t k0 = kb; k0 < ke; k0 += kTile) {
+          const uint32_t n = min(kTile, ke - k0);
+          push(s, kDescStage4, n, k0 + n >= ke ? kFlagLast : 0u, p.cw_src + k0, n * 2, p.mapper + k0, 2 * kTile,
+               n * 4, nullptr, 0, 0, a > k0 ? a - k0 : 0u, min(b2 - k0, n));
+        }
     }
   }
 }
@@ -333,6 +353,8 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
             up = A::update(sm, st, v, x[u], &out, &wbv, od[u]);
             if (up) vv[v] = out;
             if (!A::kMonotone) aux[v] = wbv;
+            // partitioned mode: publish the value stage 4 writes (the exchange payload)
+            if (p.gathered) p.gathered[off + v] = A::kMonotone ? sm[v] : wbv;
           }
           const uint32_t m = __ballot_sync(kFull, up);
           if (lane == 0 && m) atomicAdd(&s_upd, (uint32_t)__popc(m));
@@ -361,7 +383,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
             if (any) {
               const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
               const uint32_t* M = reinterpret_cast<const uint32_t*>(ring + slot * SLOT + 2 * kTile);
-              for (uint32_t i = ct; i < d.n; i += kConsumers) {
+              for (uint32_t i = d.lo + ct; i < d.hi; i += kConsumers) {
                 const uint32_t m = M[i];
                 uint32_t val;
                 if (m != trash && wb_get<A>(sm, aux, L[i], val)) { st_u32(p.srcvalue + m, val); ++stores; }
@@ -416,9 +438,49 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
       p.ctl->changed = 0;
       p.ctl->ctas_done = 0;
       p.ctl->next_shard = 0;
-      p.ctl->converged = changed ? 0u : 1u;
+      // with G partitions only the refresh after the exchange knows the global answer
+      if (p.G == 1) p.ctl->converged = changed ? 0u : 1u;
       __threadfence();
       if (p.use_cond) cudaGraphSetConditional(p.cond_handle, (changed && nit < p.ctl->max_iters) ? 1u : 0u);
+    }
+  }
+}
+
+// ------------------------------------------------- remote-window refresh (row e)
+// After a partitioned pass and the exchange of gathered[] (write-back values)
+// and active[] (which shards ran stage 4): for every active source shard i,
+// rewrite its windows in the partitions other than its owner's —
+// SrcValue[Mapper[k]] = gathered[i*N + SrcIndexCW[k]] over CW_i's sub-range
+// for that partition — then decide global convergence (no shard of any
+// partition active).  BSP across partitions, asynchronous within one.
+__global__ void __launch_bounds__(256) refresh_remote(const KParams p) {
+  __shared__ int s_act;
+  if (*reinterpret_cast<volatile uint32_t*>(&p.ctl->converged)) return;  // past convergence (host loop)
+  const uint32_t i = blockIdx.x;
+  if (threadIdx.x == 0) s_act = p.active[i];
+  __syncthreads();
+  if (s_act) {
+    const uint32_t oi = p.owner[i];
+    const uint32_t* row = p.cwp + (size_t)i * (p.G + 1);
+    const uint32_t* vals = p.gathered + (size_t)i * p.N;
+    for (uint32_t q = 0; q < p.G; ++q) {
+      if (q == oi || (p.part >= 0 && (int)q != p.part)) continue;
+      for (uint32_t k = row[q] + threadIdx.x; k < row[q + 1]; k += blockDim.x)
+        st_u32(p.srcvalue + __ldg(p.mapper + k), __ldg(vals + __ldg(p.cw_src + k)));
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    if (s_act) *reinterpret_cast<volatile uint32_t*>(&p.ctl->gchanged) = 1u;
+    __threadfence();
+    const uint32_t t = atomicAdd(&p.ctl->rctas_done, 1u);
+    if (t == gridDim.x - 1) {
+      __threadfence();
+      const uint32_t any = *reinterpret_cast<volatile uint32_t*>(&p.ctl->gchanged);
+      p.ctl->converged = any ? 0u : 1u;
+      p.ctl->gchanged = 0;
+      p.ctl->rctas_done = 0;
+      __threadfence();
     }
   }
 }
@@ -469,6 +531,8 @@ __global__ void reset_ctl(Ctl* ctl, uint32_t max_iters) {
   ctl->max_iters = max_iters;
   ctl->converged = 0;
   ctl->next_shard = 0;
+  ctl->gchanged = 0;
+  ctl->rctas_done = 0;
 }
 
 // -------------------------------------------------------------- dispatch
@@ -513,6 +577,8 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.srcloc = g.d_srcloc; p.win = g.d_win; p.cw_off = g.d_cw_off; p.cw_cnt = g.d_cw_cnt; p.active = g.d_active;
   p.cw_src = g.d_cw_src; p.mapper = g.d_mapper; p.vv = g.d_vv; p.outdeg = g.d_outdeg;
   p.ctl = g.d_ctl; p.trace = g.d_trace; p.trace_cap = g.trace_cap;
+  p.G = g.G; p.part = g.G > 1 && !g.simulate ? g.rank : -1;
+  p.bounds = g.d_bounds; p.owner = g.d_owner; p.cwp = g.d_cwp; p.gathered = g.G > 1 ? g.d_gathered : nullptr;
   p.use_cond = 0; p.cond_handle = 0;
   return p;
 }
@@ -541,6 +607,12 @@ cudaError_t launch_init(const Graph& g, int alg, uint32_t source, cudaStream_t s
     case kCS: return launch_init_t<AlgCS>(g, source, s);
   }
   return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_refresh(const Graph& g, cudaStream_t s) {
+  const KParams p = make_params(g, 0);
+  refresh_remote<<<g.S, 256, 0, s>>>(p);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_reset_ctl(Ctl* ctl, uint32_t max_iters, cudaStream_t s) {

@@ -103,6 +103,8 @@ def lib():
             "cusha_last_error": (ctypes.c_char_p, []),
             "cusha_abi_version": (i32, []),
             "cusha_nccl_unique_id": (i32, [P]),
+            "cusha_partition_shards": (i32, [u32, P, u32, P]),
+            "cusha_get_partition": (i32, [P, P, u32]),
         }
         for name, (res, args) in sigs.items():
             f = getattr(L, name)
@@ -169,10 +171,48 @@ class Graph:
         self.close()
 
 
+def _preload_nccl():
+    """libcusha dlopen()s libnccl.so.2; make torch's copy resolvable by that name."""
+    try:
+        import nvidia.nccl
+        p = os.path.join(list(nvidia.nccl.__path__)[0], "lib", "libnccl.so.2")
+        if os.path.exists(p):
+            ctypes.CDLL(p, mode=ctypes.RTLD_GLOBAL)
+    except Exception:
+        pass
+
+
+def nccl_unique_id() -> bytes:
+    """cusha_nccl_unique_id: 128 bytes for rank 0 to broadcast."""
+    _preload_nccl()
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().cusha_nccl_unique_id(buf), "cusha_nccl_unique_id")
+    return buf.raw
+
+
+def partition_shards(work, parts: int) -> np.ndarray:
+    """cusha_partition_shards (host logic): G+1 shard bounds of near-equal work."""
+    work = np.ascontiguousarray(work, dtype=np.uint64)
+    out = np.zeros(parts + 1, np.uint32)
+    _check(lib().cusha_partition_shards(len(work), _ptr(work), parts, _ptr(out)), "cusha_partition_shards")
+    return out
+
+
+def get_partition(g: "Graph") -> np.ndarray:
+    out = np.zeros(65, np.uint32)
+    k = lib().cusha_get_partition(g.handle, _ptr(out), 65)
+    if k < 0:
+        raise CushaError(k, "cusha_get_partition")
+    return out[:k + 1]
+
+
 def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertices_per_shard: int = 0,
                 smem_bytes_per_vertex: int = 0, device: int = 0, stream: Optional[int] = None,
-                host_loop: bool = False) -> Graph:
-    """cusha_build_graph.  src/dst/edge_values: numpy (host, copied in) or CUDA tensors (device)."""
+                host_loop: bool = False, world_size: int = 1, rank: int = 0,
+                nccl_id: Optional[bytes] = None) -> Graph:
+    """cusha_build_graph.  src/dst/edge_values: numpy (host, copied in) or CUDA tensors (device).
+    world_size > 1: destination-range partition; nccl_id = None simulates all
+    partitions on this device, else one process per GPU over NCCL."""
     on_dev = _is_device(src)
     if not on_dev:
         src = np.ascontiguousarray(src, dtype=np.uint32)
@@ -191,7 +231,15 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
     o.stream = stream
     o.input_location = INPUT_DEVICE if on_dev else INPUT_HOST
     o.host_loop = int(host_loop)
-    o.world_size = 1
+    o.world_size = world_size
+    o.rank = rank
+    idbuf = None
+    if nccl_id is not None:
+        if len(nccl_id) != 128:
+            raise ValueError("nccl_id must be 128 bytes")
+        _preload_nccl()
+        idbuf = ctypes.create_string_buffer(bytes(nccl_id), 128)
+        o.nccl_unique_id = ctypes.cast(idbuf, ctypes.c_void_p)
     h = ctypes.c_void_p()
     _check(lib().cusha_build_graph(num_vertices, len(src), _ptr(src), _ptr(dst), _ptr(edge_values),
                                    ctypes.byref(o), ctypes.byref(h)), "cusha_build_graph")
