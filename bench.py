@@ -203,17 +203,51 @@ def bench_cusha(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1:
-        raise SystemExit("multi-GPU bench: see DESIGN.md 'Multi-GPU' (not in this build yet)")
     torch.cuda.set_device(local)
     dev = local
+    dist = None
+    nccl_id = None
+    if world > 1:
+        # one process per GPU; the shard pass exchanges over NCCL inside libcusha
+        # (destination-range partition); torch.distributed only
+        # carries rank 0's ncclUniqueId, the barriers and the max-over-ranks time
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{dev}"))
+        idt = torch.zeros(128, dtype=torch.uint8, device=f"cuda:{dev}")
+        if rank == 0:
+            idt.copy_(torch.frombuffer(bytearray(cusha.nccl_unique_id()), dtype=torch.uint8))
+        dist.broadcast(idt, 0)
+        nccl_id = bytes(idt.cpu().numpy().tobytes())
     alg, repr_, source, desc = WORKLOADS[args.workload]
     if args.N == 0 and args.workload == "C1":
         args.N = 128  # the L310 rule gives 3 shards at this size
     if args.repr:
         repr_ = args.repr
+    if world > 1:
+        repr_ = "cw"  # the partitioned mode uses CW
     wl = load_graph(args.workload, args.cache_dir)
     stream = torch.cuda.current_stream()
+    part = dict(world_size=world, rank=rank, nccl_id=nccl_id)
+
+    def barrier():
+        if dist is not None:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def max_over_ranks(x):
+        if dist is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=f"cuda:{dev}")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def sum_over_ranks(x):
+        if dist is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=f"cuda:{dev}")
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return float(t.item())
+
     src_d = torch.from_numpy(wl.src.view(np.int32)).to(f"cuda:{dev}")
     dst_d = torch.from_numpy(wl.dst.view(np.int32)).to(f"cuda:{dev}")
     ev = None
@@ -221,14 +255,15 @@ def bench_cusha(args):
         ev = torch.from_numpy(wl.edge_u32.view(np.int32)).to(f"cuda:{dev}")
     torch.cuda.synchronize()
     g = cusha.build_graph(wl.V, src_d, dst_d, edge_values=ev, repr=repr_, vertices_per_shard=args.N, device=dev,
-                          stream=stream.cuda_stream, host_loop=args.host_loop)
+                          stream=stream.cuda_stream, host_loop=args.host_loop, **part)
     st0 = cusha.get_stats(g)
-    log(f"[bench] built {repr_} |N|={st0['vertices_per_shard']} |S|={st0['num_shards']} in {st0['build_ms']:.1f} ms")
+    log(f"[bench] rank {rank}/{world} built {repr_} |N|={st0['vertices_per_shard']} |S|={st0['num_shards']} "
+        f"in {st0['build_ms']:.1f} ms")
     del src_d, dst_d, ev
 
     for _ in range(args.warmup):
         cusha.run(alg, g, source=source)
-    torch.cuda.synchronize()
+    barrier()
     steps = []
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
@@ -241,14 +276,17 @@ def bench_cusha(args):
                           st["edges_processed"]))
         e1.record(stream)
         torch.cuda.synchronize()
+    barrier()
     clocks = clk.result()
-    total_ms = e0.elapsed_time(e1)
-    edges = sum(s[5] for s in steps)
+    total_ms = max_over_ranks(e0.elapsed_time(e1))  # device time, max over ranks
+    edges = sum(s[5] for s in steps)                 # whole graph: iterations x |E| per step
     iters = [s[1] for s in steps]
     loop_ms = sum(s[2] for s in steps)
     alg_bytes = sum(s[4] for s in steps)
     value = edges / (total_ms / 1e3) / 1e9
-    launches_per_step = [it + 3 for it in iters]       # reset_ctl + init_vertex_values + init_srcvalue + passes
+    # reset_ctl + init_vertex_values + init_srcvalue + one pass per iteration (+ one refresh when partitioned)
+    launches = sum(3 + it * (2 if world > 1 else 1) for it in iters)
+    launches = int(sum_over_ranks(launches))
     peak, peak_kind = measured_peak_gbs()
     achieved = alg_bytes / (loop_ms / 1e3) / 1e9
     st = cusha.get_stats(g)
@@ -270,7 +308,8 @@ def bench_cusha(args):
             # the user's call sequence: build from host buffers (H2D inside), run, read the result (D2H)
             gh = cusha.build_graph(wl.V, pin_s.numpy().view(np.uint32), pin_d.numpy().view(np.uint32),
                                    edge_values=None if pin_w is None else pin_w.numpy().view(np.uint32),
-                                   repr=repr_, vertices_per_shard=args.N, device=dev, stream=stream.cuda_stream)
+                                   repr=repr_, vertices_per_shard=args.N, device=dev, stream=stream.cuda_stream,
+                                   **part)
             cusha.run(alg, gh, source=source)
             n = cusha.get_stats(gh)["edges_processed"]
             rc = cusha.lib().cusha_get_values(gh.handle, cusha._ptr(out), wl.V * vb)
@@ -280,15 +319,15 @@ def bench_cusha(args):
 
         e2e_step()  # untimed warm-up (module loading, memory pool growth)
         e2e_edges = 0
-        torch.cuda.synchronize()
+        barrier()
         t0 = time.perf_counter()
         for _ in range(n_e2e):
             e2e_edges += e2e_step()
         torch.cuda.synchronize()
-        el = time.perf_counter() - t0
-        e2e = {"value": round(e2e_edges / el / 1e9, 4), "unit": "GTEPS", "h2d_bytes_per_step": h2d,
-               "d2h_bytes_per_step": wl.V * vb, "ms_per_step": round(el / n_e2e * 1e3, 3), "steps": n_e2e,
-               "warmup": 1}
+        el = max_over_ranks(time.perf_counter() - t0)
+        e2e = {"value": round(e2e_edges / el / 1e9, 4), "unit": "GTEPS", "h2d_bytes_per_step": h2d * world,
+               "d2h_bytes_per_step": wl.V * vb * world, "ms_per_step": round(el / n_e2e * 1e3, 3),
+               "steps": n_e2e, "warmup": 1}
 
     line = {
         "metric": "edges processed/sec (GTEPS) and time-to-convergence; shard-kernel HBM GB/s vs peak",
@@ -299,7 +338,7 @@ def bench_cusha(args):
         "warmup": args.warmup,
         "ms_per_step": round(total_ms / args.steps, 4),
         "higher_is_better": True,
-        "scaling": "weak",
+        "scaling": "strong",
         "vs_baseline": None,
         "dtype": "f32" if alg in ("pr", "nn", "hs", "cs") else "u32",
         "data": "synthetic",
@@ -308,14 +347,15 @@ def bench_cusha(args):
                    "iterations": iters[-1], "time_to_convergence_ms": round(total_ms / args.steps, 4),
                    "l2": f"inputs larger than L2: {per_iter_gb:.3f} GB streamed per fully-active pass vs 0.126 GB L2"
                    if per_iter_gb * 1e9 > L2_BYTES else f"L2-resident workload ({per_iter_gb*1e3:.1f} MB per pass); no flush",
-                   "build_ms": round(st0["build_ms"], 3), "parallelism": f"dp{world}"},
+                   "build_ms": round(st0["build_ms"], 3),
+                   "parallelism": f"destination-range partition x{world} (NCCL)" if world > 1 else "1 GPU"},
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                     "frac": round(achieved / peak, 4), "traffic": traffic_for(args.workload),
+                     "frac": round(achieved / peak, 4), "traffic": traffic_for(args.workload) if world == 1 else None,
                      "kernel": f"shard_pass<{alg},{repr_}>", "peak_kind": peak_kind,
                      "algorithmic_bytes_per_launch": int(alg_bytes / max(sum(iters), 1)),
                      "avg_launch_us": round(loop_ms / max(sum(iters), 1) * 1e3, 3)},
         "clocks": clocks,
-        "gpu_launches": int(sum(launches_per_step)),
+        "gpu_launches": launches,
         "e2e": e2e,
         "paper_context": {"hardware": "GTX 780 (Kepler), PCIe 3.0, CUDA 5.5 (L379)",
                           "table4_livejournal_pr_ms": {"CuSha-CW": 709, "CuSha-GS": 885, "VWC-CSR": "2814-3503"},
@@ -323,7 +363,11 @@ def bench_cusha(args):
     }
     if rank == 0 and not args.no_cpu_baseline and world == 1:
         line["cpu_baseline"] = cpu_baseline(wl, alg, source, budget_s=args.cpu_budget)
-    print(json.dumps(line), flush=True)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if dist is not None:
+        dist.barrier()
+        dist.destroy_process_group()
     return 0
 
 
