@@ -194,7 +194,7 @@ def workload(name: str, cache_dir: Optional[str] = None) -> Workload:
     else:
         raise KeyError(name)
     wl = Workload(name, V, src, dst, w)
-    if cache_dir:
+    if cache_dir and wl.E < (1 << 28):  # scale-26 lists (8.6 GB) are regenerated rather than cached
         os.makedirs(cache_dir, exist_ok=True)
         tmp = path + ".tmp%d.npz" % os.getpid()
         np.savez(tmp, V=np.int64(V), src=src, dst=dst, w=w if w is not None else np.zeros(0, np.uint32))

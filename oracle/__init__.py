@@ -50,6 +50,7 @@ def _L():
             "or_hs": [u64, u64, P, P, P, P, dbl, u64, P, P],
             "or_cs": [u64, u64, P, P, P, P, P, dbl, u64, P, P],
             "or_build_shards": [u64, u64, P, P, u32, P, P, P, P, P, P, P, P],
+            "or_pagerank_residual": [u64, u64, P, P, dbl, P, P],
         }
         for name, args in sig.items():
             f = getattr(lib, name)
@@ -114,6 +115,14 @@ def pagerank(V, src, dst, damping=0.85, tol=1e-9, max_iters=100000, allow_notcon
     _chk(_L().or_pagerank(V, len(src), _p(src), _p(dst), damping, tol, max_iters, _p(out), ctypes.byref(it)),
          "pagerank", allow_notconv=allow_notconv)
     return out, it.value
+
+
+def pagerank_residual(V, src, dst, x, damping=0.85):
+    """x_v - ((1-d) + d * sum_{u->v} x_u / outdeg(u)) for a given float32 rank vector."""
+    src, dst, x = _u32(src), _u32(dst), _f32(x)
+    out = np.empty(V, np.float64)
+    _chk(_L().or_pagerank_residual(V, len(src), _p(src), _p(dst), damping, _p(x), _p(out)), "pagerank_residual")
+    return out
 
 
 def nn(V, src, dst, weight, x0, tol=1e-9, max_iters=100000):

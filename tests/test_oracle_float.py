@@ -223,3 +223,19 @@ def test_cs_divider_closed_form():
     G = np.array([0.3, 0.3, 0.7, 0.7], np.float32)
     v, _ = oracle.cs(3, s, d, G, np.array([0, 0, 1], np.float32), np.array([1, 0, 1], np.float32), tol=1e-14)
     np.testing.assert_allclose(v, [0.0, np.float32(0.7) / (np.float64(np.float32(0.3)) + np.float32(0.7)), 1.0], atol=1e-12)
+
+
+def test_pr_residual_vs_dense_and_fixed_point():
+    """or_pagerank_residual: x - ((1-d) + d M x) equals the dense formula for
+    any x, and vanishes (to float32 rounding) at the oracle's fixed point."""
+    rng = np.random.default_rng(71)
+    V = 200
+    s, d = random_simple_graph(rng, V, 1500)
+    x = rng.uniform(0.1, 3.0, V).astype(np.float32)
+    out = np.bincount(s, minlength=V).astype(np.float64)
+    M = np.zeros((V, V))
+    np.add.at(M, (d, s), 1.0 / out[s])
+    want = x.astype(np.float64) - ((1 - D) + D * (M @ x.astype(np.float64)))
+    np.testing.assert_allclose(oracle.pagerank_residual(V, s, d, x), want, atol=1e-12)
+    xs, _ = oracle.pagerank(V, s, d, tol=1e-13)
+    assert np.abs(oracle.pagerank_residual(V, s, d, xs.astype(np.float32))).max() < 1e-5
