@@ -44,6 +44,13 @@ constexpr uint32_t kFull = 0xFFFFFFFFu;
 #ifndef CUSHA_MIN_BLOCKS
 #define CUSHA_MIN_BLOCKS 2
 #endif
+#ifndef CUSHA_GSU
+#define CUSHA_GSU 8
+#endif
+constexpr int kGSU = CUSHA_GSU;  // G-Shards write-back: SrcIndex loads in flight per lane
+#ifndef CUSHA_L2HINT
+#define CUSHA_L2HINT 0  // 1: evict-first on topology streams; 2: also on SrcValue reads
+#endif
 constexpr bool kPersistent = CUSHA_PERSISTENT != 0;  // grid = resident CTAs (queue) vs one CTA per shard
 #ifndef CUSHA_VB
 #define CUSHA_VB 8
@@ -125,18 +132,22 @@ __device__ __forceinline__ bool wb_get(const uint32_t* sm, const uint32_t* aux, 
 // ------------------------------------------------- G-Shards window walker
 // Visits every entry of the windows W_sj (j = 0..S-1) of source shard s:
 // each warp takes 32 windows at a time, scans their lengths across lanes and
-// walks the concatenation with one entry per lane (4 in flight), finding each
-// entry's window by a 5-step binary search over the lanes' prefix sums.
+// walks the concatenation with one entry per lane (kGSU in flight), finding
+// each entry's window by a 5-step binary search over the lanes' prefix sums.
+// The next batch's window bounds are loaded while the current one is walked.
 // fn(e, l): e = shard position, l = SrcIndex - s*N.
 template <class Fn>
 __device__ __forceinline__ void gs_walk(const KParams& p, uint32_t s, uint32_t lane, uint32_t warp, uint32_t nwarps,
                                         Fn&& fn) {
   const uint32_t* r0 = p.win + (size_t)s * p.S;
   const uint32_t* r1 = r0 + p.S;
+  uint32_t na = 0, nb = 0;
+  if (warp * 32 + lane < p.S) { na = __ldg(r0 + warp * 32 + lane); nb = __ldg(r1 + warp * 32 + lane); }
   for (uint32_t jb = warp * 32; jb < p.S; jb += nwarps * 32) {
-    const uint32_t j = jb + lane;
-    uint32_t a = 0, b = 0;
-    if (j < p.S) { a = __ldg(r0 + j); b = __ldg(r1 + j); }
+    const uint32_t a = na, b = nb;
+    const uint32_t jn = jb + nwarps * 32 + lane;
+    na = nb = 0;
+    if (jn < p.S) { na = __ldg(r0 + jn); nb = __ldg(r1 + jn); }
     const uint32_t len = b - a;
     uint32_t inc = len;
 #pragma unroll
@@ -146,10 +157,10 @@ __device__ __forceinline__ void gs_walk(const KParams& p, uint32_t s, uint32_t l
     }
     const uint32_t total = __shfl_sync(kFull, inc, 31);
     const uint32_t exc = inc - len;
-    for (uint32_t f0 = 0; f0 < total; f0 += 128) {
-      uint32_t e[4], l[4];
+    for (uint32_t f0 = 0; f0 < total; f0 += 32 * kGSU) {
+      uint32_t e[kGSU], l[kGSU];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
+      for (int u = 0; u < kGSU; ++u) {
         const uint32_t f = f0 + u * 32 + lane;
         int w = 0;
 #pragma unroll
@@ -161,7 +172,7 @@ __device__ __forceinline__ void gs_walk(const KParams& p, uint32_t s, uint32_t l
         l[u] = f < total ? (uint32_t)__ldg(p.srcloc + e[u]) : 0xFFFFFFFFu;
       }
 #pragma unroll
-      for (int u = 0; u < 4; ++u)
+      for (int u = 0; u < kGSU; ++u)
         if (l[u] != 0xFFFFFFFFu) fn(e[u], l[u]);
     }
   }
@@ -177,6 +188,7 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
   constexpr uint32_t SLOT = slot_bytes<A>();
   constexpr uint32_t kTile = tile_of<A>();
   uint32_t slot = 0, ph = 0, dph = 0;
+  const uint64_t pol = l2_evict_first_policy();
   auto push = [&](uint32_t shard, uint32_t kind, uint32_t n, uint32_t flags, const void* g0, uint32_t b0,
                   const void* g1, uint32_t o1, uint32_t b1, const void* g2, uint32_t o2, uint32_t b2,
                   uint32_t lo = 0, uint32_t hi = 0xFFFFFFFFu) {
@@ -186,9 +198,21 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     const uint32_t bytes = b0 + b1 + b2;
     if (bytes) {
       mbar_expect_tx(&full_bar[slot], bytes);
-      if (b0) bulk_g2s(buf, g0, b0, &full_bar[slot]);
-      if (b1) bulk_g2s(buf + o1, g1, b1, &full_bar[slot]);
-      if (b2) bulk_g2s(buf + o2, g2, b2, &full_bar[slot]);
+      // topology streams (DestIndex, EdgeValue, SrcIndexCW, Mapper) are read once per
+      // pass: evict-first; SrcValue (g0 of a stage-2 tile) keeps the default policy
+      const bool sv = kind == kDescStage2;
+      if (b0) {
+        if (CUSHA_L2HINT >= (sv ? 2 : 1)) bulk_g2s_hint(buf, g0, b0, &full_bar[slot], pol);
+        else bulk_g2s(buf, g0, b0, &full_bar[slot]);
+      }
+      if (b1) {
+        if (CUSHA_L2HINT >= 1) bulk_g2s_hint(buf + o1, g1, b1, &full_bar[slot], pol);
+        else bulk_g2s(buf + o1, g1, b1, &full_bar[slot]);
+      }
+      if (b2) {
+        if (CUSHA_L2HINT >= 1) bulk_g2s_hint(buf + o2, g2, b2, &full_bar[slot], pol);
+        else bulk_g2s(buf + o2, g2, b2, &full_bar[slot]);
+      }
     } else {
       mbar_arrive(&full_bar[slot]);
     }
