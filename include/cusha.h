@@ -216,7 +216,9 @@ typedef enum {
   CUSHA_LAYOUT_CW_SIZES = 7,        /* u32[|S|]   real entries of CW_i                      */
   CUSHA_LAYOUT_CW_SRC_LOCAL = 8,    /* u16[Q]     SrcIndex - i*|N| per padded CW entry      */
   CUSHA_LAYOUT_MAPPER = 9,          /* u32[Q]     padded shard position (filler = trash P)  */
-  CUSHA_LAYOUT_OUT_DEGREE = 10      /* u32[|V|]   out-degree (PR NbrsNum, L318)            */
+  CUSHA_LAYOUT_OUT_DEGREE = 10,     /* u32[|V|]   out-degree (PR NbrsNum, L318)            */
+  CUSHA_LAYOUT_RUN_K = 11,          /* u32[R]     CW position of each Mapper run's first entry (CW) */
+  CUSHA_LAYOUT_RUN_T = 12           /* u32[R]     its Mapper target; one run per non-empty W_ij      */
 } cusha_layout_part;
 /* Returns the element count of `part` in *count (bytes = count * element size);
  * copies it to `out` (host) when out != NULL and out_bytes is large enough.

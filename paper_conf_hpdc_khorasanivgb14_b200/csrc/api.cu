@@ -42,7 +42,8 @@ static int fail(int code, const std::string& msg) {
 static void free_graph_memory(Graph& g) {
   void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcloc, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
                   g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_srcvalue, g.d_vv, g.d_ctl, g.d_trace,
-                  g.d_active, g.d_bounds, g.d_owner, g.d_cwp, g.d_gathered};
+                  g.d_active, g.d_bounds, g.d_owner, g.d_cwp, g.d_gathered, g.d_run_k, g.d_run_t,
+                  g.d_run_unit, g.d_run_bits, g.d_run_d};
   nccl_destroy(g);
   // device memory is stream-ordered (cudaMallocAsync on g.stream): released to
   // the retained pool without unmapping or a device-wide synchronisation
@@ -500,6 +501,8 @@ int cusha_get_layout(const cusha_graph* h, cusha_layout_part part, void* out, si
     case CUSHA_LAYOUT_CW_SRC_LOCAL: src = g.d_cw_src; n = g.Q; es = 2; break;
     case CUSHA_LAYOUT_MAPPER: src = g.d_mapper; n = g.Q; break;
     case CUSHA_LAYOUT_OUT_DEGREE: src = g.d_outdeg; n = g.V; break;
+    case CUSHA_LAYOUT_RUN_K: src = g.d_run_k; n = g.R; break;
+    case CUSHA_LAYOUT_RUN_T: src = g.d_run_t; n = g.R; break;
     default: return fail(CUSHA_EINVAL, "bad layout part");
   }
   if (!src) return fail(CUSHA_EUNSUPPORTED, "part not held by this representation");

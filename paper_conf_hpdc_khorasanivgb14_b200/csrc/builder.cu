@@ -230,7 +230,98 @@ cudaError_t dalloc(T** p, uint64_t n) {
   return cudaMallocAsync(reinterpret_cast<void**>(p), (n ? n : 1) * sizeof(T), t_alloc_stream);
 }
 
+// ---- run-length form of Mapper
+// Within a window W_ij the Mapper targets of CW_i are consecutive shard
+// positions (CW_i lists W_ij in shard order, L175, and W_ij is contiguous in
+// shard j, L155), so Mapper is a run per non-empty window:
+//   RunK[r] = CW position of the run's first entry, RunT[r] = its target.
+// RunUnit[u] = last run with RunK <= u*kRunUnit (locates a tile's runs).
+__global__ void k_win_len(const uint32_t* __restrict__ win, uint32_t S, uint32_t* len, uint32_t* nonempty) {
+  GRID_STRIDE(t, (uint64_t)S * S) {
+    const uint32_t l = win[t + S] - win[t];  // row i = t / S, column j
+    len[t] = l;
+    nonempty[t] = l ? 1u : 0u;
+  }
+}
+__global__ void k_runs(const uint32_t* __restrict__ win, const uint32_t* len, const uint32_t* pos, const uint32_t* ridx,
+                       const uint32_t* cw_off, uint32_t S, uint32_t* run_k, uint32_t* run_t) {
+  GRID_STRIDE(t, (uint64_t)S * S) {
+    if (!len[t]) continue;
+    const uint32_t i = (uint32_t)(t / S);
+    const uint32_t r = ridx[t];
+    run_k[r] = cw_off[i] + (pos[t] - pos[(size_t)i * S]);
+    run_t[r] = win[t];
+  }
+}
+__global__ void k_run_pad(uint32_t R, uint32_t Rpad, uint32_t* run_k, uint32_t* run_t) {
+  GRID_STRIDE(r, (uint64_t)Rpad) {
+    if (r >= R) { run_k[r] = 0xFFFFFFFFu; run_t[r] = 0; }
+  }
+}
+__global__ void k_run_delta(const uint32_t* run_k, const uint32_t* run_t, uint64_t n, uint32_t* run_d) {
+  GRID_STRIDE(r, n) run_d[r] = run_t[r] - run_k[r];
+}
+__global__ void k_run_bits(const uint32_t* __restrict__ run_k, uint32_t R, uint32_t* bits) {
+  GRID_STRIDE(r, (uint64_t)R) atomicOr(&bits[run_k[r] >> 5], 1u << (run_k[r] & 31));
+}
+__global__ void k_run_unit(const uint32_t* __restrict__ run_k, uint32_t R, uint64_t U, uint32_t* unit) {
+  GRID_STRIDE(u, U) {
+    const uint64_t pos = u * kRunUnit;
+    uint32_t lo = 0, hi = R;  // first run with run_k > pos
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if ((uint64_t)run_k[mid] <= pos) lo = mid + 1;
+      else hi = mid;
+    }
+    unit[u] = lo ? lo - 1 : 0;
+  }
+}
+
 }  // namespace
+
+int build_runs(Graph& g, std::string& err) {
+  cudaStream_t st = g.stream;
+  t_alloc_stream = st;
+  const uint32_t S = g.S;
+  const uint64_t S2 = (uint64_t)S * S;
+  DevBuf len, nonempty, pos, ridx, t1, t2;
+  CK(dalloc((uint32_t**)&len.p, S2));
+  CK(dalloc((uint32_t**)&nonempty.p, S2));
+  CK(dalloc((uint32_t**)&pos.p, S2));
+  CK(dalloc((uint32_t**)&ridx.p, S2 + 1));
+  k_win_len<<<grid_for(S2), 256, 0, st>>>(g.d_win, S, (uint32_t*)len.p, (uint32_t*)nonempty.p);
+  CK(cudaGetLastError());
+  size_t b1 = 0, b2 = 0;
+  CK(cub::DeviceScan::ExclusiveSum(nullptr, b1, (uint32_t*)len.p, (uint32_t*)pos.p, (int64_t)S2, st));
+  CK(cudaMallocAsync(&t1.p, b1 ? b1 : 1, st));
+  CK(cub::DeviceScan::ExclusiveSum(t1.p, b1, (uint32_t*)len.p, (uint32_t*)pos.p, (int64_t)S2, st));
+  CK(cub::DeviceScan::InclusiveSum(nullptr, b2, (uint32_t*)nonempty.p, (uint32_t*)ridx.p + 1, (int64_t)S2, st));
+  CK(cudaMallocAsync(&t2.p, b2 ? b2 : 1, st));
+  CK(cudaMemsetAsync(ridx.p, 0, 4, st));
+  CK(cub::DeviceScan::InclusiveSum(t2.p, b2, (uint32_t*)nonempty.p, (uint32_t*)ridx.p + 1, (int64_t)S2, st));
+  uint32_t R = 0;
+  CK(cudaMemcpyAsync(&R, (uint32_t*)ridx.p + S2, 4, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  g.R = R;
+  const uint64_t Rpad = ((uint64_t)R + 3) / 4 * 4 + 8;  // TMA copies round run ranges to 4 (16 B)
+  CK(dalloc(&g.d_run_k, Rpad));
+  CK(dalloc(&g.d_run_t, Rpad));
+  k_run_pad<<<grid_for(Rpad), 256, 0, st>>>(R, (uint32_t)Rpad, g.d_run_k, g.d_run_t);
+  k_runs<<<grid_for(S2), 256, 0, st>>>(g.d_win, (uint32_t*)len.p, (uint32_t*)pos.p, (uint32_t*)ridx.p, g.d_cw_off, S,
+                                       g.d_run_k, g.d_run_t);
+  const uint64_t U = g.Q / kRunUnit + 2;
+  CK(dalloc(&g.d_run_unit, U + 4));  // + 4: 16-byte TMA slices rounded up
+  k_run_unit<<<grid_for(U), 256, 0, st>>>(g.d_run_k, R, U, g.d_run_unit);
+  const uint64_t W = g.Q / 32 + 16;  // run-start bitmap (+ slack for 128-entry aligned TMA slices)
+  CK(dalloc(&g.d_run_bits, W));
+  CK(cudaMemsetAsync(g.d_run_bits, 0, W * 4, st));
+  k_run_bits<<<grid_for(R), 256, 0, st>>>(g.d_run_k, R, g.d_run_bits);
+  CK(dalloc(&g.d_run_d, Rpad));
+  k_run_delta<<<grid_for(Rpad), 256, 0, st>>>(g.d_run_k, g.d_run_t, Rpad, g.d_run_d);
+  CK(cudaGetLastError());
+  CK(cudaStreamSynchronize(st));
+  return CUSHA_OK;
+}
 
 int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const uint32_t* d_val, std::string& err) {
   cudaStream_t st = g.stream;
@@ -385,8 +476,11 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
     // CW keeps the 3-tuple shards + SrcIndexCW + Mapper (L175): no per-entry SrcIndex in shard order
     cudaFreeAsync(g.d_srcloc, st);
     g.d_srcloc = nullptr;
+    pt.mark("CW offsets + scatter");
+    const int rc = build_runs(g, err);
+    if (rc) return rc;
   }
-  pt.mark("CW offsets + scatter");
+  pt.mark("Mapper runs");
   CK(cudaStreamSynchronize(st));
   return CUSHA_OK;
 }

@@ -10,6 +10,8 @@
 
 namespace cusha {
 
+constexpr uint32_t kRunUnit = 128;  // CW positions per entry of the Mapper-run locator (RunUnit)
+
 // Iteration control word block (row a5), one per graph, device resident.
 struct Ctl {
   uint32_t iter;        // shard passes completed in this run
@@ -58,6 +60,13 @@ struct KParams {
   const uint8_t* owner;        // S: partition owning shard s
   const uint32_t* cwp;         // S*(G+1): CW_i entries whose targets lie in partition p = [cwp[i][p], cwp[i][p+1])
   uint32_t* gathered;          // V: write-back value of every vertex after its last pass (exchanged)
+  // Mapper in run-length form (CW): one run per non-empty window
+  const uint32_t* run_k;       // R (+pad): CW position of each run's first entry (sorted)
+  const uint32_t* run_t;       // R (+pad): target shard position of that entry
+  const uint32_t* run_unit;    // Q/kRunUnit+2: last run starting at or before u*kRunUnit
+  const uint32_t* run_bits;    // Q/32 (+pad): bit k = a run starts at CW position k
+  const uint32_t* run_d;       // R (+pad): RunT - RunK (mod 2^32): target(k) = k + run_d[run of k]
+  uint32_t R;
 };
 
 struct PassKernel {
@@ -91,6 +100,12 @@ struct Graph {
   uint8_t* d_active = nullptr;      // S: stage-4 prefetch predictor
   uint16_t* d_cw_src = nullptr;     // Q (CW)
   uint32_t* d_mapper = nullptr;     // Q (CW)
+  uint32_t R = 0;                   // Mapper runs (non-empty windows)
+  uint32_t* d_run_k = nullptr;      // R+pad
+  uint32_t* d_run_t = nullptr;      // R+pad
+  uint32_t* d_run_unit = nullptr;   // Q/kRunUnit+2
+  uint32_t* d_run_bits = nullptr;   // Q/32 + pad
+  uint32_t* d_run_d = nullptr;      // R+pad
   uint32_t* d_outdeg = nullptr;     // V
   // per-run state
   uint32_t* d_srcvalue = nullptr;   // P+1
@@ -131,6 +146,7 @@ bool alg_needs_init(int alg);
 // builder.cu
 int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const uint32_t* d_val, std::string& err);
 int build_partition(Graph& g, std::string& err);  // bounds, owner, cwp, gathered (G > 1)
+int build_runs(Graph& g, std::string& err);       // Mapper runs (CW)
 void partition_bounds(uint32_t S, const uint64_t* work, uint32_t G, uint32_t* bounds);
 
 // api.cu

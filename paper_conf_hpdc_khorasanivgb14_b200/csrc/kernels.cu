@@ -59,6 +59,10 @@ constexpr bool kPersistent = CUSHA_PERSISTENT != 0;  // grid = resident CTAs (qu
 #define CUSHA_SPEC 1
 #endif
 constexpr uint32_t kVB = CUSHA_VB;                   // vertex loads in flight per thread in stages 1 and 3
+#ifndef CUSHA_EPT
+#define CUSHA_EPT 4
+#endif
+constexpr uint32_t kEPT = CUSHA_EPT;  // stage-2 entries per consumer thread per step (4 or 8)
 constexpr uint32_t kConsumerWarps = CUSHA_CONSUMER_WARPS;
 constexpr uint32_t kConsumers = kConsumerWarps * 32;
 constexpr uint32_t kPassThreads = kConsumers + 32;  // + 1 producer warp
@@ -76,14 +80,32 @@ template <class A>
 constexpr uint32_t slot_bytes() {
   return tile_of<A>() * (6 + (A::kEdge ? 4 : 0));
 }
+// run-start bitmap words a stage-4 slot carries (tile starts are 8-aligned;
+// the 16-byte TMA copy is aligned to 128 entries)
+template <class A>
+constexpr uint32_t bits_words() {
+  return tile_of<A>() / 32 + 8;
+}
+// Mapper runs (RunT - RunK, 4 B each) a stage-4 slot holds after SrcIndexCW and the bitmap
+template <class A>
+constexpr uint32_t run_cap() {
+  return (slot_bytes<A>() - 2 * tile_of<A>() - 4 * bits_words<A>()) / 4 / 4 * 4;
+}
+#ifndef CUSHA_RLE
+#define CUSHA_RLE 0  // measured slower (the pass is consumer-bound): DESIGN.md "Tuning log"
+#endif
+constexpr bool kRle = CUSHA_RLE != 0;  // stream Mapper as runs
 
-enum : uint32_t { kDescStage2 = 0, kDescStage4 = 1, kDescDone = 2 };
+// stage-4 tile kinds: kDescStage4 carries SrcIndexCW + Mapper per entry;
+// kDescStage4R carries SrcIndexCW + the Mapper runs overlapping the tile.
+enum : uint32_t { kDescStage2 = 0, kDescStage4 = 1, kDescDone = 2, kDescStage4R = 3 };
 enum : uint32_t { kFlagLast = 1, kFlagSpec4 = 2 };
 // flags: kFlagLast = last tile of this stage; kFlagSpec4 (on a shard's first
 // tile) = stage-4 tiles of this shard follow its stage-2 tiles.  n = entries
-// copied into the slot; [lo, hi) = the entries the consumers use.
+// copied into the slot; [lo, hi) = the entries the consumers use; base = CW
+// position of entry 0 of the slot; nruns = runs in the slot (kDescStage4R).
 struct __align__(16) TileDesc {
-  uint32_t shard, kind, n, flags, lo, hi, pad0, pad1;
+  uint32_t shard, kind, n, flags, lo, hi, base, nruns;
 };
 
 // ------------------------------------------------------------ stage 2 body
@@ -110,6 +132,36 @@ __device__ __forceinline__ void proc4(uint32_t* sm, uint32_t st, const uint4& sv
       for (int a = 0; a < A::kAcc; ++a) {
         const uint32_t l = (uint32_t)F[k][a];
         const uint32_t h = (uint32_t)(F[k][a] >> 32) + ((old[k][a] + l < old[k][a]) ? 1u : 0u);  // carry
+        if (h) atomicAdd(&sm[(A::acc_lo(a) + 1) * st + D[k]], h);
+      }
+  }
+}
+
+template <class A>
+__device__ __forceinline__ void proc8(uint32_t* sm, uint32_t st, const uint4& s0, const uint4& s1, const uint4& dd,
+                                      const uint4& e0, const uint4& e1) {
+  const uint32_t D[8] = {dd.x & 0xFFFFu, dd.x >> 16, dd.y & 0xFFFFu, dd.y >> 16,
+                         dd.z & 0xFFFFu, dd.z >> 16, dd.w & 0xFFFFu, dd.w >> 16};
+  const uint32_t S[8] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
+  const uint32_t W[8] = {e0.x, e0.y, e0.z, e0.w, e1.x, e1.y, e1.z, e1.w};
+  if constexpr (A::kAcc == 0) {
+#pragma unroll
+    for (int k = 0; k < 8; ++k) A::compute(sm, st, D[k], S[k], W[k]);
+  } else {
+    uint64_t F[8][2];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) A::contrib(sm, st, D[k], S[k], W[k], F[k]);
+    uint32_t old[8][2];
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+#pragma unroll
+      for (int a = 0; a < A::kAcc; ++a) old[k][a] = atomicAdd(&sm[A::acc_lo(a) * st + D[k]], (uint32_t)F[k][a]);
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+#pragma unroll
+      for (int a = 0; a < A::kAcc; ++a) {
+        const uint32_t l = (uint32_t)F[k][a];
+        const uint32_t h = (uint32_t)(F[k][a] >> 32) + ((old[k][a] + l < old[k][a]) ? 1u : 0u);
         if (h) atomicAdd(&sm[(A::acc_lo(a) + 1) * st + D[k]], h);
       }
   }
@@ -187,17 +239,20 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
                                          uint64_t* empty_bar, uint64_t* decide_bar, const volatile int* s_any) {
   constexpr uint32_t SLOT = slot_bytes<A>();
   constexpr uint32_t kTile = tile_of<A>();
+  constexpr uint32_t kRunCap = run_cap<A>();
   uint32_t slot = 0, ph = 0, dph = 0;
   const uint64_t pol = l2_evict_first_policy();
   auto push = [&](uint32_t shard, uint32_t kind, uint32_t n, uint32_t flags, const void* g0, uint32_t b0,
                   const void* g1, uint32_t o1, uint32_t b1, const void* g2, uint32_t o2, uint32_t b2,
-                  uint32_t lo = 0, uint32_t hi = 0xFFFFFFFFu) {
+                  uint32_t lo = 0, uint32_t hi = 0xFFFFFFFFu, uint32_t base = 0, uint32_t nruns = 0,
+                  const void* g3 = nullptr, uint32_t o3 = 0, uint32_t b3 = 0) {
     mbar_wait(&empty_bar[slot], ph ^ 1);
-    desc[slot] = TileDesc{shard, kind, n, flags, lo, hi == 0xFFFFFFFFu ? n : hi, 0, 0};
+    desc[slot] = TileDesc{shard, kind, n, flags, lo, hi == 0xFFFFFFFFu ? n : hi, base, nruns};
     uint8_t* buf = ring + slot * SLOT;
-    const uint32_t bytes = b0 + b1 + b2;
+    const uint32_t bytes = b0 + b1 + b2 + b3;
     if (bytes) {
       mbar_expect_tx(&full_bar[slot], bytes);
+      if (b3) bulk_g2s(buf + o3, g3, b3, &full_bar[slot]);
       // topology streams (DestIndex, EdgeValue, SrcIndexCW, Mapper) are read once per
       // pass: evict-first; SrcValue (g0 of a stage-2 tile) keeps the default policy
       const bool sv = kind == kDescStage2;
@@ -229,6 +284,21 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     }
     const bool spec = CUSHA_SPEC && REPR == CUSHA_REPR_CW && p.active[s];
     const uint32_t b = p.shard_off[s], e = p.shard_off[s + 1];
+    // CW_s entries whose targets lie in the shard's own partition: all of CW_s
+    // on one GPU; with G partitions the other windows are refreshed after the
+    // exchange.  Stage-4 tiles are 8-entry aligned for TMA.
+    uint32_t a = 0, b2 = 0;
+    if (REPR == CUSHA_REPR_CW) {
+      if (p.G > 1) {
+        const uint32_t o = p.owner[s];
+        a = p.cwp[(size_t)s * (p.G + 1) + o];
+        b2 = p.cwp[(size_t)s * (p.G + 1) + o + 1];
+      } else {
+        a = p.cw_off[s];
+        b2 = a + p.cw_cnt[s];
+      }
+    }
+    const uint32_t kb = a & ~7u, ke = (b2 + 7u) & ~7u;
     if (b == e) push(s, kDescStage2, 0, kFlagLast | (spec ? kFlagSpec4 : 0u), nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
     for (uint32_t t0 = b; t0 < e; t0 += kTile) {
       const uint32_t n = min(kTile, e - t0);
@@ -243,26 +313,29 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
       send4 = *s_any != 0;
     }
     if (send4) {
-      // CW_s entries whose targets lie in the shard's own partition: all of
-      // CW_s on one GPU; with G partitions the other windows are refreshed
-      // after the exchange.  Tiles are 8-entry aligned for TMA; [lo, hi)
-      // marks the valid part of each tile.
-      uint32_t a, b2;
-      if (p.G > 1) {
-        const uint32_t o = p.owner[s];
-        a = p.cwp[(size_t)s * (p.G + 1) + o];
-        b2 = p.cwp[(size_t)s * (p.G + 1) + o + 1];
-      } else {
-        a = p.cw_off[s];
-        b2 = a + p.cw_cnt[s];
-      }
-      const uint32_t kb = a & ~7u, ke = (b2 + 7u) & ~7u;
+      // [lo, hi) marks the valid part of each tile
       if (a >= b2) push(s, kDescStage4, 0, kFlagLast, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
       else
         for (uint32_t k0 = kb; k0 < ke; k0 += kTile) {
           const uint32_t n = min(kTile, ke - k0);
-          push(s, kDescStage4, n, k0 + n >= ke ? kFlagLast : 0u, p.cw_src + k0, n * 2, p.mapper + k0, 2 * kTile,
-               n * 4, nullptr, 0, 0, a > k0 ? a - k0 : 0u, min(b2 - k0, n));
+          const uint32_t fl = k0 + n >= ke ? kFlagLast : 0u, lo = a > k0 ? a - k0 : 0u, hi = min(b2 - k0, n);
+          if (kRle) {
+            // runs from the one containing position k0/128*128 (the slot's first
+            // bitmap position) through the last starting inside the tile; the
+            // TMA copy starts 4-aligned, so that run sits at list index ra - ra4
+            const uint32_t ra = p.run_unit[k0 / kRunUnit];
+            const uint32_t rb = min(p.R, p.run_unit[(k0 + n - 1) / kRunUnit + 1] + 1);
+            const uint32_t ra4 = ra & ~3u, nr = ((rb + 3u) & ~3u) - ra4;
+            if (nr <= kRunCap) {
+              // slot: SrcIndexCW | RunT-RunK per run | run-start bitmap words [k0/128*4, ceil((k0+n)/128)*4)
+              const uint32_t wa = k0 / 128 * 4, wz = (k0 + n + 127) / 128 * 4;
+              push(s, kDescStage4R, n, fl | ((ra - ra4) << 8), p.cw_src + k0, n * 2, p.run_d + ra4, 2 * kTile,
+                   nr * 4, p.run_bits + wa, 2 * kTile + 4 * kRunCap, (wz - wa) * 4, lo, hi, k0, nr);
+              continue;
+            }
+          }
+          push(s, kDescStage4, n, fl, p.cw_src + k0, n * 2, p.mapper + k0, 2 * kTile, n * 4, nullptr, 0, 0, lo, hi,
+               k0, 0);
         }
     }
   }
@@ -337,6 +410,19 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
       // ---- stage 2: the shard's entries from the ring, compute() into shared memory (lines 12-13, L269)
       for (;;) {
         const uint8_t* buf = ring + slot * SLOT;
+        if (kEPT == 8) {
+          for (uint32_t i = ct * 8; i < d.n; i += kConsumers * 8) {  // n is a multiple of 8
+            const uint4 sv0 = *reinterpret_cast<const uint4*>(buf + 4 * i);
+            const uint4 sv1 = *reinterpret_cast<const uint4*>(buf + 4 * i + 16);
+            const uint4 dd = *reinterpret_cast<const uint4*>(buf + 4 * kTile + 2 * i);
+            uint4 ev0 = make_uint4(0, 0, 0, 0), ev1 = ev0;
+            if (A::kEdge) {
+              ev0 = *reinterpret_cast<const uint4*>(buf + 6 * kTile + 4 * i);
+              ev1 = *reinterpret_cast<const uint4*>(buf + 6 * kTile + 4 * i + 16);
+            }
+            proc8<A>(sm, st, sv0, sv1, dd, ev0, ev1);
+          }
+        } else
         for (uint32_t i = ct * 4; i < d.n; i += kConsumers * 4) {
           const uint4 sv = *reinterpret_cast<const uint4*>(buf + 4 * i);
           const uint2 dd = *reinterpret_cast<const uint2*>(buf + 4 * kTile + 2 * i);
@@ -404,7 +490,45 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
           for (;;) {
             mbar_wait(&full_bar[slot], ph);
             d = desc[slot];
-            if (any) {
+            if (any && d.kind == kDescStage4R) {
+              // Mapper from runs: target(k) = k + D[r], D = RunT - RunK, for the run r
+              // containing CW position k.  Runs start where the run-start bitmap has
+              // a 1.  List entry (flags >> 8) is the run containing P = the slot's
+              // first bitmap position, so for x >= P the run of position x - 1 is
+              // that index + popc(bits in [P, x)) - bit(P).  Each warp takes a
+              // contiguous block of 32-aligned strips, seeds its count with one
+              // warp-wide popcount reduction, and lane i adds popc(word & bits <= i).
+              const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
+              const uint32_t* D = reinterpret_cast<const uint32_t*>(ring + slot * SLOT + 2 * kTile);
+              const uint32_t* BW = D + run_cap<A>();
+              const uint32_t wbase = d.base / 128 * 4;                  // word index of BW[0]
+              const uint32_t alo = d.base + d.lo, ahi = d.base + d.hi;  // valid CW positions
+              const uint32_t first = alo & ~31u;
+              const uint32_t nstrips = (ahi - first + 31) / 32;
+              const uint32_t per = (nstrips + kConsumerWarps - 1) / kConsumerWarps;
+              const uint32_t s0 = first + cwarp * per * 32;
+              const uint32_t s1 = min(first + (cwarp + 1) * per * 32, ahi);
+              if (s0 < s1) {
+                const uint32_t nw = s0 / 32 - wbase;  // bitmap words before the warp's block
+                uint32_t c = 0;
+                for (uint32_t w = lane; w < nw; w += 32) c += __popc(BW[w]);
+                c = __reduce_add_sync(kFull, c);
+                int r = (int)((d.flags >> 8) & 3u) + (int)c - (int)(BW[0] & 1u);  // run of position s0 - 1
+                const uint32_t below = (2u << lane) - 1u;                          // bits 0..lane
+#pragma unroll 4
+                for (uint32_t sp = s0; sp < s1; sp += 32) {
+                  const uint32_t word = BW[sp / 32 - wbase];
+                  const int ri = r + __popc(word & below);
+                  const uint32_t k = sp + lane;
+                  uint32_t val;
+                  if (k >= alo && k < ahi && wb_get<A>(sm, aux, L[k - d.base], val)) {
+                    st_u32(p.srcvalue + (k + D[ri]), val);
+                    ++stores;
+                  }
+                  r += __popc(word);
+                }
+              }
+            } else if (any) {
               const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
               const uint32_t* M = reinterpret_cast<const uint32_t*>(ring + slot * SLOT + 2 * kTile);
               for (uint32_t i = d.lo + ct; i < d.hi; i += kConsumers) {
@@ -603,6 +727,8 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.ctl = g.d_ctl; p.trace = g.d_trace; p.trace_cap = g.trace_cap;
   p.G = g.G; p.part = g.G > 1 && !g.simulate ? g.rank : -1;
   p.bounds = g.d_bounds; p.owner = g.d_owner; p.cwp = g.d_cwp; p.gathered = g.G > 1 ? g.d_gathered : nullptr;
+  p.run_k = g.d_run_k; p.run_t = g.d_run_t; p.run_unit = g.d_run_unit; p.run_bits = g.d_run_bits; p.run_d = g.d_run_d;
+  p.R = g.R;
   p.use_cond = 0; p.cond_handle = 0;
   return p;
 }

@@ -30,7 +30,7 @@ LAYOUT = {
     "shard_offsets": (0, np.uint32), "shard_sizes": (1, np.uint32), "src_index": (2, np.uint16),
     "dest_local": (3, np.uint16), "edge_id": (4, np.uint32), "windows": (5, np.uint32),
     "cw_offsets": (6, np.uint32), "cw_sizes": (7, np.uint32), "cw_src_local": (8, np.uint16),
-    "mapper": (9, np.uint32), "out_degree": (10, np.uint32),
+    "mapper": (9, np.uint32), "out_degree": (10, np.uint32), "run_k": (11, np.uint32), "run_t": (12, np.uint32),
 }
 
 

@@ -175,6 +175,8 @@ def test_layout_matches_oracle(repr, V, E, N):
             cw_off = cusha.get_layout(g, "cw_offsets").astype(np.int64)
             cw_src = cusha.get_layout(g, "cw_src_local")
             mapper = cusha.get_layout(g, "mapper").astype(np.int64)
+            run_k = cusha.get_layout(g, "run_k").astype(np.int64)
+            run_t = cusha.get_layout(g, "run_t").astype(np.int64)
     assert st["num_shards"] == S and st["vertices_per_shard"] == N
     np.testing.assert_array_equal(cnt, np.diff(ref["shard_off"].astype(np.int64)))
     assert (off % 8 == 0).all()
@@ -202,6 +204,13 @@ def test_layout_matches_oracle(repr, V, E, N):
         np.testing.assert_array_equal(cw_src[creal].astype(np.int64) + src_shard * N, ref["cw_src"])
         cfill = np.setdiff1d(np.arange(len(mapper)), creal)
         assert (mapper[cfill] == off[-1]).all()
+        # Mapper runs: one per non-empty window, and expanding them gives Mapper exactly
+        Wlen = np.diff(ref["win"].astype(np.int64), axis=0)
+        assert len(run_k) == int((Wlen > 0).sum())
+        assert (np.diff(run_k) > 0).all()
+        if E:
+            r = np.searchsorted(run_k, creal, side="right") - 1
+            np.testing.assert_array_equal(run_t[r] + (creal - run_k[r]), mapper[creal])
 
 
 # ----------------------------------------------------------- edge cases
