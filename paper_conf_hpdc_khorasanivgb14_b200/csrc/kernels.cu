@@ -58,6 +58,9 @@ constexpr bool kPersistent = CUSHA_PERSISTENT != 0;  // grid = resident CTAs (qu
 #ifndef CUSHA_SPEC
 #define CUSHA_SPEC 1
 #endif
+#ifndef CUSHA_SPEC_ALWAYS
+#define CUSHA_SPEC_ALWAYS 0  // 1: prefetch CW stage-4 tiles for every shard (dropped when it stays idle)
+#endif
 constexpr uint32_t kVB = CUSHA_VB;                   // vertex loads in flight per thread in stages 1 and 3
 #ifndef CUSHA_EPT
 #define CUSHA_EPT 4
@@ -282,7 +285,7 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
       push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
       return;
     }
-    const bool spec = CUSHA_SPEC && REPR == CUSHA_REPR_CW && p.active[s];
+    const bool spec = CUSHA_SPEC && REPR == CUSHA_REPR_CW && (CUSHA_SPEC_ALWAYS || p.active[s]);
     const uint32_t b = p.shard_off[s], e = p.shard_off[s + 1];
     // CW_s entries whose targets lie in the shard's own partition: all of CW_s
     // on one GPU; with G partitions the other windows are refreshed after the
