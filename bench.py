@@ -31,12 +31,13 @@ WORKLOADS = {
     "C2": ("pr", "cw", 0, "PageRank (d=0.85, eps=1e-5) on LiveJournal-shaped R-MAT 4,847,571 V / 68,993,773 E, CW"),
     "C3": ("sssp", "cw", 0, "SSSP on RoadNet-CA-shaped mesh 1,971,281 V / 5,533,214 E, CW"),
     "C3gs": ("sssp", "gs", 0, "SSSP on RoadNet-CA-shaped mesh 1,971,281 V / 5,533,214 E, G-Shards"),
+    "C3o": ("sssp", "cw", 0, "SSSP on the C3 mesh in natural (row-major) vertex order, CW"),
     "C4cc": ("cc", "cw", 0, "CC on HiggsTwitter-shaped symmetric R-MAT 456,631 V / 14,855,874 E"),
     "C4sswp": ("sswp", "cw", 0, "SSWP on HiggsTwitter-shaped symmetric R-MAT 456,631 V / 14,855,874 E"),
     "C5pr": ("pr", "cw", 0, "PageRank on R-MAT scale 26 (67,108,864 V / 1,073,741,824 E)"),
     "C5bfs": ("bfs", "cw", 0, "BFS on R-MAT scale 26 (67,108,864 V / 1,073,741,824 E)"),
 }
-GRAPH_OF = {"C1": "C1", "C2": "C2", "C3": "C3", "C3gs": "C3", "C4cc": "C4", "C4sswp": "C4", "C5pr": "C5", "C5bfs": "C5"}
+GRAPH_OF = {"C1": "C1", "C2": "C2", "C3": "C3", "C3gs": "C3", "C3o": "C3o", "C4cc": "C4", "C4sswp": "C4", "C5pr": "C5", "C5bfs": "C5"}
 L2_BYTES = 126 * 1024 * 1024
 
 
@@ -255,7 +256,8 @@ def bench_cusha(args):
         ev = torch.from_numpy(wl.edge_u32.view(np.int32)).to(f"cuda:{dev}")
     torch.cuda.synchronize()
     g = cusha.build_graph(wl.V, src_d, dst_d, edge_values=ev, repr=repr_, vertices_per_shard=args.N, device=dev,
-                          stream=stream.cuda_stream, host_loop=args.host_loop, **part)
+                          stream=stream.cuda_stream, host_loop=args.host_loop,
+                          skip_clean_shards=args.skip_clean, **part)
     st0 = cusha.get_stats(g)
     log(f"[bench] rank {rank}/{world} built {repr_} |N|={st0['vertices_per_shard']} |S|={st0['num_shards']} "
         f"in {st0['build_ms']:.1f} ms")
@@ -279,7 +281,7 @@ def bench_cusha(args):
     barrier()
     clocks = clk.result()
     total_ms = max_over_ranks(e0.elapsed_time(e1))  # device time, max over ranks
-    edges = sum(s[5] for s in steps)                 # whole graph: iterations x |E| per step
+    edges = sum_over_ranks(sum(s[5] for s in steps))  # each rank streams its partition's edges
     iters = [s[1] for s in steps]
     loop_ms = sum(s[2] for s in steps)
     alg_bytes = sum(s[4] for s in steps)
@@ -309,7 +311,7 @@ def bench_cusha(args):
             gh = cusha.build_graph(wl.V, pin_s.numpy().view(np.uint32), pin_d.numpy().view(np.uint32),
                                    edge_values=None if pin_w is None else pin_w.numpy().view(np.uint32),
                                    repr=repr_, vertices_per_shard=args.N, device=dev, stream=stream.cuda_stream,
-                                   **part)
+                                   skip_clean_shards=args.skip_clean, **part)
             cusha.run(alg, gh, source=source)
             n = cusha.get_stats(gh)["edges_processed"]
             rc = cusha.lib().cusha_get_values(gh.handle, cusha._ptr(out), wl.V * vb)
@@ -325,6 +327,7 @@ def bench_cusha(args):
             e2e_edges += e2e_step()
         torch.cuda.synchronize()
         el = max_over_ranks(time.perf_counter() - t0)
+        e2e_edges = sum_over_ranks(e2e_edges)
         e2e = {"value": round(e2e_edges / el / 1e9, 4), "unit": "GTEPS", "h2d_bytes_per_step": h2d * world,
                "d2h_bytes_per_step": wl.V * vb * world, "ms_per_step": round(el / n_e2e * 1e3, 3),
                "steps": n_e2e, "warmup": 1}
@@ -348,6 +351,7 @@ def bench_cusha(args):
                    "l2": f"inputs larger than L2: {per_iter_gb:.3f} GB streamed per fully-active pass vs 0.126 GB L2"
                    if per_iter_gb * 1e9 > L2_BYTES else f"L2-resident workload ({per_iter_gb*1e3:.1f} MB per pass); no flush",
                    "build_ms": round(st0["build_ms"], 3),
+                   "skip_clean_shards": bool(args.skip_clean),
                    "parallelism": f"destination-range partition x{world} (NCCL)" if world > 1 else "1 GPU"},
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                      "frac": round(achieved / peak, 4), "traffic": traffic_for(args.workload) if world == 1 else None,
@@ -384,6 +388,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--host-loop", action="store_true", help="host-launched passes (for ncu); default: device loop")
     ap.add_argument("--lib", default=None, help="alternative libcusha.so (tuning variants)")
+    ap.add_argument("--skip-clean", action="store_true",
+                    help="opt-in exact clean-shard skipping (not the paper's full passes; off by default)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0)

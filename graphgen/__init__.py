@@ -168,6 +168,12 @@ def workload(name: str, cache_dir: Optional[str] = None) -> Workload:
         V = 1_971_281
         src, dst = mesh(V, 1404, 2_766_607, seed=3)
         w = edge_u32(src, dst, seed=3, lo=1, hi=255, symmetric=True)
+    elif name == "C3o":
+        # C3 in the mesh's natural row-major vertex order (no id permutation):
+        # shards are bands of rows, as in a road network numbered by locality
+        V = 1_971_281
+        src, dst = mesh(V, 1404, 2_766_607, seed=3, permute=False)
+        w = edge_u32(src, dst, seed=3, lo=1, hi=255, symmetric=True)
     elif name == "C4":
         V = 456_631
         src, dst = rmat(V, 7_427_937, seed=4, symmetric=True)

@@ -42,7 +42,7 @@ extern "C" {
 #define CUSHA_API
 #endif
 
-#define CUSHA_ABI_VERSION 1
+#define CUSHA_ABI_VERSION 2
 
 /* Return codes. */
 enum {
@@ -102,6 +102,15 @@ typedef struct {
   int world_size;                  /* 1 = single partition (0 is treated as 1)                  */
   int rank;                        /* this process's rank, 0..world_size-1 (NCCL mode)          */
   const void* nccl_unique_id;      /* 128-byte ncclUniqueId, or NULL (see above)                */
+  /* Clean-shard skipping (opt-in; not in the paper, which processes every
+   * shard in every iteration, Fig. 5 line 3 / L189).  1: a shard none of whose
+   * windows was written since its own last pass is skipped — it would
+   * recompute the values it holds and commit nothing (exact for all eight
+   * algorithms; HS shards that committed re-run, their local state reads
+   * their own Q).  Results are identical; passes can differ only in that
+   * skipped shards do no work.  cusha_stats.edges_processed counts the edges
+   * actually streamed.  Default 0 = the paper's full passes.              */
+  int skip_clean_shards;
 } cusha_build_opts;
 
 typedef struct cusha_graph cusha_graph;   /* opaque; owns all device memory it allocates */
@@ -125,7 +134,9 @@ typedef struct {
   uint64_t stage2_bytes_per_iter;  /* algorithmic bytes stage 2 streams per iteration          */
   uint64_t wb_bytes_all_active;    /* stage-4 algorithmic bytes if every shard is active       */
   uint64_t algorithmic_bytes;      /* last run: sum over iterations of stage1..4 algorithmic bytes */
-  uint64_t edges_processed;        /* last run: iterations * |E|                                */
+  uint64_t edges_processed;        /* last run: edges streamed by stage 2 over all passes of this
+                                      process's shards (iterations * |E| unless shards were
+                                      skipped or partitioned)                                 */
   uint32_t device_loop;            /* 1 = the run looped on the device (CUDA-graph while node) */
   int world_size, rank;
 } cusha_stats;

@@ -43,7 +43,7 @@ static void free_graph_memory(Graph& g) {
   void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcloc, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
                   g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_srcvalue, g.d_vv, g.d_ctl, g.d_trace,
                   g.d_active, g.d_bounds, g.d_owner, g.d_cwp, g.d_gathered, g.d_run_k, g.d_run_t,
-                  g.d_run_unit, g.d_run_bits, g.d_run_d};
+                  g.d_run_unit, g.d_run_bits, g.d_run_d, g.d_dirty};
   nccl_destroy(g);
   // device memory is stream-ordered (cudaMallocAsync on g.stream): released to
   // the retained pool without unmapping or a device-wide synchronisation
@@ -151,6 +151,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   Graph& g = h->g;
   g.V = V; g.E = E; g.N = N; g.S = (V + N - 1) / N; g.repr = (int)o.repr; g.device = o.device;
   g.host_loop = o.host_loop != 0;
+  g.skip_clean = o.skip_clean_shards != 0;
   g.world_size = o.world_size;
   g.rank = o.world_size > 1 && o.nccl_unique_id ? o.rank : 0;
   g.simulate = o.world_size > 1 && !o.nccl_unique_id;
@@ -407,11 +408,14 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   const uint32_t n = std::min(c.iter, g.trace_cap);
   TraceRec* tr = new TraceRec[n ? n : 1];
   CKA(cudaMemcpy(tr, g.d_trace, sizeof(TraceRec) * n, cudaMemcpyDeviceToHost));
-  uint64_t bytes = 0;
+  uint64_t bytes = 0, edges = 0;
   for (uint32_t i = 0; i < n; ++i) {
-    bytes += g.V * vb + (a == kPR ? 4ull * g.V : 0);                 // stages 1+3 reads
+    // vertices of the processed shards (all of V unless clean shards were skipped)
+    const uint64_t nv = std::min<uint64_t>(g.V, tr[i].shards * (uint64_t)g.N);
+    bytes += nv * vb + (a == kPR ? 4ull * nv : 0);                    // stages 1+3 reads
     bytes += (uint64_t)tr[i].updated * vb;                            // stage 3 commits
-    bytes += g.E * (4 + 2 + evb);                                     // stage 2
+    bytes += tr[i].edges * (4 + 2 + evb);                             // stage 2
+    edges += tr[i].edges;
     if (g.repr == CUSHA_REPR_CW)
       bytes += tr[i].wb_entries * 6 + tr[i].wb_stores * 4;            // SrcIndexCW + Mapper, SrcValue
     else
@@ -424,7 +428,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   g.st.loop_ms = lms;
   g.st.last_algorithm = a;
   g.st.algorithmic_bytes = bytes;
-  g.st.edges_processed = (uint64_t)c.iter * g.E;
+  g.st.edges_processed = n == c.iter ? edges : (uint64_t)c.iter * g.E;
   g.st.stage2_bytes_per_iter = g.E * (4 + 2 + evb);
   g.st.wb_bytes_all_active = g.repr == CUSHA_REPR_CW ? g.E * 10 : g.E * 8;
   g.st.device_loop = g.host_loop ? 0 : 1;

@@ -30,12 +30,15 @@ struct TraceRec {
   uint32_t active_shards;    // shards that ran stage 4
   unsigned long long wb_entries;  // CW / window entries visited by stage 4
   unsigned long long wb_stores;   // SrcValue words actually stored by stage 4
+  unsigned long long edges;       // edges streamed by stage 2 (|E| unless clean shards are skipped)
+  unsigned long long shards;      // shards processed (|S| unless clean shards are skipped)
 };
 
 // Everything a shard-pass launch needs (passed by value).
 struct KParams {
   uint32_t V, N, S, source;
   const uint32_t* shard_off;   // S+1 padded start positions
+  const uint32_t* shard_cnt;   // S real entry counts
   const uint16_t* dest;        // P local DestIndex (filler = N)
   const uint32_t* ev;          // P EdgeValue or null
   uint32_t* srcvalue;          // P+1 (slot P = trash for CW filler)
@@ -67,6 +70,9 @@ struct KParams {
   const uint32_t* run_bits;    // Q/32 (+pad): bit k = a run starts at CW position k
   const uint32_t* run_d;       // R (+pad): RunT - RunK (mod 2^32): target(k) = k + run_d[run of k]
   uint32_t R;
+  // opt-in exact work skipping
+  int skip;                    // 1: a shard none of whose windows was written since its last pass is skipped
+  uint32_t* dirty;             // S: some window of shard j written since j's last pass (set by writers)
 };
 
 struct PassKernel {
@@ -98,6 +104,8 @@ struct Graph {
   uint32_t* d_cw_off = nullptr;     // S+1
   uint32_t* d_cw_cnt = nullptr;     // S
   uint8_t* d_active = nullptr;      // S: stage-4 prefetch predictor
+  uint32_t* d_dirty = nullptr;      // S: clean-shard skipping flags
+  bool skip_clean = false;
   uint16_t* d_cw_src = nullptr;     // Q (CW)
   uint32_t* d_mapper = nullptr;     // Q (CW)
   uint32_t R = 0;                   // Mapper runs (non-empty windows)

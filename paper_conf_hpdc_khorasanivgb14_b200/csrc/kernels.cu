@@ -98,6 +98,14 @@ constexpr uint32_t run_cap() {
 #define CUSHA_RLE 0  // measured slower (the pass is consumer-bound): DESIGN.md "Tuning log"
 #endif
 constexpr bool kRle = CUSHA_RLE != 0;  // stream Mapper as runs
+#ifndef CUSHA_DIAG
+#define CUSHA_DIAG 0
+#endif
+// Diagnostic variants for the per-stage cost split (tools/diag_pass.py; never
+// the product, results are wrong by design): bit 0 = every shard active in
+// every pass (no convergence), bit 1 = no stage-2 reduction, bit 2 = no
+// stage-4 stores.
+constexpr uint32_t kDiag = CUSHA_DIAG;
 
 // stage-4 tile kinds: kDescStage4 carries SrcIndexCW + Mapper per entry;
 // kDescStage4R carries SrcIndexCW + the Mapper runs overlapping the tile.
@@ -285,6 +293,19 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
       push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
       return;
     }
+    if (p.skip) {
+      // clean-shard skipping (opt-in): no
+      // window of shard s was written since its last pass, so stages 1-3 would
+      // recompute the values it already holds and commit nothing.  Clearing the
+      // flag before the tiles are read means a write landing after this point
+      // re-marks s for a later pass.
+      if (atomicExch(&p.dirty[s], 0u) == 0u) {
+        p.active[s] = 0;
+        continue;
+      }
+      __threadfence();                                      // acquire the writers' SrcValue stores ...
+      asm volatile("fence.proxy.async.global;" ::: "memory");  // ... for the TMA (async-proxy) reads below
+    }
     const bool spec = CUSHA_SPEC && REPR == CUSHA_REPR_CW && (CUSHA_SPEC_ALWAYS || p.active[s]);
     const uint32_t b = p.shard_off[s], e = p.shard_off[s + 1];
     // CW_s entries whose targets lie in the shard's own partition: all of CW_s
@@ -431,7 +452,11 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
           const uint2 dd = *reinterpret_cast<const uint2*>(buf + 4 * kTile + 2 * i);
           uint4 ev = make_uint4(0, 0, 0, 0);
           if (A::kEdge) ev = *reinterpret_cast<const uint4*>(buf + 6 * kTile + 4 * i);
-          proc4<A>(sm, st, sv, dd, ev);
+          if (kDiag & 2) {
+            if ((sv.x ^ sv.y ^ sv.z ^ sv.w ^ dd.x ^ dd.y ^ ev.x) == 0x9e3779b9u) sm[N] = 1u;  // keep the loads
+          } else {
+            proc4<A>(sm, st, sv, dd, ev);
+          }
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty_bar[slot]);
@@ -476,7 +501,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
           my_upd |= up ? 1u : 0u;
         }
       }
-      const int any = bar_sync_or(kConsumerBar, kConsumers, (int)my_upd);
+      const int any = bar_sync_or(kConsumerBar, kConsumers, (int)my_upd) | ((kDiag & 1) ? 1 : 0);
 
       // ---- stage 4: write-back into every shard's window (lines 23-26, L308)
       uint32_t stores = 0;
@@ -537,7 +562,14 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
               for (uint32_t i = d.lo + ct; i < d.hi; i += kConsumers) {
                 const uint32_t m = M[i];
                 uint32_t val;
-                if (m != trash && wb_get<A>(sm, aux, L[i], val)) { st_u32(p.srcvalue + m, val); ++stores; }
+                if (m != trash && wb_get<A>(sm, aux, L[i], val)) {
+                  if (kDiag & 4) {
+                    if (val == 0x9e3779b9u && m == 7u) st_u32(p.srcvalue + m, val);  // keep the loads
+                  } else {
+                    st_u32(p.srcvalue + m, val);
+                  }
+                  ++stores;
+                }
               }
             }
             __syncwarp();
@@ -557,10 +589,26 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
 #pragma unroll
       for (int o = 16; o; o >>= 1) stores += __shfl_xor_sync(kFull, stores, o);
       if (lane == 0 && stores) atomicAdd(&s_stores, (unsigned long long)stores);
+      if (p.skip && any) __threadfence();  // release: SrcValue stores before the dirty marks below
       bar_sync(kConsumerBar, kConsumers);
+
+      if (p.skip && any) {
+        // mark every shard j fed by a non-empty window W_sj (own partition; the
+        // refresh marks the others) and, where local state reads the vertex's
+        // own value (HS), shard s itself
+        const uint32_t* w0 = p.win + (size_t)s * p.S;
+        const uint32_t* w1 = w0 + p.S;
+        for (uint32_t j = ct; j < p.S; j += kConsumers)
+          if (__ldg(w1 + j) > __ldg(w0 + j) && (p.G == 1 || p.owner[j] == p.owner[s])) p.dirty[j] = 1u;
+        if (A::kId == kHS && ct == 0) p.dirty[s] = 1u;
+      }
 
       // ---- per-shard bookkeeping: convergence flag (line 26), predictor, trace
       if (ct == 0) {
+        if (it < p.trace_cap) {
+          atomicAdd(&p.trace[it].edges, (unsigned long long)p.shard_cnt[s]);
+          atomicAdd(&p.trace[it].shards, 1ull);
+        }
         p.active[s] = any ? 1 : 0;
         if (any) {
           *reinterpret_cast<volatile uint32_t*>(&p.ctl->changed) = 1u;
@@ -618,6 +666,9 @@ __global__ void __launch_bounds__(256) refresh_remote(const KParams p) {
       if (q == oi || (p.part >= 0 && (int)q != p.part)) continue;
       for (uint32_t k = row[q] + threadIdx.x; k < row[q + 1]; k += blockDim.x)
         st_u32(p.srcvalue + __ldg(p.mapper + k), __ldg(vals + __ldg(p.cw_src + k)));
+      if (p.skip)  // the refreshed shards of partition q have new inputs
+        for (uint32_t j = p.bounds[q] + threadIdx.x; j < p.bounds[q + 1]; j += blockDim.x)
+          if (__ldg(p.win + (size_t)(i + 1) * p.S + j) > __ldg(p.win + (size_t)i * p.S + j)) p.dirty[j] = 1u;
     }
   }
   __syncthreads();
@@ -646,8 +697,10 @@ __global__ void init_vertex_values(const KParams p, const void* user) {
   const V_t* u = reinterpret_cast<const V_t*>(user);
   for (size_t v = blockIdx.x * (size_t)blockDim.x + threadIdx.x; v < p.V; v += (size_t)gridDim.x * blockDim.x)
     vv[v] = u ? u[v] : A::start((uint32_t)v, p.source);
-  for (size_t s = blockIdx.x * (size_t)blockDim.x + threadIdx.x; s < p.S; s += (size_t)gridDim.x * blockDim.x)
+  for (size_t s = blockIdx.x * (size_t)blockDim.x + threadIdx.x; s < p.S; s += (size_t)gridDim.x * blockDim.x) {
     p.active[s] = 1;
+    if (p.dirty) p.dirty[s] = 1u;  // every shard runs the first pass
+  }
 }
 
 // SrcValue[e] <- VertexValues[SrcIndex[e]] for every entry (R20: a full
@@ -724,7 +777,7 @@ bool alg_needs_init(int alg) { return alg == kNN || alg == kHS || alg == kCS; }
 KParams make_params(const Graph& g, uint32_t source) {
   KParams p{};
   p.V = g.V; p.N = g.N; p.S = g.S; p.source = source;
-  p.shard_off = g.d_shard_off; p.dest = g.d_dest; p.ev = g.d_ev; p.srcvalue = g.d_srcvalue;
+  p.shard_off = g.d_shard_off; p.shard_cnt = g.d_shard_cnt; p.dest = g.d_dest; p.ev = g.d_ev; p.srcvalue = g.d_srcvalue;
   p.srcloc = g.d_srcloc; p.win = g.d_win; p.cw_off = g.d_cw_off; p.cw_cnt = g.d_cw_cnt; p.active = g.d_active;
   p.cw_src = g.d_cw_src; p.mapper = g.d_mapper; p.vv = g.d_vv; p.outdeg = g.d_outdeg;
   p.ctl = g.d_ctl; p.trace = g.d_trace; p.trace_cap = g.trace_cap;
@@ -732,6 +785,7 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.bounds = g.d_bounds; p.owner = g.d_owner; p.cwp = g.d_cwp; p.gathered = g.G > 1 ? g.d_gathered : nullptr;
   p.run_k = g.d_run_k; p.run_t = g.d_run_t; p.run_unit = g.d_run_unit; p.run_bits = g.d_run_bits; p.run_d = g.d_run_d;
   p.R = g.R;
+  p.skip = g.skip_clean ? 1 : 0; p.dirty = g.d_dirty;
   p.use_cond = 0; p.cond_handle = 0;
   return p;
 }

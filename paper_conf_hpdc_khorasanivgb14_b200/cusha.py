@@ -46,6 +46,7 @@ class BuildOpts(ctypes.Structure):
         ("world_size", ctypes.c_int),
         ("rank", ctypes.c_int),
         ("nccl_unique_id", ctypes.c_void_p),
+        ("skip_clean_shards", ctypes.c_int),
     ]
 
 
@@ -209,10 +210,11 @@ def get_partition(g: "Graph") -> np.ndarray:
 def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertices_per_shard: int = 0,
                 smem_bytes_per_vertex: int = 0, device: int = 0, stream: Optional[int] = None,
                 host_loop: bool = False, world_size: int = 1, rank: int = 0,
-                nccl_id: Optional[bytes] = None) -> Graph:
+                nccl_id: Optional[bytes] = None, skip_clean_shards: bool = False) -> Graph:
     """cusha_build_graph.  src/dst/edge_values: numpy (host, copied in) or CUDA tensors (device).
     world_size > 1: destination-range partition; nccl_id = None simulates all
-    partitions on this device, else one process per GPU over NCCL."""
+    partitions on this device, else one process per GPU over NCCL.
+    skip_clean_shards: opt-in exact skipping of shards whose inputs did not change."""
     on_dev = _is_device(src)
     if not on_dev:
         src = np.ascontiguousarray(src, dtype=np.uint32)
@@ -233,6 +235,7 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
     o.host_loop = int(host_loop)
     o.world_size = world_size
     o.rank = rank
+    o.skip_clean_shards = int(skip_clean_shards)
     idbuf = None
     if nccl_id is not None:
         if len(nccl_id) != 128:
