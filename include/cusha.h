@@ -111,6 +111,17 @@ typedef struct {
    * skipped shards do no work.  cusha_stats.edges_processed counts the edges
    * actually streamed.  Default 0 = the paper's full passes.              */
   int skip_clean_shards;
+  /* Host-streamed topology (row f3; the multi-streamed procedure of L455 for
+   * graphs whose representation does not fit in HBM).  0 = every array in HBM
+   * (default).  Otherwise at most this many bytes of HBM hold the per-entry
+   * topology arrays (DestIndex, EdgeValue, SrcIndex, edge ids; CW: SrcIndexCW,
+   * Mapper): shards 0..h-1 keep theirs in HBM, shards h..S-1 (h =
+   * cusha_stats.host_shard) keep theirs in pinned, mapped host memory, and
+   * every pass streams them over the host link through the same TMA ring that
+   * streams HBM tiles, overlapping the transfer with the shard computation.
+   * SrcValue, VertexValues and the O(|V| + |S|^2) arrays stay in HBM.  Results
+   * are identical to the in-HBM layout.  The build itself runs in HBM first.  */
+  uint64_t device_topology_budget;
 } cusha_build_opts;
 
 typedef struct cusha_graph cusha_graph;   /* opaque; owns all device memory it allocates */
@@ -139,6 +150,8 @@ typedef struct {
                                       skipped or partitioned)                                 */
   uint32_t device_loop;            /* 1 = the run looped on the device (CUDA-graph while node) */
   int world_size, rank;
+  uint64_t host_bytes;             /* per-entry topology bytes held in pinned host memory (f3)  */
+  uint32_t host_shard;             /* first shard whose topology is host-resident (|S|: none)   */
 } cusha_stats;
 
 /* ---------------------------------------------------------------- build */

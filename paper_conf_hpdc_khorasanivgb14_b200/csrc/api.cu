@@ -51,6 +51,9 @@ static void free_graph_memory(Graph& g) {
     if (p) cudaFreeAsync(p, g.stream);
   for (void*& p : g.d_init)
     if (p) { cudaFreeAsync(p, g.stream); p = nullptr; }
+  void* hosts[] = {g.h_dest, g.h_ev, g.h_srcloc, g.h_eid, g.h_cw_src, g.h_mapper};
+  for (void* p : hosts)
+    if (p) cudaFreeHost(p);
   delete g.h_ctl;
   g.h_ctl = nullptr;
   if (g.ev0) cudaEventDestroy(g.ev0);
@@ -81,7 +84,7 @@ static uint64_t device_bytes(const Graph& g) {
   b += (2 + 4) * g.Q;                                   // CW
   b += 4ull * g.V;                                      // outdeg
   b += 4 * (g.P + 1) + 8ull * g.V;                      // SrcValue + VertexValues
-  return b;
+  return b - g.host_bytes;                              // minus the host-streamed part (row f3)
 }
 
 }  // namespace cusha
@@ -152,6 +155,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   g.V = V; g.E = E; g.N = N; g.S = (V + N - 1) / N; g.repr = (int)o.repr; g.device = o.device;
   g.host_loop = o.host_loop != 0;
   g.skip_clean = o.skip_clean_shards != 0;
+  g.topo_budget = o.device_topology_budget;
   g.world_size = o.world_size;
   g.rank = o.world_size > 1 && o.nccl_unique_id ? o.rank : 0;
   g.simulate = o.world_size > 1 && !o.nccl_unique_id;
@@ -217,6 +221,12 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
       return bail(rc);
     }
   }
+  rc = offload_topology(g, err);  // row f3 (no-op without a budget)
+  if (rc) {
+    cudaEventDestroy(eh);
+    set_error("host topology: " + err);
+    return bail(rc);
+  }
   // per-run state: SrcValue (P entries + trash slot), VertexValues (8 B/vertex covers every Table-3 Vertex)
   g.h_ctl = new (std::nothrow) Ctl();
   if ((rc = cu(cudaMallocAsync(&g.d_srcvalue, 4 * (g.P + 1), g.stream), "cudaMallocAsync(SrcValue)")) ||
@@ -247,6 +257,8 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   g.st.entries_padded = g.P;
   g.st.world_size = g.world_size;
   g.st.rank = g.rank;
+  g.st.host_bytes = g.host_bytes;
+  g.st.host_shard = g.host_shard;
   *out = h;
   set_error("");
   return CUSHA_OK;
@@ -491,30 +503,33 @@ int cusha_get_layout(const cusha_graph* h, cusha_layout_part part, void* out, si
   if (!h) return fail(CUSHA_EINVAL, "graph is NULL");
   const Graph& g = h->g;
   const void* src = nullptr;
-  uint64_t n = 0;
+  const void* tail = nullptr;  // host-resident part (row f3) from position `split`
+  uint64_t n = 0, split = ~0ull;
   size_t es = 4;
   switch (part) {
     case CUSHA_LAYOUT_SHARD_OFFSETS: src = g.d_shard_off; n = (uint64_t)g.S + 1; break;
     case CUSHA_LAYOUT_SHARD_SIZES: src = g.d_shard_cnt; n = g.S; break;
-    case CUSHA_LAYOUT_SRC_INDEX: src = g.d_srcloc; n = g.P; es = 2; break;
-    case CUSHA_LAYOUT_DEST_LOCAL: src = g.d_dest; n = g.P; es = 2; break;
-    case CUSHA_LAYOUT_EDGE_ID: src = g.d_eid; n = g.P; break;
+    case CUSHA_LAYOUT_SRC_INDEX: src = g.d_srcloc; tail = g.h_srcloc; split = g.splitP; n = g.P; es = 2; break;
+    case CUSHA_LAYOUT_DEST_LOCAL: src = g.d_dest; tail = g.h_dest; split = g.splitP; n = g.P; es = 2; break;
+    case CUSHA_LAYOUT_EDGE_ID: src = g.d_eid; tail = g.h_eid; split = g.splitP; n = g.P; break;
     case CUSHA_LAYOUT_WINDOWS: src = g.d_win; n = ((uint64_t)g.S + 1) * g.S; break;
     case CUSHA_LAYOUT_CW_OFFSETS: src = g.d_cw_off; n = (uint64_t)g.S + 1; break;
     case CUSHA_LAYOUT_CW_SIZES: src = g.d_cw_cnt; n = g.S; break;
-    case CUSHA_LAYOUT_CW_SRC_LOCAL: src = g.d_cw_src; n = g.Q; es = 2; break;
-    case CUSHA_LAYOUT_MAPPER: src = g.d_mapper; n = g.Q; break;
+    case CUSHA_LAYOUT_CW_SRC_LOCAL: src = g.d_cw_src; tail = g.h_cw_src; split = g.splitQ; n = g.Q; es = 2; break;
+    case CUSHA_LAYOUT_MAPPER: src = g.d_mapper; tail = g.h_mapper; split = g.splitQ; n = g.Q; break;
     case CUSHA_LAYOUT_OUT_DEGREE: src = g.d_outdeg; n = g.V; break;
     case CUSHA_LAYOUT_RUN_K: src = g.d_run_k; n = g.R; break;
     case CUSHA_LAYOUT_RUN_T: src = g.d_run_t; n = g.R; break;
     default: return fail(CUSHA_EINVAL, "bad layout part");
   }
-  if (!src) return fail(CUSHA_EUNSUPPORTED, "part not held by this representation");
+  if (!src && !tail) return fail(CUSHA_EUNSUPPORTED, "part not held by this representation");
   if (count) *count = n;
   if (!out) return CUSHA_OK;
   if (out_bytes < n * es) return fail(CUSHA_EINVAL, "out_bytes too small");
   CKA(cudaSetDevice(g.device));
-  CKA(cudaMemcpy(out, src, n * es, cudaMemcpyDeviceToHost));
+  const uint64_t nd = std::min(n, split);  // HBM part
+  if (nd) CKA(cudaMemcpy(out, src, nd * es, cudaMemcpyDeviceToHost));
+  if (nd < n) std::memcpy(static_cast<char*>(out) + nd * es, tail, (n - nd) * es);
   return CUSHA_OK;
 }
 

@@ -9,16 +9,17 @@
 //
 // G-Shards order = lexicographic (shard(dst), src, dst, input index): one
 // stable radix sort of the packed key (shard(dst) | src | dst mod N) — the
-// input index tie-break (R17) comes from the sort's stability.  CW order =
-// stable sort of the G-Shards positions by source shard (positions inside one
-// source shard are already in (j, position) order, which is exactly W_i0,
-// W_i1, ... concatenated).
+// input index tie-break (R17) comes from the sort's stability.  CW needs no
+// second sort: CW_i is by definition W_i0, W_i1, ..., W_i(S-1) concatenated
+// (L175), and each W_ij is the contiguous range [win[i][j], win[i+1][j]) of
+// shard j (L155), so Mapper and SrcIndexCW are read off the window table.
 #include <cub/cub.cuh>
 
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
 #include <string>
+#include <vector>
 
 #include "common.cuh"
 #include "graph.hpp"
@@ -65,14 +66,6 @@ __global__ void k_starts(const uint64_t* __restrict__ k, uint64_t E, int shift, 
     for (int64_t t = prev + 1; t <= cur; ++t) start[t] = (uint32_t)p;
   }
 }
-__global__ void k_starts32(const uint32_t* __restrict__ k, uint64_t E, uint32_t S, uint32_t* start) {
-  GRID_STRIDE(p, E + 1) {
-    const int64_t cur = p < E ? (int64_t)k[p] : (int64_t)S;
-    const int64_t prev = p == 0 ? -1 : (int64_t)k[p - 1];
-    for (int64_t t = prev + 1; t <= cur; ++t) start[t] = (uint32_t)p;
-  }
-}
-
 // cnt[s] = start[s+1]-start[s]; padded[s] = round up to kPad; padded[S] = 0
 __global__ void k_counts(const uint32_t* start, uint32_t S, uint32_t* cnt, uint64_t* padded) {
   GRID_STRIDE(s, (uint64_t)S + 1) {
@@ -106,8 +99,7 @@ __global__ void k_fill_shard_pads(const uint32_t* off, const uint32_t* cnt, uint
 
 __global__ void k_scatter_gs(const uint64_t* __restrict__ keys, const uint32_t* __restrict__ ids, uint64_t E,
                              const uint32_t* start, const uint32_t* off, int bn, int bsrc, const uint32_t* __restrict__ val,
-                             uint32_t N, uint16_t* dest, uint16_t* srcidx, uint32_t* eid, uint32_t* ev,
-                             uint32_t* pos_of) {
+                             uint32_t N, uint16_t* dest, uint16_t* srcidx, uint32_t* eid, uint32_t* ev) {
   const uint64_t mn = (1ull << bn) - 1, ms = (1ull << bsrc) - 1;
   GRID_STRIDE(p, E) {
     const uint64_t k = keys[p];
@@ -118,12 +110,11 @@ __global__ void k_scatter_gs(const uint64_t* __restrict__ keys, const uint32_t* 
     const uint32_t id = ids[p];
     eid[pp] = id;
     if (ev) ev[pp] = val[id];
-    pos_of[p] = pp;
   }
 }
 
 // window table: win[t*S + j] = first padded position of shard j with SrcIndex >= t*N (t = 0..S)
-__global__ void k_windows(const uint64_t* __restrict__ keys, uint64_t E, const uint32_t* start, const uint32_t* pos_of,
+__global__ void k_windows(const uint64_t* __restrict__ keys, uint64_t E, const uint32_t* start, const uint32_t* off,
                           uint32_t N, uint32_t S, int bn, int bsrc, uint32_t* win) {
   const uint64_t ms = (1ull << bsrc) - 1;
   GRID_STRIDE(p, E) {
@@ -131,7 +122,8 @@ __global__ void k_windows(const uint64_t* __restrict__ keys, uint64_t E, const u
     const uint32_t j = (uint32_t)(k >> (bsrc + bn));
     const int64_t i = (int64_t)(((k >> bn) & ms) / N);
     const int64_t pi = (p == start[j]) ? -1 : (int64_t)(((keys[p - 1] >> bn) & ms) / N);
-    for (int64_t t = pi + 1; t <= i; ++t) win[(size_t)t * S + j] = pos_of[p];
+    const uint32_t pos = off[j] + (uint32_t)(p - start[j]);  // shard position of sorted entry p
+    for (int64_t t = pi + 1; t <= i; ++t) win[(size_t)t * S + j] = pos;
   }
 }
 __global__ void k_windows_tail(const uint64_t* __restrict__ keys, const uint32_t* start, const uint32_t* off,
@@ -161,21 +153,50 @@ __global__ void k_cw_counts(const uint32_t* outdeg, uint32_t V, uint32_t N, uint
   if (threadIdx.x == 0) cw_cnt[i] = acc;
 }
 
-__global__ void k_src_shard(const uint64_t* __restrict__ keys, uint64_t E, uint32_t N, int bn, int bsrc, uint32_t* ks) {
-  const uint64_t ms = (1ull << bsrc) - 1;
-  GRID_STRIDE(p, E) ks[p] = (uint32_t)(((keys[p] >> bn) & ms) / N);
+// padded[i] = cnt[i] rounded up to kPad; padded[S] = 0 (exclusive scan input)
+__global__ void k_pad_counts(const uint32_t* cnt, uint32_t S, uint64_t* padded) {
+  GRID_STRIDE(i, (uint64_t)S + 1) padded[i] = i < S ? (uint64_t)((cnt[i] + kPad - 1) / kPad) * kPad : 0ull;
 }
 
-__global__ void k_scatter_cw(const uint32_t* __restrict__ ks, const uint32_t* __restrict__ pp, uint64_t E,
-                             const uint32_t* cstart, const uint32_t* coff, const uint16_t* srcidx, uint32_t N,
-                             uint16_t* cw_src, uint32_t* mapper) {
-  GRID_STRIDE(q, E) {
-    const uint32_t i = ks[q];
-    const uint32_t pk = coff[i] + (uint32_t)(q - cstart[i]);
-    const uint32_t pos = pp[q];
-    (void)N;
-    cw_src[pk] = srcidx[pos];  // already SrcIndex - i*N
-    mapper[pk] = pos;
+// CW_i from the window table (L175, Fig. 4a): block i walks row i of the
+// table 256 windows at a time; a block scan of the window lengths gives each
+// window's offset inside CW_i, and the block's threads then copy the chunk's
+// entries (one per thread, the window found by binary search over the
+// chunk's offsets): Mapper[k] = shard position, SrcIndexCW[k] = SrcIndex there.
+__global__ void __launch_bounds__(256) k_cw_from_windows(const uint32_t* __restrict__ win, uint32_t S,
+                                                         const uint32_t* __restrict__ cw_off,
+                                                         const uint16_t* __restrict__ srcidx, uint16_t* cw_src,
+                                                         uint32_t* mapper) {
+  typedef cub::BlockScan<uint32_t, 256> BS;
+  __shared__ typename BS::TempStorage tmp;
+  __shared__ uint32_t s_off[257], s_beg[256];
+  const uint32_t i = blockIdx.x, tid = threadIdx.x;
+  const uint32_t* r0 = win + (size_t)i * S;
+  const uint32_t* r1 = r0 + S;
+  uint32_t base = cw_off[i];
+  for (uint32_t j0 = 0; j0 < S; j0 += 256) {
+    const uint32_t j = j0 + tid;
+    uint32_t b = 0, len = 0;
+    if (j < S) { b = r0[j]; len = r1[j] - b; }
+    uint32_t ex, total;
+    BS(tmp).ExclusiveSum(len, ex, total);
+    s_off[tid] = ex;
+    s_beg[tid] = b;
+    if (tid == 0) s_off[256] = total;
+    __syncthreads();
+    for (uint32_t f = tid; f < total; f += 256) {
+      uint32_t lo = 0, hi = 256;  // last window w with s_off[w] <= f
+      while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (s_off[mid] <= f) lo = mid;
+        else hi = mid;
+      }
+      const uint32_t pos = s_beg[lo] + (f - s_off[lo]);
+      mapper[base + f] = pos;
+      cw_src[base + f] = srcidx[pos];  // SrcIndex - i*N
+    }
+    base += total;
+    __syncthreads();
   }
 }
 __global__ void k_fill_cw_pads(const uint32_t* coff, const uint32_t* ccnt, uint32_t S, uint32_t trash, uint16_t* cw_src,
@@ -334,7 +355,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   PhaseTimer pt(st);
   t_alloc_stream = st;
 
-  DevBuf keys, keys2, ids, ids2, bad, start, padded, temp, pos_of;
+  DevBuf keys, keys2, ids, ids2, bad, start, padded, temp;
   CK(dalloc((uint64_t**)&keys.p, E));
   CK(dalloc((uint64_t**)&keys2.p, E));
   CK(dalloc((uint32_t**)&ids.p, E));
@@ -392,20 +413,19 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   CK(dalloc(&g.d_srcloc, P));
   CK(dalloc(&g.d_eid, P));
   if (d_val) { CK(dalloc(&g.d_ev, P)); g.has_ev = true; }
-  CK(dalloc((uint32_t**)&pos_of.p, E));
   pt.mark("offsets + alloc shard arrays");
   k_fill_shard_pads<<<grid_for((uint64_t)S * kPad), 256, 0, st>>>(g.d_shard_off, g.d_shard_cnt, S, N, g.d_dest,
                                                                    g.d_srcloc, g.d_eid, g.d_ev);
   if (E)
     k_scatter_gs<<<grid_for(E), 256, 0, st>>>(K, I, E, (uint32_t*)start.p, g.d_shard_off, bn, bsrc, d_val, N, g.d_dest,
-                                              g.d_srcloc, g.d_eid, g.d_ev, (uint32_t*)pos_of.p);
+                                              g.d_srcloc, g.d_eid, g.d_ev);
   CK(cudaGetLastError());
 
   // ---- window table W_ij (both representations keep it; GS stage 4 reads it)
   pt.mark("scatter shards");
   CK(dalloc(&g.d_win, ((uint64_t)S + 1) * S));
   if (E)
-    k_windows<<<grid_for(E), 256, 0, st>>>(K, E, (uint32_t*)start.p, (uint32_t*)pos_of.p, N, S, bn, bsrc, g.d_win);
+    k_windows<<<grid_for(E), 256, 0, st>>>(K, E, (uint32_t*)start.p, g.d_shard_off, N, S, bn, bsrc, g.d_win);
   k_windows_tail<<<grid_for(S), 256, 0, st>>>(K, (uint32_t*)start.p, g.d_shard_off, g.d_shard_cnt, N, S, bn, bsrc,
                                               g.d_win);
   CK(cudaGetLastError());
@@ -425,34 +445,11 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   // ---- Concatenated Windows + Mapper (§3.2)
   pt.mark("outdeg + cw counts");
   if (g.repr == CUSHA_REPR_CW) {
-    // reuse the key buffers: ks (u32) in keys.Alternate, positions in ids.Alternate
-    uint32_t* ks = reinterpret_cast<uint32_t*>(kb.Alternate());
-    uint32_t* ks2 = ks + E;
-    const int bks = bits_for(S - 1) ? bits_for(S - 1) : 1;
-    if (E) k_src_shard<<<grid_for(E), 256, 0, st>>>(K, E, N, bn, bsrc, ks);
-    CK(cudaGetLastError());
-    cub::DoubleBuffer<uint32_t> kk(ks, ks2);
-    cub::DoubleBuffer<uint32_t> pv((uint32_t*)pos_of.p, vb.Alternate());
-    if (E) {
-      size_t b3 = 0;
-      CK(cub::DeviceRadixSort::SortPairs(nullptr, b3, kk, pv, (int64_t)E, 0, bks, st));
-      if (b3 > tbytes) {
-        cudaFreeAsync(temp.p, st);
-        temp.p = nullptr;
-        CK(cudaMallocAsync(&temp.p, b3, st));
-        tbytes = b3;
-      }
-      CK(cub::DeviceRadixSort::SortPairs(temp.p, b3, kk, pv, (int64_t)E, 0, bks, st));
-    }
-    pt.mark("CW sort");
-    DevBuf cstart, cpad, cscan, t4;
-    CK(dalloc((uint32_t**)&cstart.p, (uint64_t)S + 1));
+    // CW_i offsets: |CW_i| = out-degree sum of shard i (cw_cnt), padded to kPad
+    DevBuf cpad, cscan, t4;
     CK(dalloc((uint64_t**)&cpad.p, (uint64_t)S + 1));
     CK(dalloc((uint64_t**)&cscan.p, (uint64_t)S + 1));
-    k_starts32<<<grid_for(E + 1), 256, 0, st>>>(kk.Current(), E, S, (uint32_t*)cstart.p);
-    DevBuf ccnt;
-    CK(dalloc((uint32_t**)&ccnt.p, S));
-    k_counts<<<grid_for((uint64_t)S + 1), 256, 0, st>>>((uint32_t*)cstart.p, S, (uint32_t*)ccnt.p, (uint64_t*)cpad.p);
+    k_pad_counts<<<grid_for((uint64_t)S + 1), 256, 0, st>>>(g.d_cw_cnt, S, (uint64_t*)cpad.p);
     CK(cudaGetLastError());
     size_t b4 = 0;
     CK(cub::DeviceScan::ExclusiveSum(nullptr, b4, (uint64_t*)cpad.p, (uint64_t*)cscan.p, (int64_t)S + 1, st));
@@ -467,11 +464,9 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
     k_narrow<<<grid_for((uint64_t)S + 1), 256, 0, st>>>((uint64_t*)cscan.p, (uint64_t)S + 1, g.d_cw_off);
     CK(dalloc(&g.d_cw_src, Q));
     CK(dalloc(&g.d_mapper, Q));
-    k_fill_cw_pads<<<grid_for((uint64_t)S * kPad), 256, 0, st>>>(g.d_cw_off, (uint32_t*)ccnt.p, S, (uint32_t)P,
+    k_fill_cw_pads<<<grid_for((uint64_t)S * kPad), 256, 0, st>>>(g.d_cw_off, g.d_cw_cnt, S, (uint32_t)P,
                                                                   g.d_cw_src, g.d_mapper);
-    if (E)
-      k_scatter_cw<<<grid_for(E), 256, 0, st>>>(kk.Current(), pv.Current(), E, (uint32_t*)cstart.p, g.d_cw_off,
-                                                g.d_srcloc, N, g.d_cw_src, g.d_mapper);
+    if (E) k_cw_from_windows<<<S, 256, 0, st>>>(g.d_win, S, g.d_cw_off, g.d_srcloc, g.d_cw_src, g.d_mapper);
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(st));
     // CW keeps the 3-tuple shards + SrcIndexCW + Mapper (L175): no per-entry SrcIndex in shard order
@@ -482,6 +477,76 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
     if (rc) return rc;
   }
   pt.mark("Mapper runs");
+  CK(cudaStreamSynchronize(st));
+  return CUSHA_OK;
+}
+
+// ------------------------------------------------ host-streamed topology (row f3)
+// "If graphs do not fit in the GPU RAM, a multi-streamed procedure should be
+// incorporated to overlap computation and data transfer" (L455).  Shards
+// [host_shard, S) keep their per-entry arrays (DestIndex, EdgeValue, SrcIndex,
+// edge ids) and, for CW, CW_i's SrcIndexCW and Mapper in pinned, mapped host
+// memory; the shard pass's TMA ring streams them over the host link each pass
+// exactly as it streams HBM tiles, so the transfer overlaps the consumers'
+// work tile by tile.  SrcValue, VertexValues and
+// the O(V + S^2) arrays stay in HBM.  host_shard is the first shard whose
+// prefix of per-entry arrays would exceed topo_budget bytes of HBM.
+namespace {
+template <class T>
+int move_tail(T*& dev, T*& host, uint64_t n, uint64_t split, cudaStream_t st, uint64_t& host_bytes,
+              std::string& err) {
+  if (!dev || split >= n) return CUSHA_OK;
+  const uint64_t m = n - split;
+  void* hp = nullptr;
+  CK(cudaHostAlloc(&hp, m * sizeof(T), cudaHostAllocMapped | cudaHostAllocPortable));
+  void* dp = nullptr;
+  CK(cudaHostGetDevicePointer(&dp, hp, 0));
+  if (dp != hp) {  // UVA: the mapped allocation has one address on host and device
+    cudaFreeHost(hp);
+    err = "mapped host memory without a unified address";
+    return CUSHA_EUNSUPPORTED;
+  }
+  host = static_cast<T*>(hp);
+  CK(cudaMemcpyAsync(host, dev + split, m * sizeof(T), cudaMemcpyDeviceToHost, st));
+  T* nd = nullptr;
+  if (split) {
+    CK(dalloc(&nd, split));
+    CK(cudaMemcpyAsync(nd, dev, split * sizeof(T), cudaMemcpyDeviceToDevice, st));
+  }
+  CK(cudaFreeAsync(dev, st));
+  dev = nd;
+  host_bytes += m * sizeof(T);
+  return CUSHA_OK;
+}
+}  // namespace
+
+int offload_topology(Graph& g, std::string& err) {
+  cudaStream_t st = g.stream;
+  t_alloc_stream = st;
+  const uint32_t S = g.S;
+  g.splitP = g.P;
+  g.splitQ = g.Q;
+  g.host_shard = S;
+  if (!g.topo_budget || !S) return CUSHA_OK;
+  std::vector<uint32_t> so(S + 1), co(S + 1, 0);
+  CK(cudaMemcpyAsync(so.data(), g.d_shard_off, 4ull * (S + 1), cudaMemcpyDeviceToHost, st));
+  if (g.d_cw_off) CK(cudaMemcpyAsync(co.data(), g.d_cw_off, 4ull * (S + 1), cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  const uint64_t bP = 2 + 4 + (g.has_ev ? 4 : 0) + (g.d_srcloc ? 2 : 0);  // DestIndex, edge id, EdgeValue, SrcIndex
+  const uint64_t bQ = g.d_cw_src ? 6 : 0;                                  // SrcIndexCW, Mapper
+  uint32_t h = 0;
+  while (h < S && (uint64_t)so[h + 1] * bP + (uint64_t)co[h + 1] * bQ <= g.topo_budget) ++h;
+  g.host_shard = h;
+  g.splitP = so[h];
+  g.splitQ = g.d_cw_src ? co[h] : g.Q;
+  int rc;
+  if ((rc = move_tail(g.d_dest, g.h_dest, g.P, g.splitP, st, g.host_bytes, err)) ||
+      (rc = move_tail(g.d_ev, g.h_ev, g.P, g.splitP, st, g.host_bytes, err)) ||
+      (rc = move_tail(g.d_eid, g.h_eid, g.P, g.splitP, st, g.host_bytes, err)) ||
+      (rc = move_tail(g.d_srcloc, g.h_srcloc, g.P, g.splitP, st, g.host_bytes, err)) ||
+      (rc = move_tail(g.d_cw_src, g.h_cw_src, g.Q, g.splitQ, st, g.host_bytes, err)) ||
+      (rc = move_tail(g.d_mapper, g.h_mapper, g.Q, g.splitQ, st, g.host_bytes, err)))
+    return rc;
   CK(cudaStreamSynchronize(st));
   return CUSHA_OK;
 }

@@ -73,7 +73,22 @@ struct KParams {
   // opt-in exact work skipping
   int skip;                    // 1: a shard none of whose windows was written since its last pass is skipped
   uint32_t* dirty;             // S: some window of shard j written since j's last pass (set by writers)
+  // host-streamed topology (row f3): entries at shard
+  // positions >= splitP / CW positions >= splitQ live in pinned host memory
+  // (x_h[i - split]); below the split, in HBM (x[i]).  splitP = P, splitQ = Q: all in HBM.
+  uint32_t splitP, splitQ;
+  const uint16_t* dest_h;
+  const uint32_t* ev_h;
+  const uint16_t* srcloc_h;
+  const uint16_t* cw_src_h;
+  const uint32_t* mapper_h;
 };
+
+// element i of a topology array split between HBM (i < split) and pinned host memory
+template <class T>
+__host__ __device__ __forceinline__ const T* topo_at(const T* dev, const T* host, uint32_t split, uint64_t i) {
+  return i < split ? dev + i : host + (i - split);
+}
 
 struct PassKernel {
   const void* func;       // __global__ shard_pass<Alg, Repr>
@@ -106,6 +121,18 @@ struct Graph {
   uint8_t* d_active = nullptr;      // S: stage-4 prefetch predictor
   uint32_t* d_dirty = nullptr;      // S: clean-shard skipping flags
   bool skip_clean = false;
+  // host-streamed topology (row f3): shards >= host_shard keep their entry
+  // arrays (and CW_i arrays) in pinned, mapped host memory
+  uint64_t topo_budget = 0;         // HBM bytes allowed for per-entry topology; 0 = unlimited
+  uint32_t host_shard = 0;          // first host-resident shard (S: none)
+  uint64_t splitP = 0, splitQ = 0;  // shard / CW positions where host residency starts
+  uint16_t* h_dest = nullptr;       // P - splitP   (pinned host, mapped)
+  uint32_t* h_ev = nullptr;
+  uint16_t* h_srcloc = nullptr;
+  uint32_t* h_eid = nullptr;
+  uint16_t* h_cw_src = nullptr;     // Q - splitQ
+  uint32_t* h_mapper = nullptr;
+  uint64_t host_bytes = 0;
   uint16_t* d_cw_src = nullptr;     // Q (CW)
   uint32_t* d_mapper = nullptr;     // Q (CW)
   uint32_t R = 0;                   // Mapper runs (non-empty windows)
@@ -155,6 +182,7 @@ bool alg_needs_init(int alg);
 int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const uint32_t* d_val, std::string& err);
 int build_partition(Graph& g, std::string& err);  // bounds, owner, cwp, gathered (G > 1)
 int build_runs(Graph& g, std::string& err);       // Mapper runs (CW)
+int offload_topology(Graph& g, std::string& err); // row f3: move shards >= host_shard to pinned host memory
 void partition_bounds(uint32_t S, const uint64_t* work, uint32_t G, uint32_t* bounds);
 
 // api.cu

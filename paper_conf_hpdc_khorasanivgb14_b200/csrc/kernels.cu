@@ -232,7 +232,7 @@ __device__ __forceinline__ void gs_walk(const KParams& p, uint32_t s, uint32_t l
           if (ex <= f) w += step;
         }
         e[u] = __shfl_sync(kFull, a, w) + (f - __shfl_sync(kFull, exc, w));
-        l[u] = f < total ? (uint32_t)__ldg(p.srcloc + e[u]) : 0xFFFFFFFFu;
+        l[u] = f < total ? (uint32_t)__ldg(topo_at(p.srcloc, p.srcloc_h, p.splitP, e[u])) : 0xFFFFFFFFu;
       }
 #pragma unroll
       for (int u = 0; u < kGSU; ++u)
@@ -327,8 +327,9 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     for (uint32_t t0 = b; t0 < e; t0 += kTile) {
       const uint32_t n = min(kTile, e - t0);
       const uint32_t flags = (t0 + n >= e ? kFlagLast : 0u) | (t0 == b && spec ? kFlagSpec4 : 0u);
-      push(s, kDescStage2, n, flags, p.srcvalue + t0, n * 4, p.dest + t0, 4 * kTile, n * 2,
-           A::kEdge ? (const void*)(p.ev + t0) : nullptr, 6 * kTile, A::kEdge ? n * 4 : 0u);
+      push(s, kDescStage2, n, flags, p.srcvalue + t0, n * 4, topo_at(p.dest, p.dest_h, p.splitP, t0), 4 * kTile,
+           n * 2, A::kEdge ? (const void*)topo_at(p.ev, p.ev_h, p.splitP, t0) : nullptr, 6 * kTile,
+           A::kEdge ? n * 4 : 0u);
     }
     bool send4 = spec;
     if (REPR == CUSHA_REPR_CW && !spec) {
@@ -353,13 +354,14 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
             if (nr <= kRunCap) {
               // slot: SrcIndexCW | RunT-RunK per run | run-start bitmap words [k0/128*4, ceil((k0+n)/128)*4)
               const uint32_t wa = k0 / 128 * 4, wz = (k0 + n + 127) / 128 * 4;
-              push(s, kDescStage4R, n, fl | ((ra - ra4) << 8), p.cw_src + k0, n * 2, p.run_d + ra4, 2 * kTile,
+              push(s, kDescStage4R, n, fl | ((ra - ra4) << 8), topo_at(p.cw_src, p.cw_src_h, p.splitQ, k0), n * 2,
+                   p.run_d + ra4, 2 * kTile,
                    nr * 4, p.run_bits + wa, 2 * kTile + 4 * kRunCap, (wz - wa) * 4, lo, hi, k0, nr);
               continue;
             }
           }
-          push(s, kDescStage4, n, fl, p.cw_src + k0, n * 2, p.mapper + k0, 2 * kTile, n * 4, nullptr, 0, 0, lo, hi,
-               k0, 0);
+          push(s, kDescStage4, n, fl, topo_at(p.cw_src, p.cw_src_h, p.splitQ, k0), n * 2,
+               topo_at(p.mapper, p.mapper_h, p.splitQ, k0), 2 * kTile, n * 4, nullptr, 0, 0, lo, hi, k0, 0);
         }
     }
   }
@@ -665,7 +667,8 @@ __global__ void __launch_bounds__(256) refresh_remote(const KParams p) {
     for (uint32_t q = 0; q < p.G; ++q) {
       if (q == oi || (p.part >= 0 && (int)q != p.part)) continue;
       for (uint32_t k = row[q] + threadIdx.x; k < row[q + 1]; k += blockDim.x)
-        st_u32(p.srcvalue + __ldg(p.mapper + k), __ldg(vals + __ldg(p.cw_src + k)));
+        st_u32(p.srcvalue + __ldg(topo_at(p.mapper, p.mapper_h, p.splitQ, k)),
+               __ldg(vals + __ldg(topo_at(p.cw_src, p.cw_src_h, p.splitQ, k))));
       if (p.skip)  // the refreshed shards of partition q have new inputs
         for (uint32_t j = p.bounds[q] + threadIdx.x; j < p.bounds[q + 1]; j += blockDim.x)
           if (__ldg(p.win + (size_t)(i + 1) * p.S + j) > __ldg(p.win + (size_t)i * p.S + j)) p.dirty[j] = 1u;
@@ -721,9 +724,9 @@ __global__ void init_srcvalue_cw(const KParams p) {
   const V_t* vv = reinterpret_cast<const V_t*>(p.vv);
   const uint32_t i = blockIdx.x, trash = p.shard_off[p.S];
   for (uint32_t k = p.cw_off[i] + threadIdx.x; k < p.cw_off[i + 1]; k += blockDim.x) {
-    const uint32_t m = p.mapper[k];
+    const uint32_t m = *topo_at(p.mapper, p.mapper_h, p.splitQ, k);
     if (m == trash) continue;
-    const uint32_t u = i * p.N + p.cw_src[k];
+    const uint32_t u = i * p.N + *topo_at(p.cw_src, p.cw_src_h, p.splitQ, k);
     p.srcvalue[m] = A::wb_value(vv[u], A::kOutDeg ? p.outdeg[u] : 0u);
   }
 }
@@ -786,6 +789,8 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.run_k = g.d_run_k; p.run_t = g.d_run_t; p.run_unit = g.d_run_unit; p.run_bits = g.d_run_bits; p.run_d = g.d_run_d;
   p.R = g.R;
   p.skip = g.skip_clean ? 1 : 0; p.dirty = g.d_dirty;
+  p.splitP = (uint32_t)g.splitP; p.splitQ = (uint32_t)g.splitQ;
+  p.dest_h = g.h_dest; p.ev_h = g.h_ev; p.srcloc_h = g.h_srcloc; p.cw_src_h = g.h_cw_src; p.mapper_h = g.h_mapper;
   p.use_cond = 0; p.cond_handle = 0;
   return p;
 }

@@ -47,6 +47,7 @@ class BuildOpts(ctypes.Structure):
         ("rank", ctypes.c_int),
         ("nccl_unique_id", ctypes.c_void_p),
         ("skip_clean_shards", ctypes.c_int),
+        ("device_topology_budget", ctypes.c_uint64),
     ]
 
 
@@ -74,6 +75,8 @@ class Stats(ctypes.Structure):
         ("device_loop", ctypes.c_uint32),
         ("world_size", ctypes.c_int),
         ("rank", ctypes.c_int),
+        ("host_bytes", ctypes.c_uint64),
+        ("host_shard", ctypes.c_uint32),
     ]
 
 
@@ -210,11 +213,13 @@ def get_partition(g: "Graph") -> np.ndarray:
 def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertices_per_shard: int = 0,
                 smem_bytes_per_vertex: int = 0, device: int = 0, stream: Optional[int] = None,
                 host_loop: bool = False, world_size: int = 1, rank: int = 0,
-                nccl_id: Optional[bytes] = None, skip_clean_shards: bool = False) -> Graph:
+                nccl_id: Optional[bytes] = None, skip_clean_shards: bool = False,
+                device_topology_budget: int = 0) -> Graph:
     """cusha_build_graph.  src/dst/edge_values: numpy (host, copied in) or CUDA tensors (device).
     world_size > 1: destination-range partition; nccl_id = None simulates all
     partitions on this device, else one process per GPU over NCCL.
-    skip_clean_shards: opt-in exact skipping of shards whose inputs did not change."""
+    skip_clean_shards: opt-in exact skipping of shards whose inputs did not change.
+    device_topology_budget: HBM bytes for per-entry topology; the rest is streamed from pinned host memory."""
     on_dev = _is_device(src)
     if not on_dev:
         src = np.ascontiguousarray(src, dtype=np.uint32)
@@ -236,6 +241,7 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
     o.world_size = world_size
     o.rank = rank
     o.skip_clean_shards = int(skip_clean_shards)
+    o.device_topology_budget = int(device_topology_budget)
     idbuf = None
     if nccl_id is not None:
         if len(nccl_id) != 128:
