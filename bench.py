@@ -257,7 +257,7 @@ def bench_cusha(args):
     torch.cuda.synchronize()
     g = cusha.build_graph(wl.V, src_d, dst_d, edge_values=ev, repr=repr_, vertices_per_shard=args.N, device=dev,
                           stream=stream.cuda_stream, host_loop=args.host_loop,
-                          skip_clean_shards=args.skip_clean, **part)
+                          skip_clean_shards=args.skip_clean, pass_barrier=args.pass_barrier, **part)
     st0 = cusha.get_stats(g)
     log(f"[bench] rank {rank}/{world} built {repr_} |N|={st0['vertices_per_shard']} |S|={st0['num_shards']} "
         f"in {st0['build_ms']:.1f} ms")
@@ -275,7 +275,7 @@ def bench_cusha(args):
             rc = cusha.run(alg, g, source=source)
             st = cusha.get_stats(g)
             steps.append((rc, st["iterations"], st["loop_ms"], st["run_ms"], st["algorithmic_bytes"],
-                          st["edges_processed"]))
+                          st["edges_processed"], st["device_loop"]))
         e1.record(stream)
         torch.cuda.synchronize()
     barrier()
@@ -286,8 +286,9 @@ def bench_cusha(args):
     loop_ms = sum(s[2] for s in steps)
     alg_bytes = sum(s[4] for s in steps)
     value = edges / (total_ms / 1e3) / 1e9
-    # reset_ctl + init_vertex_values + init_srcvalue + one pass per iteration (+ one refresh when partitioned)
-    launches = sum(3 + it * (2 if world > 1 else 1) for it in iters)
+    # reset_ctl + init_vertex_values + init_srcvalue + the passes: one launch for all of them
+    # (overlapped passes, device_loop 2) or one per iteration (+ one refresh when partitioned)
+    launches = sum(3 + (1 if s[6] == 2 else s[1] * (2 if world > 1 else 1)) for s in steps)
     launches = int(sum_over_ranks(launches))
     peak, peak_kind = measured_peak_gbs()
     achieved = alg_bytes / (loop_ms / 1e3) / 1e9
@@ -311,7 +312,7 @@ def bench_cusha(args):
             gh = cusha.build_graph(wl.V, pin_s.numpy().view(np.uint32), pin_d.numpy().view(np.uint32),
                                    edge_values=None if pin_w is None else pin_w.numpy().view(np.uint32),
                                    repr=repr_, vertices_per_shard=args.N, device=dev, stream=stream.cuda_stream,
-                                   skip_clean_shards=args.skip_clean, **part)
+                                   skip_clean_shards=args.skip_clean, pass_barrier=args.pass_barrier, **part)
             cusha.run(alg, gh, source=source)
             n = cusha.get_stats(gh)["edges_processed"]
             rc = cusha.lib().cusha_get_values(gh.handle, cusha._ptr(out), wl.V * vb)
@@ -352,6 +353,8 @@ def bench_cusha(args):
                    if per_iter_gb * 1e9 > L2_BYTES else f"L2-resident workload ({per_iter_gb*1e3:.1f} MB per pass); no flush",
                    "build_ms": round(st0["build_ms"], 3),
                    "skip_clean_shards": bool(args.skip_clean),
+                   "passes": "one launch per pass, device-wide barrier between passes" if steps[-1][6] != 2
+                   else "overlapped passes in one launch (DESIGN.md \"Overlapped passes\")",
                    "parallelism": f"destination-range partition x{world} (NCCL)" if world > 1 else "1 GPU"},
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                      "frac": round(achieved / peak, 4), "traffic": traffic_for(args.workload) if world == 1 else None,
@@ -390,6 +393,9 @@ def main():
     ap.add_argument("--lib", default=None, help="alternative libcusha.so (tuning variants)")
     ap.add_argument("--skip-clean", action="store_true",
                     help="opt-in exact clean-shard skipping (not the paper's full passes; off by default)")
+    ap.add_argument("--pass-barrier", action="store_true",
+                    help="one launch per pass with a device-wide barrier between passes (Fig. 5) instead of "
+                         "the default overlapped passes")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0)

@@ -42,7 +42,7 @@ extern "C" {
 #define CUSHA_API
 #endif
 
-#define CUSHA_ABI_VERSION 2
+#define CUSHA_ABI_VERSION 3
 
 /* Return codes. */
 enum {
@@ -122,6 +122,17 @@ typedef struct {
    * SrcValue, VertexValues and the O(|V| + |S|^2) arrays stay in HBM.  Results
    * are identical to the in-HBM layout.  The build itself runs in HBM first.  */
   uint64_t device_topology_budget;
+  /* Iteration boundary of the device loop (row a5; DESIGN.md "Overlapped
+   * passes").  0 (default) = one launch runs every pass: shards are drawn as
+   * tickets across passes, so a CTA done with its part of pass k starts pass
+   * k+1 (the asynchronous model of L45 carried across the iteration
+   * boundary; a shard's passes stay in order).  Convergence is concluded only
+   * from a pass that started after every earlier pass completed and committed
+   * nothing (L189), so results are those of the barrier mode.  1 = one launch
+   * per pass under a CUDA-graph while node, with a device-wide barrier between
+   * passes as in Fig. 5.  host_loop = 1 or world_size > 1 imply one launch
+   * per pass.                                                              */
+  int pass_barrier;
 } cusha_build_opts;
 
 typedef struct cusha_graph cusha_graph;   /* opaque; owns all device memory it allocates */
@@ -148,7 +159,8 @@ typedef struct {
   uint64_t edges_processed;        /* last run: edges streamed by stage 2 over all passes of this
                                       process's shards (iterations * |E| unless shards were
                                       skipped or partitioned)                                 */
-  uint32_t device_loop;            /* 1 = the run looped on the device (CUDA-graph while node) */
+  uint32_t device_loop;            /* 0 = passes launched by the host; 1 = CUDA-graph while node,
+                                      one launch per pass; 2 = overlapped passes, one launch    */
   int world_size, rank;
   uint64_t host_bytes;             /* per-entry topology bytes held in pinned host memory (f3)  */
   uint32_t host_shard;             /* first shard whose topology is host-resident (|S|: none)   */

@@ -43,7 +43,7 @@ static void free_graph_memory(Graph& g) {
   void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcloc, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
                   g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_srcvalue, g.d_vv, g.d_ctl, g.d_trace,
                   g.d_active, g.d_bounds, g.d_owner, g.d_cwp, g.d_gathered, g.d_run_k, g.d_run_t,
-                  g.d_run_unit, g.d_run_bits, g.d_run_d, g.d_dirty};
+                  g.d_run_unit, g.d_run_bits, g.d_run_d, g.d_dirty, g.d_shard_seq};
   nccl_destroy(g);
   // device memory is stream-ordered (cudaMallocAsync on g.stream): released to
   // the retained pool without unmapping or a device-wide synchronisation
@@ -155,6 +155,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   g.V = V; g.E = E; g.N = N; g.S = (V + N - 1) / N; g.repr = (int)o.repr; g.device = o.device;
   g.host_loop = o.host_loop != 0;
   g.skip_clean = o.skip_clean_shards != 0;
+  g.pass_barrier = o.pass_barrier != 0;
   g.topo_budget = o.device_topology_budget;
   g.world_size = o.world_size;
   g.rank = o.world_size > 1 && o.nccl_unique_id ? o.rank : 0;
@@ -366,7 +367,10 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   const size_t smem = pk.smem_bytes(g.N);
   int rc = CUSHA_OK;
   const bool host_loop = g.host_loop || g.G > 1;  // the partitioned mode exchanges between passes
-  if (host_loop) {
+  // overlapped passes (default): one launch runs every pass; it needs a trace
+  // record per pass (<= 2^20), else the CUDA-graph loop runs one launch per pass
+  const bool multi = !host_loop && !g.pass_barrier && max_iters <= g.trace_cap;
+  if (host_loop || multi) {
     if (smem > 227 * 1024)
       return fail(CUSHA_EINVAL, "vertices_per_shard too large for this algorithm's shared-memory state");
     CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -380,7 +384,14 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   CKA(launch_reset_ctl(g.d_ctl, max_iters, g.stream));
   CKA(launch_init(g, a, source, g.stream));
   CKA(cudaEventRecord(g.evm, g.stream));
-  if (max_iters > 0 && !host_loop) CKA(cudaGraphLaunch(h->exec[a], g.stream));
+  if (max_iters > 0 && multi) {
+    KParams kp = make_params(g, source);
+    kp.multi = 1;
+    void* args[] = {&kp};
+    CKA(cudaLaunchKernel(pk.func, dim3(pass_grid(g, pk, smem)), dim3(pk.threads), args, smem, g.stream));
+  } else if (max_iters > 0 && !host_loop) {
+    CKA(cudaGraphLaunch(h->exec[a], g.stream));
+  }
   if (max_iters > 0 && host_loop) {
     // passes launched by the host in chunks; a pass that finds the run
     // converged (or at max_iters) exits at once, so over-launching is exact.
@@ -413,7 +424,11 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   float ms = 0, lms = 0;
   cudaEventElapsedTime(&ms, g.ev0, g.ev1);
   cudaEventElapsedTime(&lms, g.evm, g.ev1);
-  const Ctl c = *g.h_ctl;
+  Ctl c = *g.h_ctl;
+  if (multi && max_iters > 0) {  // the confirming pass that committed nothing, else max_iters passes ran
+    c.converged = c.conv_iter != 0xFFFFFFFFu;
+    c.iter = c.converged ? c.conv_iter : max_iters;
+  }
   // statistics and algorithmic bytes
   const uint64_t vb = value_bytes(a);
   const uint64_t evb = alg_needs_edge_values(a) ? 4 : 0;
@@ -443,7 +458,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   g.st.edges_processed = n == c.iter ? edges : (uint64_t)c.iter * g.E;
   g.st.stage2_bytes_per_iter = g.E * (4 + 2 + evb);
   g.st.wb_bytes_all_active = g.repr == CUSHA_REPR_CW ? g.E * 10 : g.E * 8;
-  g.st.device_loop = g.host_loop ? 0 : 1;
+  g.st.device_loop = host_loop ? 0 : (multi ? 2 : 1);
   g.last_alg = a;
   g.have_values = true;
   return c.converged ? CUSHA_OK : CUSHA_NOT_CONVERGED;

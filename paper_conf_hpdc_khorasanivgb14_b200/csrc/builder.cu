@@ -441,6 +441,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
 
   CK(dalloc(&g.d_active, S));  // stage-4 prefetch predictor of the shard pass
   if (g.skip_clean) CK(dalloc(&g.d_dirty, S));
+  CK(dalloc(&g.d_shard_seq, S));  // overlapped passes: per-shard pass order
 
   // ---- Concatenated Windows + Mapper (§3.2)
   pt.mark("outdeg + cw counts");

@@ -22,12 +22,18 @@ struct Ctl {
   uint32_t next_shard;  // dynamic shard queue of the persistent pass
   uint32_t gchanged;    // partitioned mode: some shard of any partition was active (refresh kernel)
   uint32_t rctas_done;  // partitioned mode: refresh-kernel arrival counter
+  // overlapped passes (one launch per run)
+  unsigned long long ticket;  // shard tickets drawn: ticket t = shard t % |S| of pass t / |S|
+  uint32_t stop;              // two consecutive passes committed nothing: draw no more tickets
+  uint32_t conv_iter;         // 1 + the later of those two passes (~0u: none yet)
 };
 
 // Per-iteration trace (row f4; also the source of algorithmic byte counts).
 struct TraceRec {
   uint32_t updated;          // vertices committed in stage 3
   uint32_t active_shards;    // shards that ran stage 4
+  uint32_t done;             // overlapped passes: shard tickets of this pass completed
+  uint32_t pad_;
   unsigned long long wb_entries;  // CW / window entries visited by stage 4
   unsigned long long wb_stores;   // SrcValue words actually stored by stage 4
   unsigned long long edges;       // edges streamed by stage 2 (|E| unless clean shards are skipped)
@@ -56,6 +62,8 @@ struct KParams {
   uint32_t trace_cap;
   int use_cond;
   unsigned long long cond_handle;
+  int multi;                   // 1: one launch runs every pass (overlapped passes)
+  uint32_t* shard_seq;         // S: passes of shard s completed (overlapped passes)
   // destination-range partition (row e); G = 1: single partition
   uint32_t G;                  // partitions
   int part;                    // partition this launch processes (-1: all, the single-process simulation)
@@ -120,6 +128,8 @@ struct Graph {
   uint32_t* d_cw_cnt = nullptr;     // S
   uint8_t* d_active = nullptr;      // S: stage-4 prefetch predictor
   uint32_t* d_dirty = nullptr;      // S: clean-shard skipping flags
+  uint32_t* d_shard_seq = nullptr;  // S: overlapped passes, per-shard pass order
+  bool pass_barrier = false;        // 1: one launch per pass (CUDA-graph while loop)
   bool skip_clean = false;
   // host-streamed topology (row f3): shards >= host_shard keep their entry
   // arrays (and CW_i arrays) in pinned, mapped host memory

@@ -116,8 +116,62 @@ enum : uint32_t { kFlagLast = 1, kFlagSpec4 = 2 };
 // copied into the slot; [lo, hi) = the entries the consumers use; base = CW
 // position of entry 0 of the slot; nruns = runs in the slot (kDescStage4R).
 struct __align__(16) TileDesc {
-  uint32_t shard, kind, n, flags, lo, hi, base, nruns;
+  uint32_t shard, kind, n, flags, lo, hi, base, nruns, pass;
 };
+
+// ------------------------------------------------ overlapped passes (row a5)
+// One launch runs every pass: shard tickets
+// t = 0, 1, 2, ... are drawn from one counter (shard t % |S| of pass t / |S|),
+// so a CTA that finishes its part of pass k goes on with pass k + 1 instead of
+// idling at an iteration barrier: the paper's asynchronous model (L45) carried
+// across the iteration boundary.  Two waits bound the overlap:
+//  - pass k of shard s starts after pass k - 1 of s completed (one CTA owns a
+//    shard's VertexValues at a time, as in Fig. 5);
+//  - pass k starts after pass k - 2 completed (at most two passes in flight).
+// Convergence (L189, "a pass that commits nothing") is concluded when two
+// consecutive passes k - 1 and k both committed nothing.  Why that is exact:
+// let T0 be the moment pass k - 2 completed.  Every ticket of pass k read its
+// inputs after T0, and no write happens after T0 until some commit; take the
+// first commit after T0, by a ticket of pass q on shard s.  Passes k - 1 and
+// k commit nothing, so q > k, and that ticket read the state at T0 - as did
+// shard s's pass-k ticket, which ran between T0 and it and committed nothing
+// from the same inputs and the same VertexValues (integer and fixed-point
+// sums are order-independent, R11).  The same inputs give the same result,
+// so no such commit exists: the state at T0 is the fixed point a
+// barrier-separated pass would confirm.
+__device__ __forceinline__ uint32_t ld_vol(const uint32_t* a) { return *reinterpret_cast<const volatile uint32_t*>(a); }
+__device__ __forceinline__ void st_vol(uint32_t* a, uint32_t v) { *reinterpret_cast<volatile uint32_t*>(a) = v; }
+__device__ __forceinline__ void fence_sc_gpu() { asm volatile("fence.sc.gpu;" ::: "memory"); }
+
+// the producer's waits before ticket (s, pass) may read anything
+__device__ __forceinline__ void ticket_wait(const KParams& p, uint32_t s, uint32_t pass, uint32_t Sloc) {
+  while (ld_vol(&p.shard_seq[s]) < pass) __nanosleep(64);
+  if (pass >= 2)
+    while (ld_vol(&p.trace[pass - 2].done) < Sloc) __nanosleep(64);
+  __threadfence();                                      // acquire the completed passes' stores ...
+  asm volatile("fence.proxy.async.global;" ::: "memory");  // ... for the TMA (async-proxy) reads too
+}
+
+// ticket (s, pass) finished (its stores ordered before by the caller's
+// barrier; fences are cumulative).  The thread completing the last ticket of
+// a clean pass looks at both neighbouring passes.
+__device__ __forceinline__ void ticket_done(const KParams& p, uint32_t s, uint32_t pass, uint32_t Sloc) {
+  __threadfence();
+  st_vol(&p.shard_seq[s], pass + 1);
+  if (atomicAdd(&p.trace[pass].done, 1u) != Sloc - 1) return;
+  fence_sc_gpu();  // pairs with the other neighbour's completer: at least one of two sees both complete
+  if (ld_vol(&p.trace[pass].active_shards) != 0) return;
+  auto clean = [&](uint32_t r) {
+    return ld_vol(&p.trace[r].done) == Sloc && ld_vol(&p.trace[r].active_shards) == 0;
+  };
+  uint32_t conv = 0xFFFFFFFFu;
+  if (pass >= 1 && clean(pass - 1)) conv = pass + 1;
+  else if (pass + 1 < p.ctl->max_iters && clean(pass + 1)) conv = pass + 2;
+  if (conv != 0xFFFFFFFFu) {
+    atomicMin(&p.ctl->conv_iter, conv);
+    st_vol(&p.ctl->stop, 1u);
+  }
+}
 
 // ------------------------------------------------------------ stage 2 body
 template <class A>
@@ -251,14 +305,14 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
   constexpr uint32_t SLOT = slot_bytes<A>();
   constexpr uint32_t kTile = tile_of<A>();
   constexpr uint32_t kRunCap = run_cap<A>();
-  uint32_t slot = 0, ph = 0, dph = 0;
+  uint32_t slot = 0, ph = 0, dph = 0, cur_pass = 0;
   const uint64_t pol = l2_evict_first_policy();
   auto push = [&](uint32_t shard, uint32_t kind, uint32_t n, uint32_t flags, const void* g0, uint32_t b0,
                   const void* g1, uint32_t o1, uint32_t b1, const void* g2, uint32_t o2, uint32_t b2,
                   uint32_t lo = 0, uint32_t hi = 0xFFFFFFFFu, uint32_t base = 0, uint32_t nruns = 0,
                   const void* g3 = nullptr, uint32_t o3 = 0, uint32_t b3 = 0) {
     mbar_wait(&empty_bar[slot], ph ^ 1);
-    desc[slot] = TileDesc{shard, kind, n, flags, lo, hi == 0xFFFFFFFFu ? n : hi, base, nruns};
+    desc[slot] = TileDesc{shard, kind, n, flags, lo, hi == 0xFFFFFFFFu ? n : hi, base, nruns, cur_pass};
     uint8_t* buf = ring + slot * SLOT;
     const uint32_t bytes = b0 + b1 + b2 + b3;
     if (bytes) {
@@ -286,12 +340,30 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
   };
   // shards of this launch: one partition's range (multi-GPU) or all of them
   const uint32_t q_lo = p.part >= 0 ? p.bounds[p.part] : 0u, q_hi = p.part >= 0 ? p.bounds[p.part + 1] : p.S;
+  const uint32_t Sloc = q_hi - q_lo;
   for (uint32_t round = 0;; ++round) {
-    // persistent grid: shards from the global queue; otherwise CTA b runs shard q_lo + b only
-    const uint32_t s = q_lo + (kPersistent ? atomicAdd(&p.ctl->next_shard, 1u) : (round == 0 ? blockIdx.x : q_hi));
-    if (s >= q_hi) {
-      push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
-      return;
+    uint32_t s;
+    if (p.multi) {
+      // overlapped passes: the next ticket, whatever pass it belongs to
+      bool over = ld_vol(&p.ctl->stop) != 0;
+      if (!over) {
+        const unsigned long long t = atomicAdd(&p.ctl->ticket, 1ull);
+        cur_pass = (uint32_t)(t / Sloc);
+        s = q_lo + (uint32_t)(t - (unsigned long long)cur_pass * Sloc);
+        over = cur_pass >= p.ctl->max_iters || ld_vol(&p.ctl->stop) != 0;
+      }
+      if (over) {
+        push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
+        return;
+      }
+      ticket_wait(p, s, cur_pass, Sloc);
+    } else {
+      // persistent grid: shards from the global queue; otherwise CTA b runs shard q_lo + b only
+      s = q_lo + (kPersistent ? atomicAdd(&p.ctl->next_shard, 1u) : (round == 0 ? blockIdx.x : q_hi));
+      if (s >= q_hi) {
+        push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
+        return;
+      }
     }
     if (p.skip) {
       // clean-shard skipping (opt-in): no
@@ -301,6 +373,7 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
       // re-marks s for a later pass.
       if (atomicExch(&p.dirty[s], 0u) == 0u) {
         p.active[s] = 0;
+        if (p.multi) ticket_done(p, s, cur_pass, Sloc);
         continue;
       }
       __threadfence();                                      // acquire the writers' SrcValue stores ...
@@ -383,9 +456,10 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
   const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
   const uint32_t N = p.N, st = N + 1;
   uint32_t* const aux = sm + A::kWords * st;  // write-back values (float algs) or changed bits (integer algs)
-  const uint32_t it = *reinterpret_cast<volatile uint32_t*>(&p.ctl->iter);
+  const uint32_t it0 = *reinterpret_cast<volatile uint32_t*>(&p.ctl->iter);
   // a pass launched after the run converged / hit max_iters is a no-op (host-loop mode)
-  if (*reinterpret_cast<volatile uint32_t*>(&p.ctl->converged) || it >= p.ctl->max_iters) return;
+  if (*reinterpret_cast<volatile uint32_t*>(&p.ctl->converged) || it0 >= p.ctl->max_iters) return;
+  const uint32_t Sloc = p.part >= 0 ? p.bounds[p.part + 1] - p.bounds[p.part] : p.S;
   if (tid == 0) {
     for (uint32_t i = 0; i < kStages; ++i) {
       mbar_init(&full_bar[i], 1);                // the producer's arrive(.expect_tx)
@@ -406,6 +480,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
       TileDesc d = desc[slot];
       if (d.kind == kDescDone) break;
       const uint32_t s = d.shard;
+      const uint32_t it = p.multi ? d.pass : it0;  // the pass this shard belongs to
       const bool spec4 = d.flags & kFlagSpec4;
       const uint32_t off = s * N;
       const uint32_t nv = min(N, p.V - off);
@@ -603,6 +678,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
         for (uint32_t j = ct; j < p.S; j += kConsumers)
           if (__ldg(w1 + j) > __ldg(w0 + j) && (p.G == 1 || p.owner[j] == p.owner[s])) p.dirty[j] = 1u;
         if (A::kId == kHS && ct == 0) p.dirty[s] = 1u;
+        if (p.multi) bar_sync(kConsumerBar, kConsumers);  // the marks precede the ticket's completion
       }
 
       // ---- per-shard bookkeeping: convergence flag (line 26), predictor, trace
@@ -622,10 +698,13 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
             atomicAdd(&t->wb_stores, s_stores);
           }
         }
+        // overlapped passes: every consumer's stores precede this (barrier above; fences are cumulative)
+        if (p.multi) ticket_done(p, s, it, Sloc);
       }
     }
   }
   __syncthreads();
+  if (p.multi) return;  // overlapped passes: the last ticket of a pass closed it (ticket_done)
 
   // ---- iteration close (L189): the last CTA to finish decides whether another pass follows
   if (tid == 0) {
@@ -634,7 +713,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
     if (t == gridDim.x - 1) {
       __threadfence();
       const uint32_t changed = *reinterpret_cast<volatile uint32_t*>(&p.ctl->changed);
-      const uint32_t nit = it + 1;
+      const uint32_t nit = it0 + 1;
       p.ctl->iter = nit;
       p.ctl->changed = 0;
       p.ctl->ctas_done = 0;
@@ -703,6 +782,7 @@ __global__ void init_vertex_values(const KParams p, const void* user) {
   for (size_t s = blockIdx.x * (size_t)blockDim.x + threadIdx.x; s < p.S; s += (size_t)gridDim.x * blockDim.x) {
     p.active[s] = 1;
     if (p.dirty) p.dirty[s] = 1u;  // every shard runs the first pass
+    p.shard_seq[s] = 0;
   }
 }
 
@@ -740,6 +820,9 @@ __global__ void reset_ctl(Ctl* ctl, uint32_t max_iters) {
   ctl->next_shard = 0;
   ctl->gchanged = 0;
   ctl->rctas_done = 0;
+  ctl->ticket = 0;
+  ctl->stop = 0;
+  ctl->conv_iter = 0xFFFFFFFFu;
 }
 
 // -------------------------------------------------------------- dispatch
@@ -792,6 +875,7 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.splitP = (uint32_t)g.splitP; p.splitQ = (uint32_t)g.splitQ;
   p.dest_h = g.h_dest; p.ev_h = g.h_ev; p.srcloc_h = g.h_srcloc; p.cw_src_h = g.h_cw_src; p.mapper_h = g.h_mapper;
   p.use_cond = 0; p.cond_handle = 0;
+  p.multi = 0; p.shard_seq = g.d_shard_seq;
   return p;
 }
 

@@ -48,6 +48,7 @@ class BuildOpts(ctypes.Structure):
         ("nccl_unique_id", ctypes.c_void_p),
         ("skip_clean_shards", ctypes.c_int),
         ("device_topology_budget", ctypes.c_uint64),
+        ("pass_barrier", ctypes.c_int),
     ]
 
 
@@ -214,12 +215,14 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
                 smem_bytes_per_vertex: int = 0, device: int = 0, stream: Optional[int] = None,
                 host_loop: bool = False, world_size: int = 1, rank: int = 0,
                 nccl_id: Optional[bytes] = None, skip_clean_shards: bool = False,
-                device_topology_budget: int = 0) -> Graph:
+                device_topology_budget: int = 0, pass_barrier: bool = False) -> Graph:
     """cusha_build_graph.  src/dst/edge_values: numpy (host, copied in) or CUDA tensors (device).
     world_size > 1: destination-range partition; nccl_id = None simulates all
     partitions on this device, else one process per GPU over NCCL.
     skip_clean_shards: opt-in exact skipping of shards whose inputs did not change.
-    device_topology_budget: HBM bytes for per-entry topology; the rest is streamed from pinned host memory."""
+    device_topology_budget: HBM bytes for per-entry topology; the rest is streamed from pinned host memory.
+    pass_barrier: one launch per pass with a device-wide barrier between passes (Fig. 5) instead of
+    the default overlapped passes (one launch per run)."""
     on_dev = _is_device(src)
     if not on_dev:
         src = np.ascontiguousarray(src, dtype=np.uint32)
@@ -242,6 +245,7 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
     o.rank = rank
     o.skip_clean_shards = int(skip_clean_shards)
     o.device_topology_budget = int(device_topology_budget)
+    o.pass_barrier = int(pass_barrier)
     idbuf = None
     if nccl_id is not None:
         if len(nccl_id) != 128:

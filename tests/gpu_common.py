@@ -13,9 +13,9 @@ D = 0.85
 
 
 def gpu_run(alg, V, src, dst, ev=None, repr="gs", N=0, source=0, init=None, max_iters=1 << 20, expect_converged=True,
-            host_loop=False, skip=False, world_size=1):
+            host_loop=False, skip=False, world_size=1, pass_barrier=False):
     with cusha.build_graph(V, src, dst, edge_values=ev, repr=repr, vertices_per_shard=N, host_loop=host_loop,
-                           skip_clean_shards=skip, world_size=world_size) as g:
+                           skip_clean_shards=skip, world_size=world_size, pass_barrier=pass_barrier) as g:
         if init is not None:
             cusha.set_vertex_values(g, alg, init)
         rc = cusha.run(alg, g, source=source, max_iters=max_iters)

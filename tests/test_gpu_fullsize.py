@@ -33,7 +33,7 @@ def c2():
 
 def test_c2_pagerank_vs_oracle(c2):
     got, st = run("pr", c2)
-    assert st["num_shards"] == 1430 and st["device_loop"] == 1
+    assert st["num_shards"] == 1430 and st["device_loop"] in (1, 2)
     x_star, sweeps = oracle.pagerank(c2.V, c2.src, c2.dst, tol=1e-9)
     maxerr, n_abs = pr_check(got, x_star)
     print(f"C2 PR: {st['iterations']} passes, max|err| {maxerr:.2e}, {n_abs} vertices over 1e-4 abs")

@@ -1,0 +1,106 @@
+"""Overlapped passes (row a5) against the
+oracle and against the one-launch-per-pass barrier mode (Fig. 5).
+
+Default runs draw shard tickets across pass boundaries inside one launch
+(at most two passes in flight, a shard's passes in order); convergence is
+concluded when two consecutive passes committed nothing (L189; the argument
+is in csrc/kernels.cu).  The
+integer fixed points are unique, so both modes must match the oracle bit for
+bit; PR stays within R10.  Small |S| (down to one shard) exercises the
+per-shard pass order, where a CTA's next ticket is the shard it is still
+processing.
+"""
+import numpy as np
+import pytest
+
+import graphgen
+import oracle
+from gpu_common import gpu_run, pr_check
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def c1():
+    wl = graphgen.workload("C1")
+    return wl.V, wl.src, wl.dst, wl.edge_u32
+
+
+@pytest.mark.parametrize("barrier", [False, True])
+@pytest.mark.parametrize("repr", ["gs", "cw"])
+@pytest.mark.parametrize("alg", ["bfs", "sssp", "sswp", "cc"])
+def test_integer_both_modes(c1, alg, repr, barrier):
+    V, s, d, w = c1
+    want = {"bfs": lambda: oracle.bfs(V, s, d, 0), "sssp": lambda: oracle.sssp(V, s, d, w, 0),
+            "sswp": lambda: oracle.sswp(V, s, d, w, 0), "cc": lambda: oracle.cc(V, s, d)}[alg]()
+    got, st = gpu_run(alg, V, s, d, ev=w if alg in ("sssp", "sswp") else None, repr=repr, N=128,
+                      pass_barrier=barrier)
+    np.testing.assert_array_equal(got, want)
+    assert st["converged"] == 1
+    assert st["device_loop"] == (1 if barrier else 2)
+
+
+@pytest.mark.parametrize("N", [4096, 2048, 1366, 64, 7])
+def test_small_shard_counts(c1, N):
+    """|S| = 1, 2, 3 (fewer shards than CTAs: tickets of consecutive passes hit
+    the same shard), and many tiny shards."""
+    V, s, d, w = c1
+    want = oracle.sssp(V, s, d, w, 0)
+    for repr in ("gs", "cw"):
+        got, st = gpu_run("sssp", V, s, d, ev=w, repr=repr, N=N)
+        np.testing.assert_array_equal(got, want)
+        assert st["converged"] == 1
+
+
+def test_mesh_many_passes():
+    """A high-diameter mesh: hundreds of overlapped passes, then a confirming one."""
+    wl = graphgen.workload("mesh:60000:120:80000:41")
+    want = oracle.sssp(wl.V, wl.src, wl.dst, wl.edge_u32, 0)
+    for barrier in (False, True):
+        got, st = gpu_run("sssp", wl.V, wl.src, wl.dst, ev=wl.edge_u32, repr="cw", N=512, pass_barrier=barrier)
+        np.testing.assert_array_equal(got, want)
+        assert st["iterations"] > 50
+
+
+@pytest.mark.parametrize("barrier", [False, True])
+def test_pagerank_both_modes(barrier):
+    V = 1 << 15
+    s, d = graphgen.rmat(V, 1 << 19, seed=31)
+    x_star, _ = oracle.pagerank(V, s, d, tol=1e-9)
+    for repr in ("gs", "cw"):
+        got, st = gpu_run("pr", V, s, d, repr=repr, pass_barrier=barrier)
+        pr_check(got, x_star)
+        assert st["converged"] == 1
+
+
+def test_max_iters_stops_exactly(c1):
+    """max_iters = k: NOT_CONVERGED after exactly k passes in both modes (R23)."""
+    from paper_conf_hpdc_khorasanivgb14_b200 import cusha
+    wl = graphgen.workload("mesh:20000:100:26000:43")
+    for barrier in (False, True):
+        for k in (1, 3, 10):
+            with cusha.build_graph(wl.V, wl.src, wl.dst, edge_values=wl.edge_u32, repr="cw", vertices_per_shard=256,
+                                   pass_barrier=barrier) as g:
+                rc = cusha.run("sssp", g, source=0, max_iters=k)
+                st = cusha.get_stats(g)
+                assert rc == cusha.NOT_CONVERGED and st["iterations"] == k and st["converged"] == 0
+                vals = cusha.get_values(g)
+                # committed values are upper bounds of the exact distances, source exact
+                exact = oracle.sssp(wl.V, wl.src, wl.dst, wl.edge_u32, 0)
+                assert vals[0] == 0 and np.all(vals >= exact)
+
+
+def test_trace_cap_fallback(c1):
+    """max_iters above the per-pass trace capacity (2^20) uses the one-launch-per-pass loop."""
+    V, s, d, _ = c1
+    got, st = gpu_run("bfs", V, s, d, repr="cw", N=128, max_iters=(1 << 20) + 1)
+    np.testing.assert_array_equal(got, oracle.bfs(V, s, d, 0))
+    assert st["device_loop"] == 1
+
+
+def test_skip_clean_with_overlap():
+    wl = graphgen.workload("mesh:40000:200:52000:33")
+    want = oracle.sssp(wl.V, wl.src, wl.dst, wl.edge_u32, 0)
+    for repr in ("gs", "cw"):
+        got, st = gpu_run("sssp", wl.V, wl.src, wl.dst, ev=wl.edge_u32, repr=repr, N=400, skip=True)
+        np.testing.assert_array_equal(got, want)

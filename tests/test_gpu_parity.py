@@ -216,9 +216,12 @@ def test_layout_matches_oracle(repr, V, E, N):
 # ----------------------------------------------------------- edge cases
 @pytest.mark.parametrize("repr", REPRS)
 def test_edge_cases(repr):
-    # empty graph: one pass, nothing changes
-    got, st = gpu_run("bfs", 10, np.zeros(0, np.uint32), np.zeros(0, np.uint32), repr=repr, source=3)
-    assert got[3] == 0 and (np.delete(got, 3) == cusha.INF).all() and st["iterations"] == 1
+    # empty graph: nothing changes; the barrier mode stops after one clean pass,
+    # overlapped passes after two consecutive clean ones
+    for barrier, passes in ((True, 1), (False, 2)):
+        got, st = gpu_run("bfs", 10, np.zeros(0, np.uint32), np.zeros(0, np.uint32), repr=repr, source=3,
+                          pass_barrier=barrier)
+        assert got[3] == 0 and (np.delete(got, 3) == cusha.INF).all() and st["iterations"] == passes
     # single vertex
     got, _ = gpu_run("cc", 1, np.zeros(0, np.uint32), np.zeros(0, np.uint32), repr=repr)
     assert got.tolist() == [0]
