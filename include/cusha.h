@@ -164,6 +164,8 @@ typedef struct {
   int world_size, rank;
   uint64_t host_bytes;             /* per-entry topology bytes held in pinned host memory (f3)  */
   uint32_t host_shard;             /* first shard whose topology is host-resident (|S|: none)   */
+  uint32_t mapper_form;            /* last run, CW: 1 = stage 4 used the Mapper in window form
+                                      (u16 window index per entry + per-shard delta row), 0 = u32 Mapper */
 } cusha_stats;
 
 /* ---------------------------------------------------------------- build */
@@ -254,7 +256,10 @@ typedef enum {
   CUSHA_LAYOUT_MAPPER = 9,          /* u32[Q]     padded shard position (filler = trash P)  */
   CUSHA_LAYOUT_OUT_DEGREE = 10,     /* u32[|V|]   out-degree (PR NbrsNum, L318)            */
   CUSHA_LAYOUT_RUN_K = 11,          /* u32[R]     CW position of each Mapper run's first entry (CW) */
-  CUSHA_LAYOUT_RUN_T = 12           /* u32[R]     its Mapper target; one run per non-empty W_ij      */
+  CUSHA_LAYOUT_RUN_T = 12,          /* u32[R]     its Mapper target; one run per non-empty W_ij      */
+  CUSHA_LAYOUT_CW_WINDOW = 13,      /* u16[Q]     j of the window W_ij holding each CW_i entry (filler 0xFFFF) */
+  CUSHA_LAYOUT_CW_DELTA = 14        /* u32[|S|*|S|] Mapper in window form: Mapper[k] = delta[i*|S|+j] + k
+                                                  (mod 2^32) for every real entry k of CW_i in W_ij  */
 } cusha_layout_part;
 /* Returns the element count of `part` in *count (bytes = count * element size);
  * copies it to `out` (host) when out != NULL and out_bytes is large enough.

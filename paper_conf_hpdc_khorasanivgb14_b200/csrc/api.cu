@@ -43,7 +43,7 @@ static void free_graph_memory(Graph& g) {
   void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcloc, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
                   g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_srcvalue, g.d_vv, g.d_ctl, g.d_trace,
                   g.d_active, g.d_bounds, g.d_owner, g.d_cwp, g.d_gathered, g.d_run_k, g.d_run_t,
-                  g.d_run_unit, g.d_run_bits, g.d_run_d, g.d_dirty, g.d_shard_seq};
+                  g.d_run_unit, g.d_run_bits, g.d_run_d, g.d_dirty, g.d_shard_seq, g.d_cw_win, g.d_cw_delta};
   nccl_destroy(g);
   // device memory is stream-ordered (cudaMallocAsync on g.stream): released to
   // the retained pool without unmapping or a device-wide synchronisation
@@ -51,7 +51,7 @@ static void free_graph_memory(Graph& g) {
     if (p) cudaFreeAsync(p, g.stream);
   for (void*& p : g.d_init)
     if (p) { cudaFreeAsync(p, g.stream); p = nullptr; }
-  void* hosts[] = {g.h_dest, g.h_ev, g.h_srcloc, g.h_eid, g.h_cw_src, g.h_mapper};
+  void* hosts[] = {g.h_dest, g.h_ev, g.h_srcloc, g.h_eid, g.h_cw_src, g.h_mapper, g.h_cw_win};
   for (void* p : hosts)
     if (p) cudaFreeHost(p);
   delete g.h_ctl;
@@ -81,7 +81,8 @@ static uint64_t device_bytes(const Graph& g) {
   if (g.has_ev) b += 4 * g.P;
   if (g.d_srcloc) b += 2 * g.P;
   if (g.d_win) b += 4ull * (g.S + 1) * g.S;
-  b += (2 + 4) * g.Q;                                   // CW
+  b += (2 + 4 + 2) * g.Q;                               // CW: SrcIndexCW, Mapper, window
+  if (g.d_cw_delta) b += 4ull * g.S * g.S;             // Mapper deltas per window
   b += 4ull * g.V;                                      // outdeg
   b += 4 * (g.P + 1) + 8ull * g.V;                      // SrcValue + VertexValues
   return b - g.host_bytes;                              // minus the host-streamed part (row f3)
@@ -302,15 +303,45 @@ static uint32_t pass_grid(const Graph& g, const PassKernel& pk, size_t smem) {
   return (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(gsz, mine));
 }
 
+// Shared memory of the pass and the CW Mapper form (DESIGN.md "Mapper in
+// window form"): the window form (SrcIndexCW + u16 window index per entry, the
+// shard's delta row in shared memory) whenever the row fits without lowering
+// the CTAs per SM; otherwise the u32 Mapper.  Sets the kernel attributes.
+#ifndef CUSHA_MAPJ
+#define CUSHA_MAPJ 1  // 0: always the u32 Mapper (tuning comparison)
+#endif
+static int pass_config(const Graph& g, const PassKernel& pk, size_t* smem, int* mapj) {
+  cudaFuncAttributes fa{};
+  CKA(cudaFuncGetAttributes(&fa, pk.func));
+  const size_t kMaxSmem = 227 * 1024 - fa.sharedSizeBytes;  // dynamic part of the 227 KB per-CTA limit
+  const size_t sm_m = pk.smem_bytes(g.N);
+  if (sm_m > kMaxSmem)
+    return fail(CUSHA_EINVAL, "vertices_per_shard too large for this algorithm's shared-memory state");
+  CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem));
+  CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared));
+  *smem = sm_m;
+  *mapj = 0;
+  const size_t sm_j = pk.smem_bytes(g.N, g.S);
+  if (CUSHA_MAPJ && g.repr == CUSHA_REPR_CW && g.d_cw_win && g.d_cw_delta && !kernels_rle() && g.S <= 0xFFFFu && sm_j <= kMaxSmem) {
+    int occ_m = 0, occ_j = 0;
+    CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_m, pk.func, (int)pk.threads, sm_m));
+    CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_j, pk.func, (int)pk.threads, sm_j));
+    if (occ_j >= occ_m && occ_j > 0) {
+      *smem = sm_j;
+      *mapj = 1;
+    }
+  }
+  return CUSHA_OK;
+}
+
 static int ensure_exec(cusha_graph* h, int alg) {
   Graph& g = h->g;
   if (h->exec[alg]) return CUSHA_OK;
   const PassKernel& pk = pass_kernel(alg, g.repr);
-  const size_t smem = pk.smem_bytes(g.N);
-  if (smem > 227 * 1024)
-    return fail(CUSHA_EINVAL, "vertices_per_shard too large for this algorithm's shared-memory state");
-  CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared));
+  size_t smem = 0;
+  int mapj = 0;
+  const int prc = pass_config(g, pk, &smem, &mapj);
+  if (prc) return prc;
   cudaGraph_t graph = nullptr;
   CKA(cudaGraphCreate(&graph, 0));
   cudaGraphConditionalHandle handle;
@@ -327,6 +358,7 @@ static int ensure_exec(cusha_graph* h, int alg) {
   cudaGraph_t body = cp.conditional.phGraph_out[0];
   KParams kp = make_params(g, 0);
   kp.use_cond = 1;
+  kp.mapj = mapj;
   kp.cond_handle = handle;
   void* args[] = {&kp};
   cudaKernelNodeParams knp = {};
@@ -364,18 +396,15 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
       if (e) { cudaGraphExecDestroy(e); e = nullptr; }
   }
   const PassKernel& pk = pass_kernel(a, g.repr);
-  const size_t smem = pk.smem_bytes(g.N);
-  int rc = CUSHA_OK;
+  size_t smem = 0;
+  int mapj = 0;
+  int rc = pass_config(g, pk, &smem, &mapj);
+  if (rc) return rc;
   const bool host_loop = g.host_loop || g.G > 1;  // the partitioned mode exchanges between passes
   // overlapped passes (default): one launch runs every pass; it needs a trace
   // record per pass (<= 2^20), else the CUDA-graph loop runs one launch per pass
   const bool multi = !host_loop && !g.pass_barrier && max_iters <= g.trace_cap;
-  if (host_loop || multi) {
-    if (smem > 227 * 1024)
-      return fail(CUSHA_EINVAL, "vertices_per_shard too large for this algorithm's shared-memory state");
-    CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared));
-  } else {
+  if (!host_loop && !multi) {
     rc = ensure_exec(h, a);
     if (rc) return rc;
   }
@@ -387,6 +416,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   if (max_iters > 0 && multi) {
     KParams kp = make_params(g, source);
     kp.multi = 1;
+    kp.mapj = mapj;
     void* args[] = {&kp};
     CKA(cudaLaunchKernel(pk.func, dim3(pass_grid(g, pk, smem)), dim3(pk.threads), args, smem, g.stream));
   } else if (max_iters > 0 && !host_loop) {
@@ -399,6 +429,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     // windows + global convergence; every rank takes the same decisions
     // from the same exchanged data, so all issue the same collectives.
     KParams kp = make_params(g, source);
+    kp.mapj = mapj;
     void* args[] = {&kp};
     const dim3 grid(pass_grid(g, pk, smem));
     const int chunk = g.G > 1 && !g.simulate ? 1 : 8;
@@ -443,8 +474,9 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     bytes += (uint64_t)tr[i].updated * vb;                            // stage 3 commits
     bytes += tr[i].edges * (4 + 2 + evb);                             // stage 2
     edges += tr[i].edges;
-    if (g.repr == CUSHA_REPR_CW)
-      bytes += tr[i].wb_entries * 6 + tr[i].wb_stores * 4;            // SrcIndexCW + Mapper, SrcValue
+    if (g.repr == CUSHA_REPR_CW)  // SrcIndexCW + window index (+ delta row) or u32 Mapper; SrcValue
+      bytes += tr[i].wb_entries * (mapj ? 4 : 6) + tr[i].wb_stores * 4 +
+               (mapj ? (uint64_t)tr[i].shards * 4ull * g.S : 0);
     else
       bytes += tr[i].wb_entries * 4 + tr[i].wb_stores * 4 + (uint64_t)tr[i].active_shards * 8ull * g.S;
   }
@@ -457,7 +489,8 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   g.st.algorithmic_bytes = bytes;
   g.st.edges_processed = n == c.iter ? edges : (uint64_t)c.iter * g.E;
   g.st.stage2_bytes_per_iter = g.E * (4 + 2 + evb);
-  g.st.wb_bytes_all_active = g.repr == CUSHA_REPR_CW ? g.E * 10 : g.E * 8;
+  g.st.wb_bytes_all_active = g.repr == CUSHA_REPR_CW ? g.E * (mapj ? 8 : 10) : g.E * 8;
+  g.st.mapper_form = (uint32_t)mapj;
   g.st.device_loop = host_loop ? 0 : (multi ? 2 : 1);
   g.last_alg = a;
   g.have_values = true;
@@ -535,6 +568,8 @@ int cusha_get_layout(const cusha_graph* h, cusha_layout_part part, void* out, si
     case CUSHA_LAYOUT_OUT_DEGREE: src = g.d_outdeg; n = g.V; break;
     case CUSHA_LAYOUT_RUN_K: src = g.d_run_k; n = g.R; break;
     case CUSHA_LAYOUT_RUN_T: src = g.d_run_t; n = g.R; break;
+    case CUSHA_LAYOUT_CW_WINDOW: src = g.d_cw_win; tail = g.h_cw_win; split = g.splitQ; n = g.Q; es = 2; break;
+    case CUSHA_LAYOUT_CW_DELTA: src = g.d_cw_delta; n = (uint64_t)g.S * g.S; break;
     default: return fail(CUSHA_EINVAL, "bad layout part");
   }
   if (!src && !tail) return fail(CUSHA_EUNSUPPORTED, "part not held by this representation");

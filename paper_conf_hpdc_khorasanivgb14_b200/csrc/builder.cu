@@ -166,7 +166,7 @@ __global__ void k_pad_counts(const uint32_t* cnt, uint32_t S, uint64_t* padded) 
 __global__ void __launch_bounds__(256) k_cw_from_windows(const uint32_t* __restrict__ win, uint32_t S,
                                                          const uint32_t* __restrict__ cw_off,
                                                          const uint16_t* __restrict__ srcidx, uint16_t* cw_src,
-                                                         uint32_t* mapper) {
+                                                         uint32_t* mapper, uint16_t* cw_win, uint32_t* cw_delta) {
   typedef cub::BlockScan<uint32_t, 256> BS;
   __shared__ typename BS::TempStorage tmp;
   __shared__ uint32_t s_off[257], s_beg[256];
@@ -183,6 +183,9 @@ __global__ void __launch_bounds__(256) k_cw_from_windows(const uint32_t* __restr
     s_off[tid] = ex;
     s_beg[tid] = b;
     if (tid == 0) s_off[256] = total;
+    // Mapper in window form: W_ij's entries sit at CW positions base+ex.. and
+    // shard positions b.., so Mapper[k] = (b - (base + ex)) + k (mod 2^32)
+    if (j < S) cw_delta[(size_t)i * S + j] = b - (base + ex);
     __syncthreads();
     for (uint32_t f = tid; f < total; f += 256) {
       uint32_t lo = 0, hi = 256;  // last window w with s_off[w] <= f
@@ -193,6 +196,7 @@ __global__ void __launch_bounds__(256) k_cw_from_windows(const uint32_t* __restr
       }
       const uint32_t pos = s_beg[lo] + (f - s_off[lo]);
       mapper[base + f] = pos;
+      cw_win[base + f] = (uint16_t)(j0 + lo);
       cw_src[base + f] = srcidx[pos];  // SrcIndex - i*N
     }
     base += total;
@@ -200,13 +204,14 @@ __global__ void __launch_bounds__(256) k_cw_from_windows(const uint32_t* __restr
   }
 }
 __global__ void k_fill_cw_pads(const uint32_t* coff, const uint32_t* ccnt, uint32_t S, uint32_t trash, uint16_t* cw_src,
-                               uint32_t* mapper) {
+                               uint32_t* mapper, uint16_t* cw_win) {
   GRID_STRIDE(i, (uint64_t)S * kPad) {
     const uint32_t s = (uint32_t)(i / kPad), r = (uint32_t)(i % kPad);
     const uint32_t pos = coff[s] + ccnt[s] + r;
     if (pos < coff[s + 1]) {
       cw_src[pos] = 0;
       mapper[pos] = trash;
+      cw_win[pos] = 0xFFFFu;
     }
   }
 }
@@ -465,9 +470,13 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
     k_narrow<<<grid_for((uint64_t)S + 1), 256, 0, st>>>((uint64_t*)cscan.p, (uint64_t)S + 1, g.d_cw_off);
     CK(dalloc(&g.d_cw_src, Q));
     CK(dalloc(&g.d_mapper, Q));
+    CK(dalloc(&g.d_cw_win, Q));
+    CK(dalloc(&g.d_cw_delta, (uint64_t)S * S));
     k_fill_cw_pads<<<grid_for((uint64_t)S * kPad), 256, 0, st>>>(g.d_cw_off, g.d_cw_cnt, S, (uint32_t)P,
-                                                                  g.d_cw_src, g.d_mapper);
-    if (E) k_cw_from_windows<<<S, 256, 0, st>>>(g.d_win, S, g.d_cw_off, g.d_srcloc, g.d_cw_src, g.d_mapper);
+                                                                  g.d_cw_src, g.d_mapper, g.d_cw_win);
+    if (E)
+      k_cw_from_windows<<<S, 256, 0, st>>>(g.d_win, S, g.d_cw_off, g.d_srcloc, g.d_cw_src, g.d_mapper, g.d_cw_win,
+                                           g.d_cw_delta);
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(st));
     // CW keeps the 3-tuple shards + SrcIndexCW + Mapper (L175): no per-entry SrcIndex in shard order
@@ -534,7 +543,7 @@ int offload_topology(Graph& g, std::string& err) {
   if (g.d_cw_off) CK(cudaMemcpyAsync(co.data(), g.d_cw_off, 4ull * (S + 1), cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   const uint64_t bP = 2 + 4 + (g.has_ev ? 4 : 0) + (g.d_srcloc ? 2 : 0);  // DestIndex, edge id, EdgeValue, SrcIndex
-  const uint64_t bQ = g.d_cw_src ? 6 : 0;                                  // SrcIndexCW, Mapper
+  const uint64_t bQ = g.d_cw_src ? 8 : 0;                                  // SrcIndexCW, Mapper, window
   uint32_t h = 0;
   while (h < S && (uint64_t)so[h + 1] * bP + (uint64_t)co[h + 1] * bQ <= g.topo_budget) ++h;
   g.host_shard = h;
@@ -546,7 +555,8 @@ int offload_topology(Graph& g, std::string& err) {
       (rc = move_tail(g.d_eid, g.h_eid, g.P, g.splitP, st, g.host_bytes, err)) ||
       (rc = move_tail(g.d_srcloc, g.h_srcloc, g.P, g.splitP, st, g.host_bytes, err)) ||
       (rc = move_tail(g.d_cw_src, g.h_cw_src, g.Q, g.splitQ, st, g.host_bytes, err)) ||
-      (rc = move_tail(g.d_mapper, g.h_mapper, g.Q, g.splitQ, st, g.host_bytes, err)))
+      (rc = move_tail(g.d_mapper, g.h_mapper, g.Q, g.splitQ, st, g.host_bytes, err)) ||
+      (rc = move_tail(g.d_cw_win, g.h_cw_win, g.Q, g.splitQ, st, g.host_bytes, err)))
     return rc;
   CK(cudaStreamSynchronize(st));
   return CUSHA_OK;

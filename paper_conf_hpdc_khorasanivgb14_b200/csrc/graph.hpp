@@ -55,6 +55,8 @@ struct KParams {
   uint8_t* active;             // S: shard ran stage 4 in the last pass (stage-4 prefetch predictor; exchanged)
   const uint16_t* cw_src;      // CW: Q local SrcIndex
   const uint32_t* mapper;      // CW: Q padded shard positions
+  const uint16_t* cw_win;      // CW: Q target shard j of each entry (filler: 0xFFFF)
+  const uint32_t* cw_delta;    // CW: S*S, Mapper[k] = cw_delta[i*S + j] + k for k in W_ij's part of CW_i
   void* vv;                    // VertexValues
   const uint32_t* outdeg;      // V out-degrees (PR NbrsNum)
   Ctl* ctl;
@@ -63,6 +65,7 @@ struct KParams {
   int use_cond;
   unsigned long long cond_handle;
   int multi;                   // 1: one launch runs every pass (overlapped passes)
+  int mapj;                    // 1: CW stage 4 uses the Mapper in window form (cw_win + delta row in smem)
   uint32_t* shard_seq;         // S: passes of shard s completed (overlapped passes)
   // destination-range partition (row e); G = 1: single partition
   uint32_t G;                  // partitions
@@ -90,6 +93,7 @@ struct KParams {
   const uint16_t* srcloc_h;
   const uint16_t* cw_src_h;
   const uint32_t* mapper_h;
+  const uint16_t* cw_win_h;
 };
 
 // element i of a topology array split between HBM (i < split) and pinned host memory
@@ -106,7 +110,7 @@ struct PassKernel {
   uint32_t ring_bytes;    // TMA tile ring
   uint32_t threads;       // CTA size (producer warp + consumer warps)
   bool persistent;        // grid = resident CTAs pulling shards from a queue (else one CTA per shard)
-  size_t smem_bytes(uint32_t N) const;
+  size_t smem_bytes(uint32_t N, uint32_t delta_row = 0) const;  // delta_row: words of the window-form row
 };
 
 struct Graph {
@@ -130,6 +134,7 @@ struct Graph {
   uint32_t* d_dirty = nullptr;      // S: clean-shard skipping flags
   uint32_t* d_shard_seq = nullptr;  // S: overlapped passes, per-shard pass order
   bool pass_barrier = false;        // 1: one launch per pass (CUDA-graph while loop)
+  int mapj = -1;                    // per-run choice of the Mapper form (-1: not chosen yet)
   bool skip_clean = false;
   // host-streamed topology (row f3): shards >= host_shard keep their entry
   // arrays (and CW_i arrays) in pinned, mapped host memory
@@ -145,6 +150,9 @@ struct Graph {
   uint64_t host_bytes = 0;
   uint16_t* d_cw_src = nullptr;     // Q (CW)
   uint32_t* d_mapper = nullptr;     // Q (CW)
+  uint16_t* d_cw_win = nullptr;     // Q (CW): target shard of each entry (Mapper in window form)
+  uint32_t* d_cw_delta = nullptr;   // S*S (CW): Mapper - CW position, per window
+  uint16_t* h_cw_win = nullptr;     // Q - splitQ (row f3)
   uint32_t R = 0;                   // Mapper runs (non-empty windows)
   uint32_t* d_run_k = nullptr;      // R+pad
   uint32_t* d_run_t = nullptr;      // R+pad
@@ -185,6 +193,8 @@ cudaError_t launch_reset_ctl(Ctl* ctl, uint32_t max_iters, cudaStream_t s);
 cudaError_t launch_refresh(const Graph& g, cudaStream_t s);
 KParams make_params(const Graph& g, uint32_t source);
 size_t value_bytes(int alg);
+bool kernels_rle();  // built with the Mapper-runs stage 4 (CUSHA_RLE)
+
 bool alg_needs_edge_values(int alg);
 bool alg_needs_init(int alg);
 

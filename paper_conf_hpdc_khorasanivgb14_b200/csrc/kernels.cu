@@ -98,6 +98,20 @@ constexpr uint32_t run_cap() {
 #define CUSHA_RLE 0  // measured slower (the pass is consumer-bound): DESIGN.md "Tuning log"
 #endif
 constexpr bool kRle = CUSHA_RLE != 0;  // stream Mapper as runs
+// Mapper in window form, chosen per run
+// (KParams::mapj) when the shard's delta row fits in shared memory without
+// costing occupancy: a stage-4 tile then carries SrcIndexCW and the u16
+// window index j of each entry (4 B per entry instead of 6 B with the u32
+// Mapper), and Mapper[k] = delta_row[j] + k with the row loaded in stage 1.
+// Stage-4 entries per tile: a whole slot in either form.
+template <class A>
+constexpr uint32_t tile4j_of() {
+  return slot_bytes<A>() / 4 / 8 * 8;
+}
+template <class A>
+constexpr uint32_t tile4m_of() {
+  return kRle ? tile_of<A>() : slot_bytes<A>() / 6 / 8 * 8;
+}
 #ifndef CUSHA_DIAG
 #define CUSHA_DIAG 0
 #endif
@@ -412,10 +426,11 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     }
     if (send4) {
       // [lo, hi) marks the valid part of each tile
+      const uint32_t kT4 = p.mapj ? tile4j_of<A>() : tile4m_of<A>();
       if (a >= b2) push(s, kDescStage4, 0, kFlagLast, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
       else
-        for (uint32_t k0 = kb; k0 < ke; k0 += kTile) {
-          const uint32_t n = min(kTile, ke - k0);
+        for (uint32_t k0 = kb; k0 < ke; k0 += kT4) {
+          const uint32_t n = min(kT4, ke - k0);
           const uint32_t fl = k0 + n >= ke ? kFlagLast : 0u, lo = a > k0 ? a - k0 : 0u, hi = min(b2 - k0, n);
           if (kRle) {
             // runs from the one containing position k0/128*128 (the slot's first
@@ -433,8 +448,12 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
               continue;
             }
           }
-          push(s, kDescStage4, n, fl, topo_at(p.cw_src, p.cw_src_h, p.splitQ, k0), n * 2,
-               topo_at(p.mapper, p.mapper_h, p.splitQ, k0), 2 * kTile, n * 4, nullptr, 0, 0, lo, hi, k0, 0);
+          if (p.mapj)
+            push(s, kDescStage4, n, fl, topo_at(p.cw_src, p.cw_src_h, p.splitQ, k0), n * 2,
+                 topo_at(p.cw_win, p.cw_win_h, p.splitQ, k0), 2 * kT4, n * 2, nullptr, 0, 0, lo, hi, k0, 0);
+          else
+            push(s, kDescStage4, n, fl, topo_at(p.cw_src, p.cw_src_h, p.splitQ, k0), n * 2,
+                 topo_at(p.mapper, p.mapper_h, p.splitQ, k0), 2 * kT4, n * 4, nullptr, 0, 0, lo, hi, k0, 0);
         }
     }
   }
@@ -456,6 +475,8 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
   const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
   const uint32_t N = p.N, st = N + 1;
   uint32_t* const aux = sm + A::kWords * st;  // write-back values (float algs) or changed bits (integer algs)
+  // Mapper-delta row of the current shard (window form, p.mapj): after aux
+  uint32_t* const drow = aux + (A::kMonotone ? (N + 31) / 32 : N);
   const uint32_t it0 = *reinterpret_cast<volatile uint32_t*>(&p.ctl->iter);
   // a pass launched after the run converged / hit max_iters is a no-op (host-loop mode)
   if (*reinterpret_cast<volatile uint32_t*>(&p.ctl->converged) || it0 >= p.ctl->max_iters) return;
@@ -493,13 +514,18 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
 #pragma unroll
         for (uint32_t u = 0; u < kVB; ++u) {
           const uint32_t v = base + u * kConsumers + ct;
-          if (v < nv) x[u] = vv[v];
+          x[u] = V_t{};
+          if (A::kInitReadsV && v < nv) x[u] = vv[v];
         }
 #pragma unroll
         for (uint32_t u = 0; u < kVB; ++u) {
           const uint32_t v = base + u * kConsumers + ct;
           if (v < nv) A::init(sm, st, v, x[u]);
         }
+      }
+      if (p.mapj) {  // the shard's Mapper-delta row for stage 4 (window form)
+        const uint32_t* dg = p.cw_delta + (size_t)s * p.S;
+        for (uint32_t j = ct; j < p.S; j += kConsumers) drow[j] = __ldg(dg + j);
       }
       if (ct == 0) {
         A::init(sm, st, N, V_t{});  // trash slot for filler entries
@@ -633,9 +659,21 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
                   r += __popc(word);
                 }
               }
+            } else if (any && p.mapj) {
+              // SrcValue[delta_row[j] + k] = local[SrcIndexCW[k]] for CW position k = base + i
+              const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
+              const uint16_t* J = reinterpret_cast<const uint16_t*>(ring + slot * SLOT + 2 * tile4j_of<A>());
+              for (uint32_t i = d.lo + ct; i < d.hi; i += kConsumers) {
+                const uint32_t j = J[i];
+                uint32_t val;
+                if (j != 0xFFFFu && wb_get<A>(sm, aux, L[i], val)) {
+                  st_u32(p.srcvalue + (drow[j] + d.base + i), val);
+                  ++stores;
+                }
+              }
             } else if (any) {
               const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
-              const uint32_t* M = reinterpret_cast<const uint32_t*>(ring + slot * SLOT + 2 * kTile);
+              const uint32_t* M = reinterpret_cast<const uint32_t*>(ring + slot * SLOT + 2 * tile4m_of<A>());
               for (uint32_t i = d.lo + ct; i < d.hi; i += kConsumers) {
                 const uint32_t m = M[i];
                 uint32_t val;
@@ -826,11 +864,11 @@ __global__ void reset_ctl(Ctl* ctl, uint32_t max_iters) {
 }
 
 // -------------------------------------------------------------- dispatch
-size_t PassKernel::smem_bytes(uint32_t N) const {
+size_t PassKernel::smem_bytes(uint32_t N, uint32_t delta_row) const {
   size_t w = (size_t)words * (N + 1);
   if (wb_array) w += N;
   if (monotone) w += (N + 31) / 32;
-  return ring_bytes + 4 * w;
+  return ring_bytes + 4 * (w + delta_row);
 }
 
 template <class A, int R>
@@ -856,6 +894,9 @@ const PassKernel& pass_kernel(int alg, int repr) {
   return table[alg][repr];
 }
 
+
+bool kernels_rle() { return kRle; }
+
 size_t value_bytes(int alg) { return (alg == kHS || alg == kCS) ? 8 : 4; }
 bool alg_needs_edge_values(int alg) { return alg == kSSSP || alg == kSSWP || alg == kNN || alg == kHS || alg == kCS; }
 bool alg_needs_init(int alg) { return alg == kNN || alg == kHS || alg == kCS; }
@@ -866,6 +907,7 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.shard_off = g.d_shard_off; p.shard_cnt = g.d_shard_cnt; p.dest = g.d_dest; p.ev = g.d_ev; p.srcvalue = g.d_srcvalue;
   p.srcloc = g.d_srcloc; p.win = g.d_win; p.cw_off = g.d_cw_off; p.cw_cnt = g.d_cw_cnt; p.active = g.d_active;
   p.cw_src = g.d_cw_src; p.mapper = g.d_mapper; p.vv = g.d_vv; p.outdeg = g.d_outdeg;
+  p.cw_win = g.d_cw_win; p.cw_delta = g.d_cw_delta; p.cw_win_h = g.h_cw_win;
   p.ctl = g.d_ctl; p.trace = g.d_trace; p.trace_cap = g.trace_cap;
   p.G = g.G; p.part = g.G > 1 && !g.simulate ? g.rank : -1;
   p.bounds = g.d_bounds; p.owner = g.d_owner; p.cwp = g.d_cwp; p.gathered = g.G > 1 ? g.d_gathered : nullptr;
@@ -876,6 +918,7 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.dest_h = g.h_dest; p.ev_h = g.h_ev; p.srcloc_h = g.h_srcloc; p.cw_src_h = g.h_cw_src; p.mapper_h = g.h_mapper;
   p.use_cond = 0; p.cond_handle = 0;
   p.multi = 0; p.shard_seq = g.d_shard_seq;
+  p.mapj = 0;
   return p;
 }
 

@@ -31,6 +31,7 @@ LAYOUT = {
     "dest_local": (3, np.uint16), "edge_id": (4, np.uint32), "windows": (5, np.uint32),
     "cw_offsets": (6, np.uint32), "cw_sizes": (7, np.uint32), "cw_src_local": (8, np.uint16),
     "mapper": (9, np.uint32), "out_degree": (10, np.uint32), "run_k": (11, np.uint32), "run_t": (12, np.uint32),
+    "cw_window": (13, np.uint16), "cw_delta": (14, np.uint32),
 }
 
 
@@ -78,6 +79,7 @@ class Stats(ctypes.Structure):
         ("rank", ctypes.c_int),
         ("host_bytes", ctypes.c_uint64),
         ("host_shard", ctypes.c_uint32),
+        ("mapper_form", ctypes.c_uint32),
     ]
 
 

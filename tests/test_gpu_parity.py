@@ -177,6 +177,8 @@ def test_layout_matches_oracle(repr, V, E, N):
             mapper = cusha.get_layout(g, "mapper").astype(np.int64)
             run_k = cusha.get_layout(g, "run_k").astype(np.int64)
             run_t = cusha.get_layout(g, "run_t").astype(np.int64)
+            cw_win = cusha.get_layout(g, "cw_window").astype(np.int64)
+            cw_delta = cusha.get_layout(g, "cw_delta").astype(np.int64).reshape(S, S)
     assert st["num_shards"] == S and st["vertices_per_shard"] == N
     np.testing.assert_array_equal(cnt, np.diff(ref["shard_off"].astype(np.int64)))
     assert (off % 8 == 0).all()
@@ -211,6 +213,12 @@ def test_layout_matches_oracle(repr, V, E, N):
         if E:
             r = np.searchsorted(run_k, creal, side="right") - 1
             np.testing.assert_array_equal(run_t[r] + (creal - run_k[r]), mapper[creal])
+        # Mapper in window form: j = the shard the oracle's Mapper target lies in, and
+        # delta[i][j] + k reproduces Mapper exactly; filler entries carry j = 0xFFFF
+        tgt_shard = np.searchsorted(ref_off, ref["mapper"].astype(np.int64), side="right") - 1
+        np.testing.assert_array_equal(cw_win[creal], tgt_shard)
+        np.testing.assert_array_equal((cw_delta[src_shard, cw_win[creal]] + creal) % (1 << 32), mapper[creal])
+        assert (cw_win[cfill] == 0xFFFF).all()
 
 
 # ----------------------------------------------------------- edge cases
