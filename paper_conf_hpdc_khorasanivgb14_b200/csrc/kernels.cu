@@ -474,9 +474,13 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
   using V_t = typename A::Value;
   const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
   const uint32_t N = p.N, st = N + 1;
-  uint32_t* const aux = sm + A::kWords * st;  // write-back values (float algs) or changed bits (integer algs)
-  // Mapper-delta row of the current shard (window form, p.mapj): after aux
-  uint32_t* const drow = aux + (A::kMonotone ? (N + 31) / 32 : N);
+  // aux: the changed bits of stage 3 (integer algorithms), or the write-back
+  // values of local_vertices (float algorithms), which stage 3 stores over the
+  // first fixed-point word of the same vertex: its sum is dead once read
+  uint32_t* const tail = sm + A::kWords * st;
+  uint32_t* const aux = A::kMonotone ? tail : sm + A::acc_lo(0) * st;
+  // Mapper-delta row of the current shard (window form, p.mapj)
+  uint32_t* const drow = tail + (A::kMonotone ? (N + 31) / 32 : 0);
   const uint32_t it0 = *reinterpret_cast<volatile uint32_t*>(&p.ctl->iter);
   // a pass launched after the run converged / hit max_iters is a no-op (host-loop mode)
   if (*reinterpret_cast<volatile uint32_t*>(&p.ctl->converged) || it0 >= p.ctl->max_iters) return;
@@ -865,8 +869,7 @@ __global__ void reset_ctl(Ctl* ctl, uint32_t max_iters) {
 
 // -------------------------------------------------------------- dispatch
 size_t PassKernel::smem_bytes(uint32_t N, uint32_t delta_row) const {
-  size_t w = (size_t)words * (N + 1);
-  if (wb_array) w += N;
+  size_t w = (size_t)words * (N + 1);  // (float write-back values overlay the first sum word)
   if (monotone) w += (N + 31) / 32;
   return ring_bytes + 4 * (w + delta_row);
 }
