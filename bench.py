@@ -108,11 +108,14 @@ def load_graph(name, cache):
     return wl
 
 
-def traffic_for(workload):
+def traffic_for(workload, overlapped):
+    """DRAM bytes (read + write) of one shard_pass launch from the committed ncu
+    capture (profiles/traffic.json), for the launch shape this run used."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(p):
         with open(p) as f:
-            return json.load(f).get(workload)
+            t = json.load(f)
+        return t.get(f"{workload}:{'run' if overlapped else 'pass'}")
     return None
 
 
@@ -290,6 +293,8 @@ def bench_cusha(args):
     # (overlapped passes, device_loop 2) or one per iteration (+ one refresh when partitioned)
     launches = sum(3 + (1 if s[6] == 2 else s[1] * (2 if world > 1 else 1)) for s in steps)
     launches = int(sum_over_ranks(launches))
+    overlapped = steps[-1][6] == 2
+    n_pass_launches = len(steps) if overlapped else sum(iters)
     peak, peak_kind = measured_peak_gbs()
     achieved = alg_bytes / (loop_ms / 1e3) / 1e9
     st = cusha.get_stats(g)
@@ -357,10 +362,15 @@ def bench_cusha(args):
                    else "overlapped passes in one launch (DESIGN.md \"Overlapped passes\")",
                    "parallelism": f"destination-range partition x{world} (NCCL)" if world > 1 else "1 GPU"},
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                     "frac": round(achieved / peak, 4), "traffic": traffic_for(args.workload) if world == 1 else None,
+                     "frac": round(achieved / peak, 4),
+                     "traffic": traffic_for(args.workload, overlapped) if world == 1 else None,
+                     "launch": "one shard_pass launch per run (overlapped passes)" if overlapped
+                     else "one shard_pass launch per pass",
+                     "passes_per_step": round(sum(iters) / len(iters), 2),
+                     "avg_pass_us": round(loop_ms / max(sum(iters), 1) * 1e3, 3),
                      "kernel": f"shard_pass<{alg},{repr_}>", "peak_kind": peak_kind,
-                     "algorithmic_bytes_per_launch": int(alg_bytes / max(sum(iters), 1)),
-                     "avg_launch_us": round(loop_ms / max(sum(iters), 1) * 1e3, 3)},
+                     "algorithmic_bytes_per_launch": int(alg_bytes / max(n_pass_launches, 1)),
+                     "avg_launch_us": round(loop_ms / max(n_pass_launches, 1) * 1e3, 3)},
         "clocks": clocks,
         "gpu_launches": launches,
         "e2e": e2e,
