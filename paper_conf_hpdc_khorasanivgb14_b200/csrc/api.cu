@@ -391,7 +391,9 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     g.d_trace = nullptr;
     g.trace_cap = 0;
     CKA(cudaMallocAsync(&g.d_trace, sizeof(TraceRec) * (size_t)want_cap, g.stream));
+    CKA(cudaMemsetAsync(g.d_trace, 0, sizeof(TraceRec) * (size_t)want_cap, g.stream));
     g.trace_cap = want_cap;
+    g.trace_dirty = 0;
     for (auto& e : h->exec)  // kernel params captured the old trace pointer
       if (e) { cudaGraphExecDestroy(e); e = nullptr; }
   }
@@ -408,7 +410,9 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     rc = ensure_exec(h, a);
     if (rc) return rc;
   }
-  CKA(cudaMemsetAsync(g.d_trace, 0, sizeof(TraceRec) * (size_t)g.trace_cap, g.stream));
+  // records a previous run may have written (the rest are still zero)
+  if (g.trace_dirty) CKA(cudaMemsetAsync(g.d_trace, 0, sizeof(TraceRec) * (size_t)g.trace_dirty, g.stream));
+  g.trace_dirty = g.trace_cap;  // until this run's extent is known
   CKA(cudaEventRecord(g.ev0, g.stream));
   CKA(launch_reset_ctl(g.d_ctl, max_iters, g.stream));
   CKA(launch_init(g, a, source, g.stream));
@@ -456,6 +460,10 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   cudaEventElapsedTime(&ms, g.ev0, g.ev1);
   cudaEventElapsedTime(&lms, g.evm, g.ev1);
   Ctl c = *g.h_ctl;
+  {  // passes whose trace records this run touched: its iterations, or every drawn ticket's pass
+    const uint64_t drawn = multi && g.S ? c.ticket / g.S + 1 : 0;
+    g.trace_dirty = (uint32_t)std::min<uint64_t>(g.trace_cap, std::max<uint64_t>(c.iter, drawn) + 2);
+  }
   if (multi && max_iters > 0) {  // the confirming pass that committed nothing, else max_iters passes ran
     c.converged = c.conv_iter != 0xFFFFFFFFu;
     c.iter = c.converged ? c.conv_iter : max_iters;

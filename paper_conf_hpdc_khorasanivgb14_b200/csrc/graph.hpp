@@ -167,6 +167,7 @@ struct Graph {
   Ctl* d_ctl = nullptr;
   TraceRec* d_trace = nullptr;
   uint32_t trace_cap = 0;
+  uint32_t trace_dirty = 0;         // leading trace records a previous run may have written
   Ctl* h_ctl = nullptr;             // host mirror
   cudaEvent_t ev0 = nullptr, ev1 = nullptr, evm = nullptr;
   // destination-range partition (row e)

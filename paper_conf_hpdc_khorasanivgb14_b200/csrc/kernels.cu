@@ -829,27 +829,34 @@ __global__ void init_vertex_values(const KParams p, const void* user) {
 }
 
 // SrcValue[e] <- VertexValues[SrcIndex[e]] for every entry (R20: a full
-// write-back at t = 0), one CTA per source shard i.
+// write-back at t = 0), one CTA per source shard i.  Every source of shard i's
+// windows lies in shard i, so the CTA first stages the write-back values of
+// its |N| vertices in shared memory (coalesced) and then streams its windows
+// (G-Shards) or CW_i (CW) against them, as stage 4 of a pass does.
 template <class A>
-__global__ void init_srcvalue_gs(const KParams p) {
+__device__ __forceinline__ void stage_wb_values(const KParams& p, uint32_t i, uint32_t* wb) {
   using V_t = typename A::Value;
   const V_t* vv = reinterpret_cast<const V_t*>(p.vv);
-  const uint32_t i = blockIdx.x, lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
-  gs_walk(p, i, lane, warp, blockDim.x / 32, [&](uint32_t e, uint32_t l) {
-    const uint32_t u = i * p.N + l;
-    p.srcvalue[e] = A::wb_value(vv[u], A::kOutDeg ? p.outdeg[u] : 0u);
-  });
+  const uint32_t off = i * p.N, nv = min(p.N, p.V - off);
+  for (uint32_t v = threadIdx.x; v < nv; v += blockDim.x)
+    wb[v] = A::wb_value(vv[off + v], A::kOutDeg ? __ldg(p.outdeg + off + v) : 0u);
+  __syncthreads();
 }
 template <class A>
-__global__ void init_srcvalue_cw(const KParams p) {
-  using V_t = typename A::Value;
-  const V_t* vv = reinterpret_cast<const V_t*>(p.vv);
+__global__ void __launch_bounds__(512) init_srcvalue_gs(const KParams p) {
+  extern __shared__ uint32_t wb[];
+  const uint32_t i = blockIdx.x, lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+  stage_wb_values<A>(p, i, wb);
+  gs_walk(p, i, lane, warp, blockDim.x / 32, [&](uint32_t e, uint32_t l) { p.srcvalue[e] = wb[l]; });
+}
+template <class A>
+__global__ void __launch_bounds__(512) init_srcvalue_cw(const KParams p) {
+  extern __shared__ uint32_t wb[];
   const uint32_t i = blockIdx.x, trash = p.shard_off[p.S];
+  stage_wb_values<A>(p, i, wb);
   for (uint32_t k = p.cw_off[i] + threadIdx.x; k < p.cw_off[i + 1]; k += blockDim.x) {
-    const uint32_t m = *topo_at(p.mapper, p.mapper_h, p.splitQ, k);
-    if (m == trash) continue;
-    const uint32_t u = i * p.N + *topo_at(p.cw_src, p.cw_src_h, p.splitQ, k);
-    p.srcvalue[m] = A::wb_value(vv[u], A::kOutDeg ? p.outdeg[u] : 0u);
+    const uint32_t m = __ldg(topo_at(p.mapper, p.mapper_h, p.splitQ, k));
+    if (m != trash) p.srcvalue[m] = wb[__ldg(topo_at(p.cw_src, p.cw_src_h, p.splitQ, k))];
   }
 }
 
@@ -931,8 +938,12 @@ static cudaError_t launch_init_t(const Graph& g, uint32_t source, cudaStream_t s
   const uint32_t vb = (uint32_t)((g.V + 255) / 256);
   init_vertex_values<A><<<vb < 148 * 16 ? vb : 148 * 16, 256, 0, s>>>(p, g.d_init[A::kId]);
   if (g.S) {
-    if (g.repr == CUSHA_REPR_CW) init_srcvalue_cw<A><<<g.S, 256, 0, s>>>(p);
-    else init_srcvalue_gs<A><<<g.S, 256, 0, s>>>(p);
+    const size_t sm = 4ull * g.N;  // the shard's write-back values (|N| <= 65534: at most 256 KB)
+    const void* fn = g.repr == CUSHA_REPR_CW ? (const void*)&init_srcvalue_cw<A> : (const void*)&init_srcvalue_gs<A>;
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e != cudaSuccess) return e;  // |N| beyond the shared-memory limit cannot run the pass either
+    if (g.repr == CUSHA_REPR_CW) init_srcvalue_cw<A><<<g.S, 512, sm, s>>>(p);
+    else init_srcvalue_gs<A><<<g.S, 512, sm, s>>>(p);
   }
   return cudaGetLastError();
 }
