@@ -108,15 +108,19 @@ def load_graph(name, cache):
     return wl
 
 
-def traffic_for(workload, overlapped):
+def traffic_for(workload, overlapped, passes):
     """DRAM bytes (read + write) of one shard_pass launch from the committed ncu
-    capture (profiles/traffic.json), for the launch shape this run used."""
+    --set full capture (profiles/traffic.json), for the launch shape this run
+    used.  A captured whole-run launch is scaled by passes (this launch's over
+    the captured one's): the pass count of a PR run varies by a few between runs."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(p):
-        with open(p) as f:
-            t = json.load(f)
-        return t.get(f"{workload}:{'run' if overlapped else 'pass'}")
-    return None
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        t = json.load(f).get(f"{workload}:{'run' if overlapped else 'pass'}")
+    if not t:
+        return None
+    return int(t["bytes"] * (passes / t["passes"] if overlapped else 1))
 
 
 def cpu_baseline(wl, alg, source, budget_s=15.0):
@@ -363,7 +367,7 @@ def bench_cusha(args):
                    "parallelism": f"destination-range partition x{world} (NCCL)" if world > 1 else "1 GPU"},
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                      "frac": round(achieved / peak, 4),
-                     "traffic": traffic_for(args.workload, overlapped) if world == 1 else None,
+                     "traffic": traffic_for(args.workload, overlapped, sum(iters) / len(iters)) if world == 1 else None,
                      "launch": "one shard_pass launch per run (overlapped passes)" if overlapped
                      else "one shard_pass launch per pass",
                      "passes_per_step": round(sum(iters) / len(iters), 2),
