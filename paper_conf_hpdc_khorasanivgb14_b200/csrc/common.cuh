@@ -63,6 +63,14 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
                : "memory");
 }
 
+// TMA bulk prefetch of [src, src + bytes) into L2 (no shared memory, no
+// completion to wait for); the range is widened to 16-byte bounds
+__device__ __forceinline__ void bulk_prefetch_l2(const void* src, uint32_t bytes) {
+  const uintptr_t a = reinterpret_cast<uintptr_t>(src) & ~uintptr_t(15);
+  const uint32_t n = (uint32_t)(((reinterpret_cast<uintptr_t>(src) + bytes + 15) & ~uintptr_t(15)) - a);
+  if (n) asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"(n) : "memory");
+}
+
 // L2 policy for streams read once per pass (topology arrays): evict first, so
 // that SrcValue lines written by stage 4 stay in L2 until stage 2 reads them
 __device__ __forceinline__ uint64_t l2_evict_first_policy() {

@@ -65,7 +65,14 @@ constexpr uint32_t kVB = CUSHA_VB;                   // vertex loads in flight p
 #ifndef CUSHA_EPT
 #define CUSHA_EPT 4
 #endif
-constexpr uint32_t kEPT = CUSHA_EPT;  // stage-2 entries per consumer thread per step (4 or 8)
+constexpr uint32_t kEPT = CUSHA_EPT;
+#ifndef CUSHA_PF
+#define CUSHA_PF 0  // 1: producer prefetches a shard's stage-1/3 vertex data and delta row into L2
+#endif
+#ifndef CUSHA_S4U
+#define CUSHA_S4U 1
+#endif
+constexpr uint32_t kS4U = CUSHA_S4U;  // stage-4 entries per consumer thread per step (loads before stores)  // stage-2 entries per consumer thread per step (4 or 8)
 constexpr uint32_t kConsumerWarps = CUSHA_CONSUMER_WARPS;
 constexpr uint32_t kConsumers = kConsumerWarps * 32;
 constexpr uint32_t kPassThreads = kConsumers + 32;  // + 1 producer warp
@@ -395,6 +402,14 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     }
     const bool spec = CUSHA_SPEC && REPR == CUSHA_REPR_CW && (CUSHA_SPEC_ALWAYS || p.active[s]);
     const uint32_t b = p.shard_off[s], e = p.shard_off[s + 1];
+    if (CUSHA_PF) {
+      // the consumers' global reads of this shard (stage 1/3 VertexValues and
+      // NbrsNum, the stage-4 delta row) become L2 hits: one TMA prefetch each
+      const uint32_t off = s * p.N, nv = min(p.N, p.V - off);
+      bulk_prefetch_l2(reinterpret_cast<const typename A::Value*>(p.vv) + off, nv * (uint32_t)sizeof(typename A::Value));
+      if (A::kOutDeg) bulk_prefetch_l2(p.outdeg + off, nv * 4);
+      if (REPR == CUSHA_REPR_CW && p.mapj) bulk_prefetch_l2(p.cw_delta + (size_t)s * p.S, p.S * 4);
+    }
     // CW_s entries whose targets lie in the shard's own partition: all of CW_s
     // on one GPU; with G partitions the other windows are refreshed after the
     // exchange.  Stage-4 tiles are 8-entry aligned for TMA.
@@ -664,31 +679,46 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
                 }
               }
             } else if (any && p.mapj) {
-              // SrcValue[delta_row[j] + k] = local[SrcIndexCW[k]] for CW position k = base + i
+              // SrcValue[delta_row[j] + k] = local[SrcIndexCW[k]] for CW position k = base + i;
+              // kS4U entries per thread: every shared load of a step before its stores
               const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
               const uint16_t* J = reinterpret_cast<const uint16_t*>(ring + slot * SLOT + 2 * tile4j_of<A>());
-              for (uint32_t i = d.lo + ct; i < d.hi; i += kConsumers) {
-                const uint32_t j = J[i];
-                uint32_t val;
-                if (j != 0xFFFFu && wb_get<A>(sm, aux, L[i], val)) {
-                  st_u32(p.srcvalue + (drow[j] + d.base + i), val);
-                  ++stores;
+              for (uint32_t i0 = d.lo + ct; i0 < d.hi; i0 += kS4U * kConsumers) {
+                uint32_t tg[kS4U], val[kS4U];
+                bool ok[kS4U];
+#pragma unroll
+                for (uint32_t u = 0; u < kS4U; ++u) {
+                  const uint32_t i = i0 + u * kConsumers;
+                  const uint32_t j = i < d.hi ? (uint32_t)J[i] : 0xFFFFu;
+                  ok[u] = j != 0xFFFFu && wb_get<A>(sm, aux, L[i], val[u]);
+                  tg[u] = (ok[u] ? drow[j] : 0u) + d.base + i;
                 }
+#pragma unroll
+                for (uint32_t u = 0; u < kS4U; ++u)
+                  if (ok[u]) { st_u32(p.srcvalue + tg[u], val[u]); ++stores; }
               }
             } else if (any) {
               const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
               const uint32_t* M = reinterpret_cast<const uint32_t*>(ring + slot * SLOT + 2 * tile4m_of<A>());
-              for (uint32_t i = d.lo + ct; i < d.hi; i += kConsumers) {
-                const uint32_t m = M[i];
-                uint32_t val;
-                if (m != trash && wb_get<A>(sm, aux, L[i], val)) {
-                  if (kDiag & 4) {
-                    if (val == 0x9e3779b9u && m == 7u) st_u32(p.srcvalue + m, val);  // keep the loads
-                  } else {
-                    st_u32(p.srcvalue + m, val);
-                  }
-                  ++stores;
+              for (uint32_t i0 = d.lo + ct; i0 < d.hi; i0 += kS4U * kConsumers) {
+                uint32_t tg[kS4U], val[kS4U];
+                bool ok[kS4U];
+#pragma unroll
+                for (uint32_t u = 0; u < kS4U; ++u) {
+                  const uint32_t i = i0 + u * kConsumers;
+                  tg[u] = i < d.hi ? M[i] : trash;
+                  ok[u] = tg[u] != trash && wb_get<A>(sm, aux, L[i], val[u]);
                 }
+#pragma unroll
+                for (uint32_t u = 0; u < kS4U; ++u)
+                  if (ok[u]) {
+                    if (kDiag & 4) {
+                      if (val[u] == 0x9e3779b9u && tg[u] == 7u) st_u32(p.srcvalue + tg[u], val[u]);  // keep the loads
+                    } else {
+                      st_u32(p.srcvalue + tg[u], val[u]);
+                    }
+                    ++stores;
+                  }
               }
             }
             __syncwarp();
