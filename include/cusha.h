@@ -266,6 +266,14 @@ typedef enum {
  * Parts not held by the representation return CUSHA_EUNSUPPORTED.          */
 CUSHA_API int cusha_get_layout(const cusha_graph* g, cusha_layout_part part, void* out, size_t out_bytes, uint64_t* count);
 
+/* Diagnostic timeline (tools/timeline.py): only a library built with
+ * -DCUSHA_TIMELINE=1 records it; the product build returns CUSHA_EUNSUPPORTED.
+ * Copies up to out_bytes of the per-ticket %globaltimer stamps of the last
+ * overlapped-pass run into `out` (host): 10 u32 words per ticket
+ * (ticket = pass * |S| + shard; word meaning in csrc/kernels.cu, kTlSlots).
+ * Returns the number of tickets copied (>= 0) or a negative error code.    */
+CUSHA_API int cusha_diag_timeline(void* out, size_t out_bytes);
+
 /* ---------------------------------------------------------- host logic */
 /*
  * The shard-size rule of L310 (§4 "Selecting shard size"), pure host code:

@@ -618,4 +618,11 @@ int cusha_get_partition(const cusha_graph* h, uint32_t* bounds, uint32_t cap) {
   return (int)g.G;
 }
 
+int cusha_diag_timeline(void* out, size_t out_bytes) {
+  if (!out) return fail(CUSHA_EINVAL, "null argument");
+  cudaDeviceSynchronize();
+  const int n = timeline_copy(out, out_bytes);
+  return n < 0 ? fail(CUSHA_EUNSUPPORTED, "library built without CUSHA_TIMELINE") : n;
+}
+
 }  // extern "C"

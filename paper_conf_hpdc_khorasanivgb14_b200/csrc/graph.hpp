@@ -194,6 +194,7 @@ cudaError_t launch_reset_ctl(Ctl* ctl, uint32_t max_iters, cudaStream_t s);
 cudaError_t launch_refresh(const Graph& g, cudaStream_t s);
 KParams make_params(const Graph& g, uint32_t source);
 size_t value_bytes(int alg);
+int timeline_copy(void* out, size_t bytes);  // CUSHA_TIMELINE builds: per-ticket stamps (else -1)
 bool kernels_rle();  // built with the Mapper-runs stage 4 (CUSHA_RLE)
 
 bool alg_needs_edge_values(int alg);

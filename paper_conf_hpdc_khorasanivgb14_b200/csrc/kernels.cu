@@ -67,7 +67,7 @@ constexpr uint32_t kVB = CUSHA_VB;                   // vertex loads in flight p
 #endif
 constexpr uint32_t kEPT = CUSHA_EPT;
 #ifndef CUSHA_PF
-#define CUSHA_PF 0  // 1: producer prefetches a shard's stage-1/3 vertex data and delta row into L2
+#define CUSHA_PF 0  // L2 prefetch of a shard's stage-3 vertex data (and delta row): 1 by the producer at ticket draw, 2 by a consumer at stage-2 start
 #endif
 #ifndef CUSHA_S4U
 #define CUSHA_S4U 1
@@ -75,7 +75,20 @@ constexpr uint32_t kEPT = CUSHA_EPT;
 constexpr uint32_t kS4U = CUSHA_S4U;  // stage-4 entries per consumer thread per step (loads before stores)  // stage-2 entries per consumer thread per step (4 or 8)
 constexpr uint32_t kConsumerWarps = CUSHA_CONSUMER_WARPS;
 constexpr uint32_t kConsumers = kConsumerWarps * 32;
-constexpr uint32_t kPassThreads = kConsumers + 32;  // + 1 producer warp
+#ifndef CUSHA_BK
+#define CUSHA_BK 1
+#endif
+// 1: a bookkeeper warp does each shard's end-of-ticket bookkeeping (trace
+// counters, predictor, convergence flag, ticket_done's fence and atomics) so
+// that the consumer warps go straight on with the next shard
+constexpr bool kBk = CUSHA_BK != 0;
+constexpr uint32_t kPassThreads = kConsumers + 32 + (kBk ? 32 : 0);  // + 1 producer warp (+ 1 bookkeeper warp)
+constexpr uint32_t kBkWarp = kConsumerWarps + 1;
+// one finished ticket, handed from the consumers to the bookkeeper warp
+struct BkRec {
+  uint32_t s, it, any, upd;
+  unsigned long long stores;
+};
 // entries per ring slot
 template <class A>
 constexpr uint32_t tile_of() {
@@ -125,8 +138,27 @@ constexpr uint32_t tile4m_of() {
 // Diagnostic variants for the per-stage cost split (tools/diag_pass.py; never
 // the product, results are wrong by design): bit 0 = every shard active in
 // every pass (no convergence), bit 1 = no stage-2 reduction, bit 2 = no
-// stage-4 stores.
+// stage-4 stores, bit 3 = no per-pass trace counters (stats only).
 constexpr uint32_t kDiag = CUSHA_DIAG;
+#ifndef CUSHA_TIMELINE
+#define CUSHA_TIMELINE 0
+#endif
+// Diagnostic timeline (tools/timeline.py; never the product): %globaltimer
+// stamps of each ticket's steps, kTlSlots words per ticket, ticket = pass * |S|
+// + shard.  0 producer drew it, 1 producer passed ticket_wait, 2 consumers got
+// its first tile, 3 stage 1 done, 4 stage 2 done, 5 stage 3 done, 6 stage 4
+// done, 7 ticket completed, 8 CTA index, 9 stage-4 tiles were prefetched.
+constexpr uint32_t kTlSlots = 10, kTlCap = 1u << 18;
+#if CUSHA_TIMELINE
+__device__ uint32_t g_timeline[kTlCap * kTlSlots];
+__device__ __forceinline__ void tl_mark(uint32_t ticket, uint32_t k, uint32_t v = 0xFFFFFFFFu) {
+  if (ticket >= kTlCap) return;
+  if (v == 0xFFFFFFFFu) asm volatile("mov.u32 %0, %%globaltimer_lo;" : "=r"(v));
+  g_timeline[ticket * kTlSlots + k] = v;
+}
+#else
+__device__ __forceinline__ void tl_mark(uint32_t, uint32_t, uint32_t = 0) {}
+#endif
 
 // stage-4 tile kinds: kDescStage4 carries SrcIndexCW + Mapper per entry;
 // kDescStage4R carries SrcIndexCW + the Mapper runs overlapping the tile.
@@ -372,12 +404,14 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
         cur_pass = (uint32_t)(t / Sloc);
         s = q_lo + (uint32_t)(t - (unsigned long long)cur_pass * Sloc);
         over = cur_pass >= p.ctl->max_iters || ld_vol(&p.ctl->stop) != 0;
+        if (CUSHA_TIMELINE && !over) tl_mark((uint32_t)t, 0);
       }
       if (over) {
         push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
         return;
       }
       ticket_wait(p, s, cur_pass, Sloc);
+      if (CUSHA_TIMELINE) tl_mark(cur_pass * Sloc + (s - q_lo), 1);
     } else {
       // persistent grid: shards from the global queue; otherwise CTA b runs shard q_lo + b only
       s = q_lo + (kPersistent ? atomicAdd(&p.ctl->next_shard, 1u) : (round == 0 ? blockIdx.x : q_hi));
@@ -402,7 +436,7 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     }
     const bool spec = CUSHA_SPEC && REPR == CUSHA_REPR_CW && (CUSHA_SPEC_ALWAYS || p.active[s]);
     const uint32_t b = p.shard_off[s], e = p.shard_off[s + 1];
-    if (CUSHA_PF) {
+    if (CUSHA_PF == 1) {
       // the consumers' global reads of this shard (stage 1/3 VertexValues and
       // NbrsNum, the stage-4 delta row) become L2 hits: one TMA prefetch each
       const uint32_t off = s * p.N, nv = min(p.N, p.V - off);
@@ -474,6 +508,32 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
   }
 }
 
+// end-of-ticket bookkeeping of shard s in pass it: trace counters, the
+// stage-4 predictor, the paper's is_converged = false (line 26), and - with
+// overlapped passes - the ticket's completion (ticket_done)
+__device__ __forceinline__ void ticket_bookkeeping(const KParams& p, uint32_t s, uint32_t it, bool any, uint32_t upd,
+                                                   unsigned long long stores, uint32_t Sloc) {
+  if (it < p.trace_cap && !(kDiag & 8)) {
+    atomicAdd(&p.trace[it].edges, (unsigned long long)p.shard_cnt[s]);
+    atomicAdd(&p.trace[it].shards, 1ull);
+  }
+  p.active[s] = any ? 1 : 0;
+  if (any) {
+    *reinterpret_cast<volatile uint32_t*>(&p.ctl->changed) = 1u;
+    if (it < p.trace_cap) {
+      TraceRec* t = p.trace + it;
+      atomicAdd(&t->active_shards, 1u);  // read by the convergence test (ticket_done)
+      if (!(kDiag & 8)) {
+        atomicAdd(&t->updated, upd);
+        atomicAdd(&t->wb_entries, (unsigned long long)p.cw_cnt[s]);
+        atomicAdd(&t->wb_stores, stores);
+      }
+    }
+  }
+  // overlapped passes: every consumer's stores precede this (barriers; fences are cumulative)
+  if (p.multi) ticket_done(p, s, it, Sloc);
+}
+
 template <class A, int REPR>
 __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(const KParams p) {
   extern __shared__ __align__(128) uint8_t dyn[];
@@ -486,6 +546,8 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
   __shared__ uint32_t s_upd;
   __shared__ int s_any;
   __shared__ unsigned long long s_stores;
+  __shared__ uint64_t bk_full[2], bk_empty[2];
+  __shared__ BkRec bk[2];
   using V_t = typename A::Value;
   const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
   const uint32_t N = p.N, st = N + 1;
@@ -506,15 +568,20 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
       mbar_init(&empty_bar[i], kConsumerWarps);  // one arrive per consumer warp
     }
     mbar_init(&decide_bar, 1);  // stage-3 decision of a non-prefetched CW shard
+    for (uint32_t i = 0; i < 2; ++i) {
+      mbar_init(&bk_full[i], 1);   // the consumers' hand-over of a finished ticket
+      mbar_init(&bk_empty[i], 1);  // the bookkeeper is done with it
+    }
     mbar_fence_init();
   }
   __syncthreads();
 
   if (warp == 0) {
     if (lane == 0) producer<A, REPR>(p, ring, desc, full_bar, empty_bar, &decide_bar, &s_any);
-  } else {
+  } else if (warp <= kConsumerWarps) {
     const uint32_t ct = tid - 32, cwarp = warp - 1;  // consumer thread / warp index
     uint32_t slot = 0, ph = 0;
+    uint32_t ntk = 0;  // tickets handed to the bookkeeper (kBk)
     for (;;) {
       mbar_wait(&full_bar[slot], ph);
       TileDesc d = desc[slot];
@@ -525,6 +592,8 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
       const uint32_t off = s * N;
       const uint32_t nv = min(N, p.V - off);
       V_t* vv = reinterpret_cast<V_t*>(p.vv) + off;
+      const uint32_t tk = it * Sloc + (s - (p.part >= 0 ? p.bounds[p.part] : 0u));  // timeline ticket
+      if (CUSHA_TIMELINE && ct == 0) { tl_mark(tk, 2); tl_mark(tk, 8, blockIdx.x); tl_mark(tk, 9, spec4 ? 1u : 0u); }
 
       // ---- stage 1: local_vertices <- init_compute(VertexValues) (Fig. 5 lines 8-10, L267)
       // (kVB loads in flight per thread before any is used)
@@ -552,8 +621,13 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
         s_stores = 0;
       }
       bar_sync(kConsumerBar, kConsumers);
+      if (CUSHA_TIMELINE && ct == 0) tl_mark(tk, 3);
 
       // ---- stage 2: the shard's entries from the ring, compute() into shared memory (lines 12-13, L269)
+      if (CUSHA_PF == 2 && ct == 0) {
+        bulk_prefetch_l2(vv, nv * (uint32_t)sizeof(V_t));
+        if (A::kOutDeg) bulk_prefetch_l2(p.outdeg + off, nv * 4);
+      }
       for (;;) {
         const uint8_t* buf = ring + slot * SLOT;
         if (kEPT == 8) {
@@ -588,6 +662,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
         d = desc[slot];
       }
       bar_sync(kConsumerBar, kConsumers);
+      if (CUSHA_TIMELINE && ct == 0) tl_mark(tk, 4);
 
       // ---- stage 3: update_condition, commit to VertexValues, values_updated (lines 15-20, L271)
       uint32_t my_upd = 0;
@@ -624,6 +699,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
         }
       }
       const int any = bar_sync_or(kConsumerBar, kConsumers, (int)my_upd) | ((kDiag & 1) ? 1 : 0);
+      if (CUSHA_TIMELINE && ct == 0) tl_mark(tk, 5);
 
       // ---- stage 4: write-back into every shard's window (lines 23-26, L308)
       uint32_t stores = 0;
@@ -740,6 +816,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
       if (lane == 0 && stores) atomicAdd(&s_stores, (unsigned long long)stores);
       if (p.skip && any) __threadfence();  // release: SrcValue stores before the dirty marks below
       bar_sync(kConsumerBar, kConsumers);
+      if (CUSHA_TIMELINE && ct == 0) tl_mark(tk, 6);
 
       if (p.skip && any) {
         // mark every shard j fed by a non-empty window W_sj (own partition; the
@@ -755,23 +832,37 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
 
       // ---- per-shard bookkeeping: convergence flag (line 26), predictor, trace
       if (ct == 0) {
-        if (it < p.trace_cap) {
-          atomicAdd(&p.trace[it].edges, (unsigned long long)p.shard_cnt[s]);
-          atomicAdd(&p.trace[it].shards, 1ull);
+        if (kBk) {
+          // hand the ticket to the bookkeeper warp (every consumer's stores precede
+          // this through the barrier above; the bookkeeper's fence is cumulative)
+          const uint32_t b = ntk & 1u;
+          mbar_wait(&bk_empty[b], ((ntk >> 1) & 1u) ^ 1u);
+          bk[b] = BkRec{s, it, (uint32_t)any, s_upd, s_stores};
+          mbar_arrive(&bk_full[b]);
+          ++ntk;
+        } else {
+          ticket_bookkeeping(p, s, it, any != 0, s_upd, s_stores, Sloc);
+          if (CUSHA_TIMELINE) tl_mark(tk, 7);
         }
-        p.active[s] = any ? 1 : 0;
-        if (any) {
-          *reinterpret_cast<volatile uint32_t*>(&p.ctl->changed) = 1u;
-          if (it < p.trace_cap) {
-            TraceRec* t = p.trace + it;
-            atomicAdd(&t->updated, s_upd);
-            atomicAdd(&t->active_shards, 1u);
-            atomicAdd(&t->wb_entries, (unsigned long long)p.cw_cnt[s]);
-            atomicAdd(&t->wb_stores, s_stores);
-          }
-        }
-        // overlapped passes: every consumer's stores precede this (barrier above; fences are cumulative)
-        if (p.multi) ticket_done(p, s, it, Sloc);
+      }
+    }
+    if (kBk && ct == 0) {  // no more tickets: release the bookkeeper
+      const uint32_t b = ntk & 1u;
+      mbar_wait(&bk_empty[b], ((ntk >> 1) & 1u) ^ 1u);
+      bk[b].s = 0xFFFFFFFFu;
+      mbar_arrive(&bk_full[b]);
+    }
+  } else {
+    // bookkeeper warp (kBk): the end-of-ticket bookkeeping, in ticket order
+    if (lane == 0) {
+      for (uint32_t n = 0;; ++n) {
+        const uint32_t b = n & 1u;
+        mbar_wait(&bk_full[b], (n >> 1) & 1u);
+        const BkRec r = bk[b];
+        if (r.s == 0xFFFFFFFFu) break;
+        ticket_bookkeeping(p, r.s, r.it, r.any != 0, r.upd, r.stores, Sloc);
+        if (CUSHA_TIMELINE) tl_mark(r.it * Sloc + (r.s - (p.part >= 0 ? p.bounds[p.part] : 0u)), 7);
+        mbar_arrive(&bk_empty[b]);
       }
     }
   }
@@ -936,6 +1027,17 @@ const PassKernel& pass_kernel(int alg, int repr) {
 
 
 bool kernels_rle() { return kRle; }
+
+// diagnostic timeline builds only: copy the stamps out (tools/timeline.py)
+int timeline_copy(void* out, size_t bytes) {
+#if CUSHA_TIMELINE
+  const size_t n = bytes < sizeof(g_timeline) ? bytes : sizeof(g_timeline);
+  return cudaMemcpyFromSymbol(out, g_timeline, n) == cudaSuccess ? (int)(n / (4 * kTlSlots)) : -1;
+#else
+  (void)out; (void)bytes;
+  return -1;
+#endif
+}
 
 size_t value_bytes(int alg) { return (alg == kHS || alg == kCS) ? 8 : 4; }
 bool alg_needs_edge_values(int alg) { return alg == kSSSP || alg == kSSWP || alg == kNN || alg == kHS || alg == kCS; }

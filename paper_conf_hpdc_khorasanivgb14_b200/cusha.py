@@ -112,6 +112,7 @@ def lib():
             "cusha_nccl_unique_id": (i32, [P]),
             "cusha_partition_shards": (i32, [u32, P, u32, P]),
             "cusha_get_partition": (i32, [P, P, u32]),
+            "cusha_diag_timeline": (i32, [P, sz]),
         }
         for name, (res, args) in sigs.items():
             f = getattr(L, name)
