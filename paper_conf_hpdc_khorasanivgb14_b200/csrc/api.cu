@@ -310,7 +310,10 @@ static uint32_t pass_grid(const Graph& g, const PassKernel& pk, size_t smem) {
 #ifndef CUSHA_MAPJ
 #define CUSHA_MAPJ 1  // 0: always the u32 Mapper (tuning comparison)
 #endif
-static int pass_config(const Graph& g, const PassKernel& pk, size_t* smem, int* mapj) {
+#ifndef CUSHA_STASH
+#define CUSHA_STASH 1  // 0: stage 3 of the integer algorithms re-reads VertexValues (tuning comparison)
+#endif
+static int pass_config(const Graph& g, const PassKernel& pk, size_t* smem, int* mapj, int* stash) {
   cudaFuncAttributes fa{};
   CKA(cudaFuncGetAttributes(&fa, pk.func));
   const size_t kMaxSmem = 227 * 1024 - fa.sharedSizeBytes;  // dynamic part of the 227 KB per-CTA limit
@@ -331,6 +334,20 @@ static int pass_config(const Graph& g, const PassKernel& pk, size_t* smem, int* 
       *mapj = 1;
     }
   }
+  // integer algorithms: keep the shard's VertexValues from stage 1 in shared
+  // memory for stage 3's update_condition (no second global read) whenever
+  // that costs no CTAs per SM
+  *stash = 0;
+  const size_t sm_s = *smem + 4ull * g.N;
+  if (CUSHA_STASH && pk.monotone && sm_s <= kMaxSmem) {
+    int occ_0 = 0, occ_s = 0;
+    CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_0, pk.func, (int)pk.threads, *smem));
+    CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_s, pk.func, (int)pk.threads, sm_s));
+    if (occ_s >= occ_0 && occ_s > 0) {
+      *smem = sm_s;
+      *stash = 1;
+    }
+  }
   return CUSHA_OK;
 }
 
@@ -339,8 +356,8 @@ static int ensure_exec(cusha_graph* h, int alg) {
   if (h->exec[alg]) return CUSHA_OK;
   const PassKernel& pk = pass_kernel(alg, g.repr);
   size_t smem = 0;
-  int mapj = 0;
-  const int prc = pass_config(g, pk, &smem, &mapj);
+  int mapj = 0, stash = 0;
+  const int prc = pass_config(g, pk, &smem, &mapj, &stash);
   if (prc) return prc;
   cudaGraph_t graph = nullptr;
   CKA(cudaGraphCreate(&graph, 0));
@@ -359,6 +376,7 @@ static int ensure_exec(cusha_graph* h, int alg) {
   KParams kp = make_params(g, 0);
   kp.use_cond = 1;
   kp.mapj = mapj;
+    kp.stash = stash;
   kp.cond_handle = handle;
   void* args[] = {&kp};
   cudaKernelNodeParams knp = {};
@@ -399,8 +417,8 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   }
   const PassKernel& pk = pass_kernel(a, g.repr);
   size_t smem = 0;
-  int mapj = 0;
-  int rc = pass_config(g, pk, &smem, &mapj);
+  int mapj = 0, stash = 0;
+  int rc = pass_config(g, pk, &smem, &mapj, &stash);
   if (rc) return rc;
   const bool host_loop = g.host_loop || g.G > 1;  // the partitioned mode exchanges between passes
   // overlapped passes (default): one launch runs every pass; it needs a trace
@@ -421,6 +439,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     KParams kp = make_params(g, source);
     kp.multi = 1;
     kp.mapj = mapj;
+    kp.stash = stash;
     void* args[] = {&kp};
     CKA(cudaLaunchKernel(pk.func, dim3(pass_grid(g, pk, smem)), dim3(pk.threads), args, smem, g.stream));
   } else if (max_iters > 0 && !host_loop) {
@@ -434,6 +453,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     // from the same exchanged data, so all issue the same collectives.
     KParams kp = make_params(g, source);
     kp.mapj = mapj;
+    kp.stash = stash;
     void* args[] = {&kp};
     const dim3 grid(pass_grid(g, pk, smem));
     const int chunk = g.G > 1 && !g.simulate ? 1 : 8;

@@ -66,6 +66,7 @@ struct KParams {
   unsigned long long cond_handle;
   int multi;                   // 1: one launch runs every pass (overlapped passes)
   int mapj;                    // 1: CW stage 4 uses the Mapper in window form (cw_win + delta row in smem)
+  int stash;                   // 1: integer algorithms keep stage 1's VertexValues in smem for stage 3
   uint32_t* shard_seq;         // S: passes of shard s completed (overlapped passes)
   // destination-range partition (row e); G = 1: single partition
   uint32_t G;                  // partitions

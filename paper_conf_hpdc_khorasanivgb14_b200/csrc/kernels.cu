@@ -67,7 +67,7 @@ constexpr uint32_t kVB = CUSHA_VB;                   // vertex loads in flight p
 #endif
 constexpr uint32_t kEPT = CUSHA_EPT;
 #ifndef CUSHA_PF
-#define CUSHA_PF 0  // L2 prefetch of a shard's stage-3 vertex data (and delta row): 1 by the producer at ticket draw, 2 by a consumer at stage-2 start
+#define CUSHA_PF 2  // L2 prefetch of a shard's stage-3 vertex data (and delta row): 1 by the producer at ticket draw, 2 by a consumer at stage-2 start
 #endif
 #ifndef CUSHA_S4U
 #define CUSHA_S4U 1
@@ -558,6 +558,8 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
   uint32_t* const aux = A::kMonotone ? tail : sm + A::acc_lo(0) * st;
   // Mapper-delta row of the current shard (window form, p.mapj)
   uint32_t* const drow = tail + (A::kMonotone ? (N + 31) / 32 : 0);
+  // stage 1's VertexValues of the shard, for stage 3 (integer algorithms, p.stash)
+  uint32_t* const stash = drow + (p.mapj ? p.S : 0u);
   const uint32_t it0 = *reinterpret_cast<volatile uint32_t*>(&p.ctl->iter);
   // a pass launched after the run converged / hit max_iters is a no-op (host-loop mode)
   if (*reinterpret_cast<volatile uint32_t*>(&p.ctl->converged) || it0 >= p.ctl->max_iters) return;
@@ -608,7 +610,10 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
 #pragma unroll
         for (uint32_t u = 0; u < kVB; ++u) {
           const uint32_t v = base + u * kConsumers + ct;
-          if (v < nv) A::init(sm, st, v, x[u]);
+          if (v < nv) {
+            A::init(sm, st, v, x[u]);
+            if constexpr (A::kMonotone) if (p.stash) stash[v] = x[u];
+          }
         }
       }
       if (p.mapj) {  // the shard's Mapper-delta row for stage 4 (window form)
@@ -674,7 +679,8 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
           const uint32_t v = base + u * kConsumers + ct;
           od[u] = 0;
           if (v < nv) {
-            x[u] = vv[v];
+            if constexpr (A::kMonotone) x[u] = p.stash ? stash[v] : vv[v];
+            else x[u] = vv[v];
             if (A::kOutDeg) od[u] = __ldg(p.outdeg + off + v);
           }
         }
@@ -1061,6 +1067,7 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.use_cond = 0; p.cond_handle = 0;
   p.multi = 0; p.shard_seq = g.d_shard_seq;
   p.mapj = 0;
+  p.stash = 0;
   return p;
 }
 
