@@ -124,3 +124,11 @@ def test_no_cpu_fallback_without_gpu():
     with pytest.raises(cusha.CushaError) as ei:
         cusha.build_graph(4, np.array([0, 1], np.uint32), np.array([1, 2], np.uint32))
     assert ei.value.code == cusha.ECUDA
+
+
+def test_diag_timeline_absent_from_product_build():
+    """The per-ticket timeline exists only in -DCUSHA_TIMELINE=1 diagnostic
+    builds (tools/timeline.py); the product library refuses the call."""
+    buf = np.zeros(40, dtype=np.uint32)
+    assert cusha.lib().cusha_diag_timeline(buf.ctypes.data, buf.nbytes) == cusha.EUNSUPPORTED
+    assert cusha.lib().cusha_diag_timeline(None, 0) == cusha.EINVAL
