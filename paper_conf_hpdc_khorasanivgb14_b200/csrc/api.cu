@@ -351,6 +351,17 @@ static int pass_config(const Graph& g, const PassKernel& pk, size_t* smem, int* 
   return CUSHA_OK;
 }
 
+// L2 prefetch of stage-2 tiles beyond the ring (KParams::ahead) pays when a
+// pass streams from HBM; on passes that stay in L2 it only adds producer
+// latency: on when the entry streams of one pass
+// exceed twice the L2.
+static int pass_ahead(const Graph& g, int alg) {
+  int l2 = 0;
+  if (cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, g.device) != cudaSuccess || l2 <= 0) l2 = 126 << 20;
+  const uint64_t bytes = (uint64_t)g.P * (6 + (alg_needs_edge_values(alg) ? 4 : 0)) + (uint64_t)g.Q * 8;
+  return bytes > 2ull * (uint64_t)l2 ? 1 : 0;
+}
+
 static int ensure_exec(cusha_graph* h, int alg) {
   Graph& g = h->g;
   if (h->exec[alg]) return CUSHA_OK;
@@ -376,7 +387,8 @@ static int ensure_exec(cusha_graph* h, int alg) {
   KParams kp = make_params(g, 0);
   kp.use_cond = 1;
   kp.mapj = mapj;
-    kp.stash = stash;
+  kp.stash = stash;
+  kp.ahead = pass_ahead(g, alg);
   kp.cond_handle = handle;
   void* args[] = {&kp};
   cudaKernelNodeParams knp = {};
@@ -440,6 +452,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     kp.multi = 1;
     kp.mapj = mapj;
     kp.stash = stash;
+    kp.ahead = pass_ahead(g, a);
     void* args[] = {&kp};
     CKA(cudaLaunchKernel(pk.func, dim3(pass_grid(g, pk, smem)), dim3(pk.threads), args, smem, g.stream));
   } else if (max_iters > 0 && !host_loop) {
@@ -454,6 +467,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     KParams kp = make_params(g, source);
     kp.mapj = mapj;
     kp.stash = stash;
+    kp.ahead = pass_ahead(g, a);
     void* args[] = {&kp};
     const dim3 grid(pass_grid(g, pk, smem));
     const int chunk = g.G > 1 && !g.simulate ? 1 : 8;

@@ -67,6 +67,7 @@ struct KParams {
   int multi;                   // 1: one launch runs every pass (overlapped passes)
   int mapj;                    // 1: CW stage 4 uses the Mapper in window form (cw_win + delta row in smem)
   int stash;                   // 1: integer algorithms keep stage 1's VertexValues in smem for stage 3
+  int ahead;                   // 1: the producer prefetches stage-2 tiles into L2 beyond the ring (HBM-resident passes)
   uint32_t* shard_seq;         // S: passes of shard s completed (overlapped passes)
   // destination-range partition (row e); G = 1: single partition
   uint32_t G;                  // partitions

@@ -82,6 +82,9 @@ constexpr uint32_t kConsumers = kConsumerWarps * 32;
 // counters, predictor, convergence flag, ticket_done's fence and atomics) so
 // that the consumer warps go straight on with the next shard
 constexpr bool kBk = CUSHA_BK != 0;
+#ifndef CUSHA_AHEAD
+#define CUSHA_AHEAD 1  // stage-2 tiles the producer prefetches into L2 beyond the one it pushes (KParams::ahead)
+#endif
 constexpr uint32_t kPassThreads = kConsumers + 32 + (kBk ? 32 : 0);  // + 1 producer warp (+ 1 bookkeeper warp)
 constexpr uint32_t kBkWarp = kConsumerWarps + 1;
 // one finished ticket, handed from the consumers to the bookkeeper warp
@@ -394,6 +397,18 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
   // shards of this launch: one partition's range (multi-GPU) or all of them
   const uint32_t q_lo = p.part >= 0 ? p.bounds[p.part] : 0u, q_hi = p.part >= 0 ? p.bounds[p.part + 1] : p.S;
   const uint32_t Sloc = q_hi - q_lo;
+  // L2 prefetch of stage-2 tile [t0, t0 + kTile) of a shard ending at e (device-resident parts only)
+  auto pf2 = [&](uint32_t t0, uint32_t e) {
+    if (t0 >= e) return;
+    const uint32_t n = min(kTile, e - t0);
+    bulk_prefetch_l2(p.srcvalue + t0, n * 4);
+    if (t0 + n <= p.splitP) {
+      bulk_prefetch_l2(p.dest + t0, n * 2);
+      if (A::kEdge) bulk_prefetch_l2(p.ev + t0, n * 4);
+    }
+  };
+  // tiles prefetched into L2 beyond the ring, when the pass streams from HBM (KParams::ahead)
+  const uint32_t ahead = p.ahead ? CUSHA_AHEAD : 0u;
   for (uint32_t round = 0;; ++round) {
     uint32_t s;
     if (p.multi) {
@@ -460,12 +475,14 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     }
     const uint32_t kb = a & ~7u, ke = (b2 + 7u) & ~7u;
     if (b == e) push(s, kDescStage2, 0, kFlagLast | (spec ? kFlagSpec4 : 0u), nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
+    for (uint32_t j = 1; j <= ahead; ++j) pf2(b + j * kTile, e);
     for (uint32_t t0 = b; t0 < e; t0 += kTile) {
       const uint32_t n = min(kTile, e - t0);
       const uint32_t flags = (t0 + n >= e ? kFlagLast : 0u) | (t0 == b && spec ? kFlagSpec4 : 0u);
       push(s, kDescStage2, n, flags, p.srcvalue + t0, n * 4, topo_at(p.dest, p.dest_h, p.splitP, t0), 4 * kTile,
            n * 2, A::kEdge ? (const void*)topo_at(p.ev, p.ev_h, p.splitP, t0) : nullptr, 6 * kTile,
            A::kEdge ? n * 4 : 0u);
+      if (ahead) pf2(t0 + (ahead + 1) * kTile, e);
     }
     bool send4 = spec;
     if (REPR == CUSHA_REPR_CW && !spec) {
@@ -1068,6 +1085,7 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.multi = 0; p.shard_seq = g.d_shard_seq;
   p.mapj = 0;
   p.stash = 0;
+  p.ahead = 0;
   return p;
 }
 
