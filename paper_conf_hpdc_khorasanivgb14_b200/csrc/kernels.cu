@@ -85,6 +85,9 @@ constexpr bool kBk = CUSHA_BK != 0;
 #ifndef CUSHA_AHEAD
 #define CUSHA_AHEAD 1  // stage-2 tiles the producer prefetches into L2 beyond the one it pushes (KParams::ahead)
 #endif
+#ifndef CUSHA_AHEAD4
+#define CUSHA_AHEAD4 1  // the L2 read-ahead also covers CW stage-4 tiles
+#endif
 constexpr uint32_t kPassThreads = kConsumers + 32 + (kBk ? 32 : 0);  // + 1 producer warp (+ 1 bookkeeper warp)
 constexpr uint32_t kBkWarp = kConsumerWarps + 1;
 // one finished ticket, handed from the consumers to the bookkeeper warp
@@ -407,6 +410,14 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
       if (A::kEdge) bulk_prefetch_l2(p.ev + t0, n * 4);
     }
   };
+  // L2 prefetch of the CW stage-4 tile at CW position k0 (< ke), device-resident parts only
+  auto pf4 = [&](uint32_t k0, uint32_t ke) {
+    if (k0 >= ke || k0 >= p.splitQ) return;
+    const uint32_t n = min(p.mapj ? tile4j_of<A>() : tile4m_of<A>(), ke - k0);
+    bulk_prefetch_l2(p.cw_src + k0, n * 2);
+    if (p.mapj) bulk_prefetch_l2(p.cw_win + k0, n * 2);
+    else bulk_prefetch_l2(p.mapper + k0, n * 4);
+  };
   // tiles prefetched into L2 beyond the ring, when the pass streams from HBM (KParams::ahead)
   const uint32_t ahead = p.ahead ? CUSHA_AHEAD : 0u;
   for (uint32_t round = 0;; ++round) {
@@ -482,7 +493,10 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
       push(s, kDescStage2, n, flags, p.srcvalue + t0, n * 4, topo_at(p.dest, p.dest_h, p.splitP, t0), 4 * kTile,
            n * 2, A::kEdge ? (const void*)topo_at(p.ev, p.ev_h, p.splitP, t0) : nullptr, 6 * kTile,
            A::kEdge ? n * 4 : 0u);
-      if (ahead) pf2(t0 + (ahead + 1) * kTile, e);
+      if (ahead) {
+        if (t0 + (ahead + 1) * kTile < e) pf2(t0 + (ahead + 1) * kTile, e);
+        else if (CUSHA_AHEAD4 && spec && t0 + kTile >= e && a < b2) pf4(kb, ke);  // the first stage-4 tile
+      }
     }
     bool send4 = spec;
     if (REPR == CUSHA_REPR_CW && !spec) {
@@ -520,6 +534,7 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
           else
             push(s, kDescStage4, n, fl, topo_at(p.cw_src, p.cw_src_h, p.splitQ, k0), n * 2,
                  topo_at(p.mapper, p.mapper_h, p.splitQ, k0), 2 * kT4, n * 4, nullptr, 0, 0, lo, hi, k0, 0);
+          if (CUSHA_AHEAD4 && ahead) pf4(k0 + kT4, ke);
         }
     }
   }
