@@ -85,6 +85,9 @@ constexpr bool kBk = CUSHA_BK != 0;
 #ifndef CUSHA_AHEAD
 #define CUSHA_AHEAD 1  // stage-2 tiles the producer prefetches into L2 beyond the one it pushes (KParams::ahead)
 #endif
+#ifndef CUSHA_AHEAD_WAIT
+#define CUSHA_AHEAD_WAIT 1  // the read-ahead starts before the producer's ticket_wait
+#endif
 #ifndef CUSHA_AHEAD4
 #define CUSHA_AHEAD4 1  // the L2 read-ahead also covers CW stage-4 tiles
 #endif
@@ -436,6 +439,10 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
         push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
         return;
       }
+      // the shard's first stage-2 tiles start towards L2 while the producer
+      // waits (a prefetch reads nothing into the CTA, so it needs no ordering)
+      if (CUSHA_AHEAD_WAIT && ahead)
+        for (uint32_t j = 0; j <= ahead; ++j) pf2(p.shard_off[s] + j * kTile, p.shard_off[s + 1]);
       ticket_wait(p, s, cur_pass, Sloc);
       if (CUSHA_TIMELINE) tl_mark(cur_pass * Sloc + (s - q_lo), 1);
     } else {
@@ -486,7 +493,8 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     }
     const uint32_t kb = a & ~7u, ke = (b2 + 7u) & ~7u;
     if (b == e) push(s, kDescStage2, 0, kFlagLast | (spec ? kFlagSpec4 : 0u), nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
-    for (uint32_t j = 1; j <= ahead; ++j) pf2(b + j * kTile, e);
+    if (!(CUSHA_AHEAD_WAIT && p.multi))
+      for (uint32_t j = 1; j <= ahead; ++j) pf2(b + j * kTile, e);
     for (uint32_t t0 = b; t0 < e; t0 += kTile) {
       const uint32_t n = min(kTile, e - t0);
       const uint32_t flags = (t0 + n >= e ? kFlagLast : 0u) | (t0 == b && spec ? kFlagSpec4 : 0u);
