@@ -310,10 +310,13 @@ static uint32_t pass_grid(const Graph& g, const PassKernel& pk, size_t smem) {
 #ifndef CUSHA_MAPJ
 #define CUSHA_MAPJ 1  // 0: always the u32 Mapper (tuning comparison)
 #endif
+#ifndef CUSHA_DEEP_RING
+#define CUSHA_DEEP_RING 1  // 0: always the default ring depth (tuning comparison)
+#endif
 #ifndef CUSHA_STASH
 #define CUSHA_STASH 1  // 0: stage 3 of the integer algorithms re-reads VertexValues (tuning comparison)
 #endif
-static int pass_config(const Graph& g, const PassKernel& pk, size_t* smem, int* mapj, int* stash) {
+static int pass_config(const Graph& g, const PassKernel& pk, size_t* smem, int* mapj, int* stash, uint32_t* nst) {
   cudaFuncAttributes fa{};
   CKA(cudaFuncGetAttributes(&fa, pk.func));
   const size_t kMaxSmem = 227 * 1024 - fa.sharedSizeBytes;  // dynamic part of the 227 KB per-CTA limit
@@ -348,6 +351,20 @@ static int pass_config(const Graph& g, const PassKernel& pk, size_t* smem, int* 
       *stash = 1;
     }
   }
+  // a deeper TMA ring whenever another slot fits at the same CTAs per SM
+  // (more bytes in flight per SM; e.g. C5 at one CTA per SM)
+  *nst = pk.ring_bytes / pk.slot_bytes;
+  if (CUSHA_DEEP_RING) {
+    int occ_0 = 0;
+    CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_0, pk.func, (int)pk.threads, *smem));
+    while (*nst < pk.max_stages && *smem + pk.slot_bytes <= kMaxSmem) {
+      int occ_d = 0;
+      CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_d, pk.func, (int)pk.threads, *smem + pk.slot_bytes));
+      if (occ_d < occ_0 || occ_d == 0) break;
+      *smem += pk.slot_bytes;
+      ++*nst;
+    }
+  }
   return CUSHA_OK;
 }
 
@@ -368,7 +385,8 @@ static int ensure_exec(cusha_graph* h, int alg) {
   const PassKernel& pk = pass_kernel(alg, g.repr);
   size_t smem = 0;
   int mapj = 0, stash = 0;
-  const int prc = pass_config(g, pk, &smem, &mapj, &stash);
+  uint32_t nst = 0;
+  const int prc = pass_config(g, pk, &smem, &mapj, &stash, &nst);
   if (prc) return prc;
   cudaGraph_t graph = nullptr;
   CKA(cudaGraphCreate(&graph, 0));
@@ -388,6 +406,7 @@ static int ensure_exec(cusha_graph* h, int alg) {
   kp.use_cond = 1;
   kp.mapj = mapj;
   kp.stash = stash;
+  kp.nst = nst;
   kp.ahead = pass_ahead(g, alg);
   kp.cond_handle = handle;
   void* args[] = {&kp};
@@ -430,7 +449,8 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   const PassKernel& pk = pass_kernel(a, g.repr);
   size_t smem = 0;
   int mapj = 0, stash = 0;
-  int rc = pass_config(g, pk, &smem, &mapj, &stash);
+  uint32_t nst = 0;
+  int rc = pass_config(g, pk, &smem, &mapj, &stash, &nst);
   if (rc) return rc;
   const bool host_loop = g.host_loop || g.G > 1;  // the partitioned mode exchanges between passes
   // overlapped passes (default): one launch runs every pass; it needs a trace
@@ -452,6 +472,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     kp.multi = 1;
     kp.mapj = mapj;
     kp.stash = stash;
+    kp.nst = nst;
     kp.ahead = pass_ahead(g, a);
     void* args[] = {&kp};
     CKA(cudaLaunchKernel(pk.func, dim3(pass_grid(g, pk, smem)), dim3(pk.threads), args, smem, g.stream));
@@ -467,6 +488,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     KParams kp = make_params(g, source);
     kp.mapj = mapj;
     kp.stash = stash;
+    kp.nst = nst;
     kp.ahead = pass_ahead(g, a);
     void* args[] = {&kp};
     const dim3 grid(pass_grid(g, pk, smem));

@@ -68,6 +68,7 @@ struct KParams {
   int mapj;                    // 1: CW stage 4 uses the Mapper in window form (cw_win + delta row in smem)
   int stash;                   // 1: integer algorithms keep stage 1's VertexValues in smem for stage 3
   int ahead;                   // 1: the producer prefetches stage-2 tiles into L2 beyond the ring (HBM-resident passes)
+  uint32_t nst;                // ring slots of this run (kStages, or more when shared memory has room)
   uint32_t* shard_seq;         // S: passes of shard s completed (overlapped passes)
   // destination-range partition (row e); G = 1: single partition
   uint32_t G;                  // partitions
@@ -109,7 +110,9 @@ struct PassKernel {
   uint32_t words;         // shared 32-bit words per vertex (local state)
   bool wb_array;          // separate write-back value array in shared memory
   bool monotone;          // changed-bit array in shared memory
-  uint32_t ring_bytes;    // TMA tile ring
+  uint32_t ring_bytes;    // TMA tile ring (the default kStages slots)
+  uint32_t slot_bytes;    // one ring slot
+  uint32_t max_stages;    // most slots a run may use
   uint32_t threads;       // CTA size (producer warp + consumer warps)
   bool persistent;        // grid = resident CTAs pulling shards from a queue (else one CTA per shard)
   size_t smem_bytes(uint32_t N, uint32_t delta_row = 0) const;  // delta_row: words of the window-form row

@@ -65,14 +65,14 @@ constexpr uint32_t kVB = CUSHA_VB;                   // vertex loads in flight p
 #ifndef CUSHA_EPT
 #define CUSHA_EPT 4
 #endif
-constexpr uint32_t kEPT = CUSHA_EPT;
+constexpr uint32_t kEPT = CUSHA_EPT;  // stage-2 entries per consumer thread per step (4 or 8)
 #ifndef CUSHA_PF
 #define CUSHA_PF 2  // L2 prefetch of a shard's stage-3 vertex data (and delta row): 1 by the producer at ticket draw, 2 by a consumer at stage-2 start
 #endif
 #ifndef CUSHA_S4U
 #define CUSHA_S4U 1
 #endif
-constexpr uint32_t kS4U = CUSHA_S4U;  // stage-4 entries per consumer thread per step (loads before stores)  // stage-2 entries per consumer thread per step (4 or 8)
+constexpr uint32_t kS4U = CUSHA_S4U;  // stage-4 entries per consumer thread per step (loads before stores)
 constexpr uint32_t kConsumerWarps = CUSHA_CONSUMER_WARPS;
 constexpr uint32_t kConsumers = kConsumerWarps * 32;
 #ifndef CUSHA_BK
@@ -103,7 +103,13 @@ template <class A>
 constexpr uint32_t tile_of() {
   return A::kEdge ? CUSHA_TILE / 2 : CUSHA_TILE;
 }
-constexpr uint32_t kStages = CUSHA_STAGES;          // ring depth
+constexpr uint32_t kStages = CUSHA_STAGES;          // ring depth (the default)
+#ifndef CUSHA_MAX_STAGES
+#define CUSHA_MAX_STAGES 4
+#endif
+// ring depth of a run (KParams::nst): kStages, or more when shared memory has
+// room for another slot at the same CTAs per SM (chosen by the host)
+constexpr uint32_t kMaxStages = CUSHA_MAX_STAGES > CUSHA_STAGES ? CUSHA_MAX_STAGES : CUSHA_STAGES;
 constexpr uint32_t kConsumerBar = 1;                // named barrier of the consumer warps
 
 // ring slot: stage 2 = SrcValue (4T) | DestIndex (2T) | EdgeValue (4T);
@@ -398,7 +404,7 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     } else {
       mbar_arrive(&full_bar[slot]);
     }
-    if (++slot == kStages) { slot = 0; ph ^= 1; }
+    if (++slot == p.nst) { slot = 0; ph ^= 1; }
   };
   // shards of this launch: one partition's range (multi-GPU) or all of them
   const uint32_t q_lo = p.part >= 0 ? p.bounds[p.part] : 0u, q_hi = p.part >= 0 ? p.bounds[p.part + 1] : p.S;
@@ -580,9 +586,10 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
   constexpr uint32_t SLOT = slot_bytes<A>();
   constexpr uint32_t kTile = tile_of<A>();
   uint8_t* const ring = dyn;
-  uint32_t* const sm = reinterpret_cast<uint32_t*>(dyn + kStages * SLOT);
-  __shared__ uint64_t full_bar[kStages], empty_bar[kStages], decide_bar;
-  __shared__ TileDesc desc[kStages];
+  const uint32_t nst = p.nst;
+  uint32_t* const sm = reinterpret_cast<uint32_t*>(dyn + nst * SLOT);
+  __shared__ uint64_t full_bar[kMaxStages], empty_bar[kMaxStages], decide_bar;
+  __shared__ TileDesc desc[kMaxStages];
   __shared__ uint32_t s_upd;
   __shared__ int s_any;
   __shared__ unsigned long long s_stores;
@@ -605,7 +612,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
   if (*reinterpret_cast<volatile uint32_t*>(&p.ctl->converged) || it0 >= p.ctl->max_iters) return;
   const uint32_t Sloc = p.part >= 0 ? p.bounds[p.part + 1] - p.bounds[p.part] : p.S;
   if (tid == 0) {
-    for (uint32_t i = 0; i < kStages; ++i) {
+    for (uint32_t i = 0; i < nst; ++i) {
       mbar_init(&full_bar[i], 1);                // the producer's arrive(.expect_tx)
       mbar_init(&empty_bar[i], kConsumerWarps);  // one arrive per consumer warp
     }
@@ -701,7 +708,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty_bar[slot]);
-        if (++slot == kStages) { slot = 0; ph ^= 1; }
+        if (++slot == nst) { slot = 0; ph ^= 1; }
         if (d.flags & kFlagLast) break;
         mbar_wait(&full_bar[slot], ph);
         d = desc[slot];
@@ -845,7 +852,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty_bar[slot]);
-            if (++slot == kStages) { slot = 0; ph ^= 1; }
+            if (++slot == nst) { slot = 0; ph ^= 1; }
             if (d.flags & kFlagLast) break;
           }
         }
@@ -1056,6 +1063,8 @@ static PassKernel make_pk() {
   k.wb_array = !A::kMonotone;
   k.monotone = A::kMonotone;
   k.ring_bytes = kStages * slot_bytes<A>();
+  k.slot_bytes = slot_bytes<A>();
+  k.max_stages = kMaxStages;
   k.threads = kPassThreads;
   k.persistent = kPersistent;
   return k;
@@ -1109,6 +1118,7 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.mapj = 0;
   p.stash = 0;
   p.ahead = 0;
+  p.nst = kStages;
   return p;
 }
 
