@@ -131,7 +131,11 @@ typedef struct {
    * nothing (L189), so results are those of the barrier mode.  1 = one launch
    * per pass under a CUDA-graph while node, with a device-wide barrier between
    * passes as in Fig. 5.  host_loop = 1 or world_size > 1 imply one launch
-   * per pass.                                                              */
+   * per pass.  0 is automatic: with many small shards (>= 16 shards per
+   * resident CTA and <= 16384 entries per shard on average) the per-ticket
+   * costs of overlapped passes outweigh the barrier they save, and the run
+   * uses one launch per pass (measured);
+   * 2 = overlapped passes always.                                          */
   int pass_barrier;
 } cusha_build_opts;
 

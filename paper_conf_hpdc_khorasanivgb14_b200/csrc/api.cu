@@ -148,6 +148,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
     return fail(CUSHA_EINVAL, "rank out of range");
   uint32_t N = o.vertices_per_shard ? o.vertices_per_shard : cusha_shard_size(V, E, o.smem_bytes_per_vertex, 0, 0);
   if (N > 65534) return fail(CUSHA_EINVAL, "vertices_per_shard must be <= 65534");
+  if (o.pass_barrier < 0 || o.pass_barrier > 2) return fail(CUSHA_EINVAL, "pass_barrier must be 0, 1 or 2");
   if (N > V) N = V;
 
   cusha_graph* h = new (std::nothrow) cusha_graph();
@@ -156,7 +157,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   g.V = V; g.E = E; g.N = N; g.S = (V + N - 1) / N; g.repr = (int)o.repr; g.device = o.device;
   g.host_loop = o.host_loop != 0;
   g.skip_clean = o.skip_clean_shards != 0;
-  g.pass_barrier = o.pass_barrier != 0;
+  g.pass_barrier = o.pass_barrier;
   g.topo_budget = o.device_topology_budget;
   g.world_size = o.world_size;
   g.rank = o.world_size > 1 && o.nccl_unique_id ? o.rank : 0;
@@ -328,7 +329,12 @@ static int pass_config(const Graph& g, const PassKernel& pk, size_t* smem, int* 
   *smem = sm_m;
   *mapj = 0;
   const size_t sm_j = pk.smem_bytes(g.N, g.S);
-  if (CUSHA_MAPJ && g.repr == CUSHA_REPR_CW && g.d_cw_win && g.d_cw_delta && !kernels_rle() && g.S <= 0xFFFFu && sm_j <= kMaxSmem) {
+  // ... and only when the rows cost less traffic than they save: an active
+  // shard reads its 4|S|-byte row, so |S| rows per pass (4|S|^2 bytes) against
+  // 2 bytes per CW entry (|Q| entries) saved over the u32 Mapper
+  const bool row_pays = 4ull * g.S * g.S <= (uint64_t)g.Q;
+  if (CUSHA_MAPJ && row_pays && g.repr == CUSHA_REPR_CW && g.d_cw_win && g.d_cw_delta && !kernels_rle() &&
+      g.S <= 0xFFFFu && sm_j <= kMaxSmem) {
     int occ_m = 0, occ_j = 0;
     CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_m, pk.func, (int)pk.threads, sm_m));
     CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_j, pk.func, (int)pk.threads, sm_j));
@@ -455,7 +461,14 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   const bool host_loop = g.host_loop || g.G > 1;  // the partitioned mode exchanges between passes
   // overlapped passes (default): one launch runs every pass; it needs a trace
   // record per pass (<= 2^20), else the CUDA-graph loop runs one launch per pass
-  const bool multi = !host_loop && !g.pass_barrier && max_iters <= g.trace_cap;
+  // automatic mode: many small shards per CTA favour one launch per pass
+  // (67_16 at |N| = 1536: 4.40 vs 5.48 ms)
+  bool barrier = g.pass_barrier == 1;
+  if (g.pass_barrier == 0 && g.S) {
+    const uint64_t grid = pass_grid(g, pk, smem);
+    barrier = (uint64_t)g.S >= 16 * grid && g.P <= 16384ull * g.S;
+  }
+  const bool multi = !host_loop && !barrier && max_iters <= g.trace_cap;
   if (!host_loop && !multi) {
     rc = ensure_exec(h, a);
     if (rc) return rc;
@@ -492,7 +505,11 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     kp.ahead = pass_ahead(g, a);
     void* args[] = {&kp};
     const dim3 grid(pass_grid(g, pk, smem));
-    const int chunk = g.G > 1 && !g.simulate ? 1 : 8;
+    // 8 passes per host check, multi-GPU too: a pass launched after the run
+    // converged exits at once and the exchange / refresh after it change
+    // nothing, and every rank reads the same convergence flag after the same
+    // chunk, so all ranks issue the same collectives
+    const int chunk = 8;
     std::string err;
     for (;;) {
       for (int k = 0; k < chunk; ++k) {

@@ -138,7 +138,7 @@ struct Graph {
   uint8_t* d_active = nullptr;      // S: stage-4 prefetch predictor
   uint32_t* d_dirty = nullptr;      // S: clean-shard skipping flags
   uint32_t* d_shard_seq = nullptr;  // S: overlapped passes, per-shard pass order
-  bool pass_barrier = false;        // 1: one launch per pass (CUDA-graph while loop)
+  int pass_barrier = 0;             // 0: automatic, 1: one launch per pass (CUDA-graph while loop), 2: overlapped
   int mapj = -1;                    // per-run choice of the Mapper form (-1: not chosen yet)
   bool skip_clean = false;
   // host-streamed topology (row f3): shards >= host_shard keep their entry

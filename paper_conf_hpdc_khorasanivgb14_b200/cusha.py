@@ -218,14 +218,15 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
                 smem_bytes_per_vertex: int = 0, device: int = 0, stream: Optional[int] = None,
                 host_loop: bool = False, world_size: int = 1, rank: int = 0,
                 nccl_id: Optional[bytes] = None, skip_clean_shards: bool = False,
-                device_topology_budget: int = 0, pass_barrier: bool = False) -> Graph:
+                device_topology_budget: int = 0, pass_barrier: int = 0) -> Graph:
     """cusha_build_graph.  src/dst/edge_values: numpy (host, copied in) or CUDA tensors (device).
     world_size > 1: destination-range partition; nccl_id = None simulates all
     partitions on this device, else one process per GPU over NCCL.
     skip_clean_shards: opt-in exact skipping of shards whose inputs did not change.
     device_topology_budget: HBM bytes for per-entry topology; the rest is streamed from pinned host memory.
-    pass_barrier: one launch per pass with a device-wide barrier between passes (Fig. 5) instead of
-    the default overlapped passes (one launch per run)."""
+    pass_barrier: True / 1 = one launch per pass with a device-wide barrier between passes (Fig. 5);
+    2 = always overlapped passes (one launch per run); False / 0 = automatic (overlapped unless the
+    graph has many small shards per CTA, include/cusha.h)."""
     on_dev = _is_device(src)
     if not on_dev:
         src = np.ascontiguousarray(src, dtype=np.uint32)

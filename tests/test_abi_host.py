@@ -106,6 +106,11 @@ def test_build_graph_argument_errors():
     o = cusha.BuildOpts()
     o.vertices_per_shard = 70000
     assert L.cusha_build_graph(100000, 1, cusha._ptr(s), cusha._ptr(s), None, ctypes.byref(o), ctypes.byref(h)) == cusha.EINVAL
+    # iteration-boundary mode outside {0 auto, 1 barrier, 2 overlapped}
+    o = cusha.BuildOpts()
+    o.pass_barrier = 3
+    assert L.cusha_build_graph(4, 1, cusha._ptr(s), cusha._ptr(s), None, ctypes.byref(o), ctypes.byref(h)) == cusha.EINVAL
+    assert b"pass_barrier" in L.cusha_last_error()
     # multi-GPU through the single-GPU entry point
     o = cusha.BuildOpts()
     o.world_size = 2

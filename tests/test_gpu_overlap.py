@@ -104,3 +104,19 @@ def test_skip_clean_with_overlap():
     for repr in ("gs", "cw"):
         got, st = gpu_run("sssp", wl.V, wl.src, wl.dst, ev=wl.edge_u32, repr=repr, N=400, skip=True)
         np.testing.assert_array_equal(got, want)
+
+
+@pytest.mark.parametrize("mode", [0, 2])
+@pytest.mark.parametrize("alg", ["bfs", "sssp"])
+def test_automatic_mode_many_small_shards(alg, mode):
+    """pass_barrier = 0 (automatic) picks one launch per pass when there are
+    >= 16 shards per resident CTA of <= 16K entries each (include/cusha.h);
+    2 forces overlapped passes.  Both reach the oracle's fixed point."""
+    V = 400_000
+    s, d = graphgen.rmat(V, 2_000_000, seed=91)
+    w = graphgen.edge_u32(s, d, seed=91, lo=1, hi=255)
+    want = oracle.bfs(V, s, d, 0) if alg == "bfs" else oracle.sssp(V, s, d, w, 0)
+    got, st = gpu_run(alg, V, s, d, ev=w if alg == "sssp" else None, repr="cw", N=64, pass_barrier=mode)
+    np.testing.assert_array_equal(got, want)
+    assert st["num_shards"] == 6250
+    assert st["device_loop"] == (1 if mode == 0 else 2)
