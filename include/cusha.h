@@ -123,19 +123,21 @@ typedef struct {
    * are identical to the in-HBM layout.  The build itself runs in HBM first.  */
   uint64_t device_topology_budget;
   /* Iteration boundary of the device loop (row a5; DESIGN.md "Overlapped
-   * passes").  0 (default) = one launch runs every pass: shards are drawn as
-   * tickets across passes, so a CTA done with its part of pass k starts pass
-   * k+1 (the asynchronous model of L45 carried across the iteration
-   * boundary; a shard's passes stay in order).  Convergence is concluded only
-   * from a pass that started after every earlier pass completed and committed
-   * nothing (L189), so results are those of the barrier mode.  1 = one launch
-   * per pass under a CUDA-graph while node, with a device-wide barrier between
-   * passes as in Fig. 5.  host_loop = 1 or world_size > 1 imply one launch
-   * per pass.  0 is automatic: with many small shards (>= 16 shards per
-   * resident CTA and <= 16384 entries per shard on average) the per-ticket
-   * costs of overlapped passes outweigh the barrier they save, and the run
-   * uses one launch per pass (measured);
-   * 2 = overlapped passes always.                                          */
+   * passes").
+   *  2 = overlapped passes: one launch runs every pass; shards are drawn as
+   *      tickets across passes, so a CTA done with its part of pass k starts
+   *      pass k+1 (the asynchronous model of L45 carried across the iteration
+   *      boundary; a shard's passes stay in order).  Convergence is concluded
+   *      only from a pass that started after every earlier pass completed and
+   *      committed nothing (L189), so results are those of the barrier mode.
+   *  1 = one launch per pass under a CUDA-graph while node, with a
+   *      device-wide barrier between passes as in Fig. 5.
+   *  0 (default) = automatic: 2, except with many small shards (>= 16 shards
+   *      per resident CTA and <= 16384 entries per shard on average), where
+   *      the per-ticket costs of overlapped passes outweigh the barrier they
+   *      save and the run uses 1 (measured).
+   * host_loop = 1 or world_size > 1 imply one launch per pass.  Other values:
+   * CUSHA_EINVAL.                                                          */
   int pass_barrier;
 } cusha_build_opts;
 
