@@ -3,7 +3,7 @@
 // whose body kernel sets the condition from device code, with none of the
 // shard-pass code involved?
 //   nvcc -gencode arch=compute_100a,code=sm_100a -o cond_memcheck cond_memcheck.cu -lcudadevrt -rdc=true
-//   ./cond_memcheck [runs] [pad] [async]; compute-sanitizer --tool memcheck ./cond_memcheck [runs] [pad]
+//   ./cond_memcheck [runs] [pad] [async] [iters]; compute-sanitizer --tool memcheck ./cond_memcheck [runs] [pad]
 // `pad` = 1 passes a large by-value parameter struct (like the shard pass's KParams);
 // `pad` = 2 runs the TMA/mbarrier/last-CTA body below.
 #include <cstdio>
@@ -126,7 +126,10 @@ int main(int argc, char** argv) {
   cudaGraphExec_t ex;
   CK(cudaGraphInstantiate(&ex, graph, 0));
   for (int r = 0; r < runs; ++r) {
-    Ctl c0 = {0u, 7u + (unsigned)r};
+    // argv[4]: iterations per run (default 7), so a run can still be looping on the
+    // device when the host issues its next API call
+    const unsigned base = argc > 4 ? (unsigned)std::atoi(argv[4]) : 7u;
+    Ctl c0 = {0u, base + (unsigned)r};
     CK(cudaMemcpyAsync(ctl, &c0, sizeof c0, cudaMemcpyHostToDevice, s));
     CK(cudaGraphLaunch(ex, s));
     Ctl c1;
