@@ -120,3 +120,28 @@ def test_automatic_mode_many_small_shards(alg, mode):
     np.testing.assert_array_equal(got, want)
     assert st["num_shards"] == 6250
     assert st["device_loop"] == (1 if mode == 0 else 2)
+
+
+@pytest.mark.parametrize("repr", ["gs", "cw"])
+def test_pass_barrier_graph_reuse(c1, repr):
+    """pass_barrier = 1: the instantiated CUDA graph (one per algorithm) is
+    reused across runs on one handle, with changing sources and algorithms
+    interleaved; every run must still reach the oracle's fixed point (L189)."""
+    from paper_conf_hpdc_khorasanivgb14_b200 import cusha
+    V, s, d, w = c1
+    with cusha.build_graph(V, s, d, edge_values=w, repr=repr, vertices_per_shard=128, pass_barrier=1) as g:
+        for source in (0, 17, V - 1, 0):
+            for alg in ("bfs", "sssp", "cc", "sswp"):
+                rc = cusha.run(alg, g, source=source)
+                assert rc == cusha.OK
+                got = cusha.get_values(g)
+                if alg == "bfs":
+                    want = oracle.bfs(V, s, d, source)
+                elif alg == "sssp":
+                    want = oracle.sssp(V, s, d, w, source)
+                elif alg == "sswp":
+                    want = oracle.sswp(V, s, d, w, source)
+                else:
+                    want = oracle.cc(V, s, d)
+                np.testing.assert_array_equal(got, want, err_msg=f"{alg} source {source}")
+                assert cusha.get_stats(g)["device_loop"] == 1
