@@ -1,5 +1,5 @@
 """Small runs of every launch mode for compute-sanitizer (profiles/r1/sanitizer/).
-usage: compute-sanitizer --tool memcheck python tools/san_small.py [all | mode ...]  (SAN_REPR=gs|cw)"""
+usage: compute-sanitizer --tool memcheck python tools/san_small.py [all | mode ...]  (SAN_REPR=gs|cw, SAN_N=500)"""
 import os
 import sys
 
@@ -17,6 +17,7 @@ names = sys.argv[1:] or ["default"]
 if names == ["all"]:
     names = list(ALL)
 reprs = [r for r in ("gs", "cw") if os.environ.get("SAN_REPR", r) == r]
+NPS = int(os.environ.get("SAN_N", "500"))  # vertices per shard
 for mname in names:
     kw = ALL[mname]
     for repr_ in reprs:
@@ -24,7 +25,7 @@ for mname in names:
             continue  # the partitioned mode uses CW (include/cusha.h)
         for alg in ("bfs", "sssp", "pr", "cc"):
             with cusha.build_graph(V, s, d, edge_values=w if alg == "sssp" else None, repr=repr_,
-                                   vertices_per_shard=500, **kw) as g:
+                                   vertices_per_shard=NPS, **kw) as g:
                 cusha.run(alg, g, source=0)
                 cusha.get_values(g)
             print(mname, repr_, alg, "ok", flush=True)
