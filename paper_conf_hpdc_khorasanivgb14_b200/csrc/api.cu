@@ -385,6 +385,9 @@ static int pass_ahead(const Graph& g, int alg) {
   return bytes > 2ull * (uint64_t)l2 ? 1 : 0;
 }
 
+#ifndef CUSHA_DIAG_FIXED_GRAPH
+#define CUSHA_DIAG_FIXED_GRAPH 0
+#endif
 static int ensure_exec(cusha_graph* h, int alg) {
   Graph& g = h->g;
   if (h->exec[alg]) return CUSHA_OK;
@@ -396,6 +399,35 @@ static int ensure_exec(cusha_graph* h, int alg) {
   if (prc) return prc;
   cudaGraph_t graph = nullptr;
   CKA(cudaGraphCreate(&graph, 0));
+#if CUSHA_DIAG_FIXED_GRAPH
+  // sanitizer diagnostic only (profiles/r1/sanitizer/README.md): a chain of
+  // CUSHA_DIAG_FIXED_GRAPH per-pass launches without the conditional node; a
+  // pass launched after convergence is a no-op, as in the host loop
+  {
+    KParams kp = make_params(g, 0);
+    kp.mapj = mapj;
+    kp.stash = stash;
+    kp.nst = nst;
+    kp.ahead = pass_ahead(g, alg);
+    void* args[] = {&kp};
+    cudaKernelNodeParams knp = {};
+    knp.func = const_cast<void*>(pk.func);
+    knp.gridDim = dim3(pass_grid(g, pk, smem));
+    knp.blockDim = dim3(pk.threads);
+    knp.sharedMemBytes = (unsigned)smem;
+    knp.kernelParams = args;
+    cudaGraphNode_t prev = nullptr, kn;
+    cudaError_t e = cudaSuccess;
+    for (int i = 0; i < CUSHA_DIAG_FIXED_GRAPH && e == cudaSuccess; ++i) {
+      e = cudaGraphAddKernelNode(&kn, graph, prev ? &prev : nullptr, prev ? 1 : 0, &knp);
+      prev = kn;
+    }
+    if (e == cudaSuccess) e = cudaGraphInstantiate(&h->exec[alg], graph, 0);
+    cudaGraphDestroy(graph);
+    if (e != cudaSuccess) { h->exec[alg] = nullptr; return fail(CUSHA_ECUDA, std::string("graph: ") + cudaGetErrorString(e)); }
+    return CUSHA_OK;
+  }
+#endif
   cudaGraphConditionalHandle handle;
   cudaError_t e = cudaGraphConditionalHandleCreate(&handle, graph, 1, cudaGraphCondAssignDefault);
   if (e != cudaSuccess) { cudaGraphDestroy(graph); return fail(CUSHA_ECUDA, std::string("conditional handle: ") + cudaGetErrorString(e)); }

@@ -1,11 +1,14 @@
 """Small runs of every launch mode for compute-sanitizer (profiles/r1/sanitizer/).
-usage: compute-sanitizer --tool memcheck python tools/san_small.py [all | mode ...]  (SAN_REPR=gs|cw, SAN_N=500)"""
+usage: compute-sanitizer --tool memcheck python tools/san_small.py [all | mode ...]  (SAN_REPR=gs|cw, SAN_N=500, SAN_LIB=variant .so)"""
 import os
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import graphgen  # noqa: E402
 from paper_conf_hpdc_khorasanivgb14_b200 import cusha  # noqa: E402
+
+if os.environ.get("SAN_LIB"):  # a variant library (tools/tune.sh build)
+    cusha.LIB_PATH = os.path.abspath(os.environ["SAN_LIB"])
 
 V = 20000
 s, d = graphgen.rmat(V, 200000, seed=71)
