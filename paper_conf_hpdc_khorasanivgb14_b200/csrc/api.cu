@@ -388,6 +388,17 @@ static int pass_ahead(const Graph& g, int alg) {
 #ifndef CUSHA_DIAG_FIXED_GRAPH
 #define CUSHA_DIAG_FIXED_GRAPH 0
 #endif
+#ifndef CUSHA_DIAG_COND_NODE
+#define CUSHA_DIAG_COND_NODE 0
+#endif
+#if CUSHA_DIAG_COND_NODE
+// sanitizer diagnostic only: the while condition set by a one-thread kernel
+// after the pass (the pass runs with use_cond = 0 and closes the iteration)
+__global__ void diag_set_cond(const Ctl* ctl, cudaGraphConditionalHandle h) {
+  const uint32_t more = !*reinterpret_cast<const volatile uint32_t*>(&ctl->converged) && ctl->iter < ctl->max_iters;
+  cudaGraphSetConditional(h, more ? 1u : 0u);
+}
+#endif
 static int ensure_exec(cusha_graph* h, int alg) {
   Graph& g = h->g;
   if (h->exec[alg]) return CUSHA_OK;
@@ -441,7 +452,7 @@ static int ensure_exec(cusha_graph* h, int alg) {
   if (e != cudaSuccess) { cudaGraphDestroy(graph); return fail(CUSHA_ECUDA, std::string("conditional node: ") + cudaGetErrorString(e)); }
   cudaGraph_t body = cp.conditional.phGraph_out[0];
   KParams kp = make_params(g, 0);
-  kp.use_cond = 1;
+  kp.use_cond = CUSHA_DIAG_COND_NODE ? 0 : 1;
   kp.mapj = mapj;
   kp.stash = stash;
   kp.nst = nst;
@@ -456,6 +467,19 @@ static int ensure_exec(cusha_graph* h, int alg) {
   knp.kernelParams = args;
   cudaGraphNode_t kn;
   e = cudaGraphAddKernelNode(&kn, body, nullptr, 0, &knp);
+#if CUSHA_DIAG_COND_NODE
+  if (e == cudaSuccess) {
+    const Ctl* ctlp = g.d_ctl;
+    void* cargs[] = {&ctlp, &handle};
+    cudaKernelNodeParams cnp = {};
+    cnp.func = reinterpret_cast<void*>(diag_set_cond);
+    cnp.gridDim = dim3(1);
+    cnp.blockDim = dim3(1);
+    cnp.kernelParams = cargs;
+    cudaGraphNode_t sn;
+    e = cudaGraphAddKernelNode(&sn, body, &kn, 1, &cnp);
+  }
+#endif
   if (e == cudaSuccess) e = cudaGraphInstantiate(&h->exec[alg], graph, 0);
   cudaGraphDestroy(graph);
   if (e != cudaSuccess) { h->exec[alg] = nullptr; return fail(CUSHA_ECUDA, std::string("graph: ") + cudaGetErrorString(e)); }
