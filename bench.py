@@ -112,16 +112,40 @@ def load_graph(name, cache):
 def traffic_for(workload, overlapped, passes):
     """DRAM bytes (read + write) of one shard_pass launch from the committed ncu
     --set full capture (profiles/traffic.json), for the launch shape this run
-    used.  A captured whole-run launch is scaled by passes (this launch's over
-    the captured one's): the pass count of a PR run varies by a few between runs."""
+    used, and where that capture came from.  A captured whole-run launch is
+    scaled by passes (this launch's over the captured one's): the pass count of
+    a PR run varies by a few between runs.  It is NOT measured in this run (ncu
+    replays each kernel ~40 times; a number taken under a profiler is never a
+    bench value), hence the label."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
     if not os.path.exists(p):
-        return None
+        return None, None
     with open(p) as f:
         t = json.load(f).get(f"{workload}:{'run' if overlapped else 'pass'}")
     if not t:
-        return None
-    return int(t["bytes"] * (passes / t["passes"] if overlapped else 1))
+        return None, None
+    src = {"file": "profiles/traffic.json", "capture": t.get("file"), "commit": t.get("commit"),
+           "captured_passes": t.get("passes"), "kind": "committed ncu --set full capture, scaled per launch"}
+    return int(t["bytes"] * (passes / t["passes"] if overlapped else 1)), src
+
+
+def oracle_pr_sweeps(wl, k):
+    """Wall time of k fp64 Jacobi sweeps of oracle.pagerank over the full edge
+    list, CSR build excluded: the difference of a (k+1)-sweep and a 1-sweep
+    call (each call builds its own CSR)."""
+    import oracle
+    t0 = time.perf_counter()
+    oracle.pagerank(wl.V, wl.src, wl.dst, tol=0.0, max_iters=1, allow_notconv=True)
+    t1 = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    oracle.pagerank(wl.V, wl.src, wl.dst, tol=0.0, max_iters=k + 1, allow_notconv=True)
+    tk = time.perf_counter() - t0
+    return max(tk - t1, 1e-9), t1
+
+
+def pr_sample_text(wl, k):
+    return (f"{k} fp64 Jacobi sweeps of oracle.pagerank over the full {wl.name} edge list ({wl.E} edges each); "
+            "CSR build excluded (difference of a (k+1)-sweep and a 1-sweep call)")
 
 
 def cpu_baseline(wl, alg, source, budget_s=15.0):
@@ -129,16 +153,11 @@ def cpu_baseline(wl, alg, source, budget_s=15.0):
     import oracle
     V, s, d = wl.V, wl.src, wl.dst
     if alg == "pr":
-        t0 = time.perf_counter()
-        oracle.pagerank(V, s, d, tol=0.0, max_iters=1, allow_notconv=True)
-        t1 = time.perf_counter() - t0            # CSR build + 1 sweep
+        _, t1 = oracle_pr_sweeps(wl, 1)          # ~ CSR build + 2 sweeps: sizes the sample
         k = max(2, int(budget_s / max(t1, 1e-3)))
-        t0 = time.perf_counter()
-        oracle.pagerank(V, s, d, tol=0.0, max_iters=k + 1, allow_notconv=True)
-        tk = time.perf_counter() - t0
-        sweeps_time = max(tk - t1, 1e-9)
-        val = k * wl.E / sweeps_time / 1e9
-        sample = f"{k} fp64 Jacobi sweeps of oracle.pagerank over the full {GRAPH_OF_NAME(wl)} edge list ({wl.E} edges each); CSR build excluded"
+        el, _ = oracle_pr_sweeps(wl, k)
+        val = k * wl.E / el / 1e9
+        sample = pr_sample_text(wl, k)
     else:
         fn = {"bfs": lambda: oracle.bfs(V, s, d, source), "cc": lambda: oracle.cc(V, s, d),
               "sssp": lambda: oracle.sssp(V, s, d, wl.edge_u32, source),
@@ -152,13 +171,21 @@ def cpu_baseline(wl, alg, source, budget_s=15.0):
                 break
         el = time.perf_counter() - t0
         val = n * wl.E / el / 1e9
-        sample = f"{n} full oracle.{alg} runs (textbook definition; each edge relaxed once) on {GRAPH_OF_NAME(wl)}"
+        sample = f"{n} full oracle.{alg} runs (textbook definition; each edge relaxed once) on {wl.name}"
     return {"value": round(val, 6), "unit": "GTEPS", "cores": 1, "kind": "oracle", "sample": sample,
             "host_cores_available": os.cpu_count()}
 
 
-def GRAPH_OF_NAME(wl):
-    return wl.name
+def static_config(workload, wl, alg, repr_):
+    """`config` of both arms (identical): the workload, and whether a pass's
+    inputs exceed L2 (no flush is needed then).  Per-run facts go to `run`."""
+    desc = WORKLOADS[workload][3]
+    evb = 4 if alg in ("sssp", "sswp", "nn", "hs", "cs") else 0
+    per_pass = wl.E * (6 + evb)                # stage-2 stream of one pass (compressed layout, DESIGN.md §7)
+    l2 = (f"inputs larger than L2: {per_pass / 1e9:.3f} GB streamed by stage 2 per pass vs 0.126 GB L2"
+          if per_pass > L2_BYTES else f"L2-resident workload ({per_pass / 1e6:.1f} MB per pass); no flush")
+    return {"workload": workload, "description": desc, "V": wl.V, "E": wl.E, "algorithm": alg, "repr": repr_,
+            "l2": l2}
 
 
 def bench_reference(args):
@@ -167,6 +194,10 @@ def bench_reference(args):
     if rank != 0:
         return 0
     alg, repr_, source, desc = WORKLOADS[args.workload]
+    if args.repr:
+        repr_ = args.repr
+    if args.gpus > 1:
+        repr_ = "cw"  # as the cusha arm: the partitioned mode uses CW
     wl = load_graph(args.workload, args.cache_dir)
     import oracle
     V, s, d = wl.V, wl.src, wl.dst
@@ -183,24 +214,45 @@ def bench_reference(args):
         else:
             oracle.sswp(V, s, d, wl.edge_u32, source)
 
-    for _ in range(args.warmup):
-        step()
-    t0 = time.perf_counter()
-    for _ in range(args.steps):
-        step()
-    el = time.perf_counter() - t0
+    if alg == "pr":
+        # the same measurement as the cusha arm's cpu_baseline: a step = one
+        # fp64 sweep over the whole graph, the CSR build excluded
+        if args.warmup:
+            oracle.pagerank(V, s, d, tol=0.0, max_iters=args.warmup, allow_notconv=True)
+        el, _ = oracle_pr_sweeps(wl, args.steps)
+        sample = pr_sample_text(wl, args.steps)
+    else:
+        for _ in range(args.warmup):
+            step()
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            step()
+        el = time.perf_counter() - t0
+        sample = f"{args.steps} full oracle.{alg} runs (textbook definition; each edge relaxed once) on {wl.name}"
     val = args.steps * wl.E / el / 1e9
-    sample = ("one fp64 Jacobi sweep of oracle.pagerank (incl. its CSR build) per step" if alg == "pr"
-              else f"one full oracle.{alg} run per step")
     line = {"impl": "reference", "metric": METRIC,
             "value": round(val, 6), "unit": "GTEPS", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": round(el / args.steps * 1e3, 3), "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64" if alg == "pr" else "u32", "data": "synthetic",
-            "config": {"workload": args.workload, "description": desc, "V": V, "E": wl.E},
-            "cpu_baseline": {"value": round(val, 6), "unit": "GTEPS", "cores": 1, "kind": "oracle", "sample": sample},
+            "config": static_config(args.workload, wl, alg, repr_),
+            "cpu_baseline": {"value": round(val, 6), "unit": "GTEPS", "cores": 1, "kind": "oracle", "sample": sample,
+                             "host_cores_available": os.cpu_count()},
             "e2e": {"value": round(val, 6), "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
+
+
+def kernel_launches(st, world_local_parts):
+    """Our kernels in one cusha_run: reset_ctl,
+    init_vertex_values and init_srcvalue per partition, then the passes: one
+    launch (overlapped passes, device_loop 2) or chunks of 16 per-pass launches
+    per partition (+ one close_parts per pass slot when partitioned)."""
+    parts = world_local_parts
+    n = 3 * parts
+    if st["device_loop"] == 2:
+        return n + 1
+    chunks = max(1, -(-st["iterations"] // 16))
+    return n + 16 * chunks * (parts + (1 if st["partitions"] > 1 else 0))
 
 
 def bench_cusha(args):
@@ -217,9 +269,11 @@ def bench_cusha(args):
     dist = None
     nccl_id = None
     if world > 1:
-        # one process per GPU; the shard pass exchanges over NCCL inside libcusha
-        # (destination-range partition); torch.distributed only
-        # carries rank 0's ncclUniqueId, the barriers and the max-over-ranks time
+        # one process per GPU; libcusha's stage 4 stores into the other ranks'
+        # SrcValue over NVLink (CUDA IPC) and NCCL all-reduces the per-pass
+        # convergence word (destination-range partition);
+        # torch.distributed only carries rank 0's ncclUniqueId, the barriers and
+        # the max-over-ranks time
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device(f"cuda:{dev}"))
         idt = torch.zeros(128, dtype=torch.uint8, device=f"cuda:{dev}")
@@ -232,11 +286,14 @@ def bench_cusha(args):
         args.N = 128  # the L310 rule gives 3 shards at this size
     if args.repr:
         repr_ = args.repr
-    if world > 1:
+    if world > 1 or args.sim_parts > 1:
         repr_ = "cw"  # the partitioned mode uses CW
     wl = load_graph(args.workload, args.cache_dir)
     stream = torch.cuda.current_stream()
-    part = dict(world_size=world, rank=rank, nccl_id=nccl_id)
+    if world > 1:
+        part = dict(world_size=world, rank=rank, nccl_id=nccl_id)
+    else:
+        part = dict(world_size=max(1, args.sim_parts))  # > 1: one-process partition simulation (tests/tools)
 
     def barrier():
         if dist is not None:
@@ -268,8 +325,10 @@ def bench_cusha(args):
                           skip_clean_shards=args.skip_clean, pass_barrier=args.pass_barrier, **part)
     st0 = cusha.get_stats(g)
     log(f"[bench] rank {rank}/{world} built {repr_} |N|={st0['vertices_per_shard']} |S|={st0['num_shards']} "
-        f"in {st0['build_ms']:.1f} ms")
+        f"partitions={st0['partitions']} in {st0['build_ms']:.1f} ms; device bytes {st0['device_bytes'] / 1e9:.3f} GB "
+        f"(largest partition {st0['max_part_device_bytes'] / 1e9:.3f} GB)")
     del src_d, dst_d, ev
+    local_parts = st0["partitions"] if world == 1 else 1
 
     for _ in range(args.warmup):
         cusha.run(alg, g, source=source)
@@ -281,29 +340,26 @@ def bench_cusha(args):
         e0.record(stream)
         for _ in range(args.steps):
             rc = cusha.run(alg, g, source=source)
-            st = cusha.get_stats(g)
-            steps.append((rc, st["iterations"], st["loop_ms"], st["run_ms"], st["algorithmic_bytes"],
-                          st["edges_processed"], st["device_loop"]))
+            steps.append(cusha.get_stats(g))
         e1.record(stream)
         torch.cuda.synchronize()
     barrier()
     clocks = clk.result()
     total_ms = max_over_ranks(e0.elapsed_time(e1))  # device time, max over ranks
-    edges = sum_over_ranks(sum(s[5] for s in steps))  # each rank streams its partition's edges
-    iters = [s[1] for s in steps]
-    loop_ms = sum(s[2] for s in steps)
-    alg_bytes = sum(s[4] for s in steps)
+    edges = sum_over_ranks(sum(s["edges_processed"] for s in steps))  # each rank streams its partition's edges
+    iters = [s["iterations"] for s in steps]
+    loop_ms = max_over_ranks(sum(s["loop_ms"] for s in steps))
+    alg_bytes = sum_over_ranks(sum(s["algorithmic_bytes"] for s in steps))
+    paper_bytes = sum_over_ranks(sum(s["paper_bytes"] for s in steps))
     value = edges / (total_ms / 1e3) / 1e9
-    # reset_ctl + init_vertex_values + init_srcvalue + the passes: one launch for all of them
-    # (overlapped passes, device_loop 2) or one per iteration (+ one refresh when partitioned)
-    launches = sum(3 + (1 if s[6] == 2 else s[1] * (2 if world > 1 else 1)) for s in steps)
-    launches = int(sum_over_ranks(launches))
-    overlapped = steps[-1][6] == 2
+    launches = int(sum_over_ranks(sum(kernel_launches(s, local_parts) for s in steps)))
+    overlapped = steps[-1]["device_loop"] == 2
     n_pass_launches = len(steps) if overlapped else sum(iters)
     peak, peak_kind = measured_peak_gbs()
-    achieved = alg_bytes / (loop_ms / 1e3) / 1e9
+    # one GPU's bandwidth is the roofline of its shard passes: bytes per GPU per second
+    achieved = alg_bytes / world / (loop_ms / 1e3) / 1e9
+    achieved_paper = paper_bytes / world / (loop_ms / 1e3) / 1e9
     st = cusha.get_stats(g)
-    per_iter_gb = (st["stage2_bytes_per_iter"] + st["wb_bytes_all_active"]) / 1e9
     g.close()
 
     # ---- e2e through the public API from pinned host buffers
@@ -343,6 +399,8 @@ def bench_cusha(args):
                "d2h_bytes_per_step": wl.V * vb * world, "ms_per_step": round(el / n_e2e * 1e3, 3),
                "steps": n_e2e, "warmup": 1}
 
+    traffic, traffic_src = traffic_for(args.workload, overlapped, sum(iters) / len(iters)) \
+        if world == 1 and local_parts == 1 else (None, None)
     line = {
         "metric": METRIC,
         "value": round(value, 4),
@@ -356,26 +414,33 @@ def bench_cusha(args):
         "vs_baseline": None,
         "dtype": "f32" if alg in ("pr", "nn", "hs", "cs") else "u32",
         "data": "synthetic",
-        "config": {"workload": args.workload, "description": desc, "V": wl.V, "E": wl.E, "algorithm": alg,
-                   "repr": repr_, "vertices_per_shard": st0["vertices_per_shard"], "num_shards": st0["num_shards"],
-                   "iterations": iters[-1], "time_to_convergence_ms": round(total_ms / args.steps, 4),
-                   "l2": f"inputs larger than L2: {per_iter_gb:.3f} GB streamed per fully-active pass vs 0.126 GB L2"
-                   if per_iter_gb * 1e9 > L2_BYTES else f"L2-resident workload ({per_iter_gb*1e3:.1f} MB per pass); no flush",
-                   "build_ms": round(st0["build_ms"], 3),
-                   "skip_clean_shards": bool(args.skip_clean),
-                   "passes": "one launch per pass, device-wide barrier between passes" if steps[-1][6] != 2
-                   else "overlapped passes in one launch (DESIGN.md \"Overlapped passes\")",
-                   "parallelism": f"destination-range partition x{world} (NCCL)" if world > 1 else "1 GPU"},
+        "config": static_config(args.workload, wl, alg, repr_),
+        "run": {"vertices_per_shard": st0["vertices_per_shard"], "num_shards": st0["num_shards"],
+                "iterations": iters[-1], "time_to_convergence_ms": round(total_ms / args.steps, 4),
+                "build_ms": round(st0["build_ms"], 3), "skip_clean_shards": bool(args.skip_clean),
+                "passes": "one launch per pass, device-wide barrier between passes" if not overlapped
+                else "overlapped passes in one launch (DESIGN.md \"Overlapped passes\")",
+                "parallelism": (f"destination-range partition x{world}: stage-4 stores over NVLink (CUDA IPC), "
+                                "NCCL all-reduce of the convergence word") if world > 1 else
+                               (f"1 GPU, {local_parts} simulated partitions" if local_parts > 1 else "1 GPU"),
+                "partitions": st0["partitions"], "device_bytes_per_gpu": st0["max_part_device_bytes"]},
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                      "frac": round(achieved / peak, 4),
-                     "traffic": traffic_for(args.workload, overlapped, sum(iters) / len(iters)) if world == 1 else None,
+                     "traffic": traffic, "traffic_source": traffic_src,
                      "launch": "one shard_pass launch per run (overlapped passes)" if overlapped
                      else "one shard_pass launch per pass",
                      "passes_per_step": round(sum(iters) / len(iters), 2),
                      "avg_pass_us": round(loop_ms / max(sum(iters), 1) * 1e3, 3),
                      "kernel": f"shard_pass<{alg},{repr_}>", "peak_kind": peak_kind,
-                     "algorithmic_bytes_per_launch": int(alg_bytes / max(n_pass_launches, 1)),
-                     "avg_launch_us": round(loop_ms / max(n_pass_launches, 1) * 1e3, 3)},
+                     "bytes": "compressed layout actually streamed (u16 indices, pre-divided PR, window-form Mapper; "
+                              "DESIGN.md §7)",
+                     "algorithmic_bytes_per_launch": int(alg_bytes / world / max(n_pass_launches, 1)),
+                     "avg_launch_us": round(loop_ms / max(n_pass_launches, 1) * 1e3, 3),
+                     "paper_layout": {"bytes": "SURVEY §8(d) per-unit figures (4-byte fields: stage 2 12 B/edge for PR, "
+                                               "stage 4 12 B per active CW edge, 8 B/vertex); not physical here",
+                                      "algorithmic_bytes_per_launch": int(paper_bytes / world / max(n_pass_launches, 1)),
+                                      "achieved": round(achieved_paper, 1),
+                                      "frac": round(achieved_paper / peak, 4)}},
         "clocks": clocks,
         "gpu_launches": launches,
         "e2e": e2e,
@@ -391,6 +456,28 @@ def bench_cusha(args):
         dist.barrier()
         dist.destroy_process_group()
     return 0
+
+
+def relaunch_under_torchrun(args) -> int:
+    """`python bench.py --gpus N` (N > 1) without torchrun: start N ranks on
+    this node (the contract's launch line), or refuse when fewer GPUs exist."""
+    import socket
+    import torch
+    have = torch.cuda.device_count()
+    if have < args.gpus:
+        log(f"[bench] --gpus {args.gpus} but only {have} CUDA device(s) visible; refusing to report a "
+            f"{args.gpus}-GPU number")
+        return 2
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")          # NCCL's init log (rank count) stays visible
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    log("[bench] launching " + " ".join(cmd[2:7]))
+    return subprocess.call(cmd, env=env)
 
 
 def main():
@@ -412,9 +499,20 @@ def main():
                     help="one launch per pass with a device-wide barrier between passes (Fig. 5) instead of "
                          "the default overlapped passes")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--sim-parts", type=int, default=1,
+                    help="one process: simulate this many destination-range partitions on one GPU (tools/tests)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     args = ap.parse_args()
+    world = int(os.environ.get("WORLD_SIZE", "0"))
+    if world and world != args.gpus:
+        log(f"[bench] WORLD_SIZE={world} but --gpus {args.gpus}")
+        return 2
+    if args.gpus > 1 and not world and args.impl == "cusha":
+        return relaunch_under_torchrun(args)
+    if world > 1:
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
     if args.warmup < 3 and args.impl == "cusha":
         log("[bench] warmup raised to 3 (timing rules)")
         args.warmup = 3

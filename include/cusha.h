@@ -25,6 +25,15 @@
  *    graph must not be used concurrently.
  *  - Limits: |V| < 2^31, |E| < 2^32 - 2^26 (offsets are 32-bit), and
  *    vertices_per_shard <= 65534 (16-bit local indices).
+ *  - Fixed-point range (PR, NN, HS, CS): stage 2 sums the per-edge terms of
+ *    Table 3 as 64-bit fixed point with 32 fraction bits (order-independent,
+ *    DESIGN.md R11).  Each term is truncated toward zero to a multiple of
+ *    2^-32 (so a vertex's sum is within in-degree * 2^-32 of the exact sum of
+ *    its f32 terms) and every sum must stay below 2^31 in magnitude.  PR meets
+ *    this by construction (the ranks sum to at most |V| < 2^31 at every pass);
+ *    for NN / HS / CS cusha_run returns CUSHA_EINVAL when max|initial value| x
+ *    max|edge value| x max in-degree (NN: max(|x0|, 1) * |w|; HS: 2 |Q0| |c|;
+ *    CS: max(|V0|, 1) * max(|G|, 1)) reaches 2^31 or is not finite.
  */
 #ifndef CUSHA_H
 #define CUSHA_H
@@ -42,7 +51,7 @@ extern "C" {
 #define CUSHA_API
 #endif
 
-#define CUSHA_ABI_VERSION 3
+#define CUSHA_ABI_VERSION 4
 
 /* Return codes. */
 enum {
@@ -81,24 +90,38 @@ typedef struct {
   int device;                      /* CUDA device ordinal                                      */
   void* stream;                    /* cudaStream_t to run on; NULL = a library-owned stream    */
   cusha_input_location input_location; /* host (copied in, timed as H2D) or device            */
-  int host_loop;                   /* 0 = loop on the device (CUDA-graph while node, default);
-                                      1 = host launches passes in chunks of 8 (for profilers that
-                                      cannot see kernels inside conditional graphs); passes past
-                                      convergence exit at once, so results are identical      */
+  int host_loop;                   /* 0 = loop on the device (default);
+                                      1 = host launches passes in chunks of 16 (one launch per
+                                      pass, for profilers); passes past convergence exit at once,
+                                      so results are identical                                */
   /* Destination-range partition (row e; north_star (4)).  With
    * world_size = G > 1 the shards are split into G contiguous ranges of
    * near-equal work (cusha_partition_shards); partition r owns the vertices
    * of its shards.  Within a partition the pass is asynchronous (L45); across
-   * partitions it is BSP: after each pass every partition's write-back values
-   * are exchanged and the windows fed by other partitions are refreshed.
-   * CW representation only.
+   * partitions it is BSP: every pass of every partition ends before the next
+   * pass starts anywhere.  Each partition keeps only its own shards (the
+   * in-edges of its vertices) and the Concatenated Windows of its own source
+   * shards; stage 4 of a source shard stores each window's new SrcValues
+   * directly into the SrcValue array of the partition that owns the window
+   * (the windows aimed at one partition are one contiguous segment of CW_i,
+   * L175).  Only shards that committed an update write back (Fig. 5 line 23),
+   * and the integer algorithms store only changed vertices, so the exchange is
+   * exactly the changed values, overlapped with the other shards' work.
+   * After each pass the partitions' "committed an update" words are OR-ed:
+   * the global convergence test of L189.  CW representation only; no
+   * host-streamed topology.
    *   nccl_unique_id != NULL: one process per GPU; every rank passes the full
    *     edge list, its rank and the same 128-byte ncclUniqueId
-   *     (cusha_nccl_unique_id on rank 0, broadcast by the caller); the
-   *     exchange is NCCL broadcasts over NVLink.
+   *     (cusha_nccl_unique_id on rank 0, broadcast by the caller).  The ranks
+   *     map each other's SrcValue arrays with CUDA IPC (handles exchanged by
+   *     an NCCL all-gather during this call), so stage-4 stores travel over
+   *     NVLink / NVSwitch; the per-pass OR is an NCCL all-reduce.  Every rank
+   *     must make the same sequence of calls (build, run, get_values).
    *   nccl_unique_id == NULL: all G partitions run in this process on one
-   *     device and exchange through device memory (the same kernels; used to
-   *     test the partitioned algorithm on one GPU).                            */
+   *     device (each partition with its own arrays, the same kernels and the
+   *     same stores into the sibling partitions' SrcValue; the OR is a kernel
+   *     over the partitions' words).  Used to test the partitioned algorithm
+   *     on one GPU.                                                            */
   int world_size;                  /* 1 = single partition (0 is treated as 1)                  */
   int rank;                        /* this process's rank, 0..world_size-1 (NCCL mode)          */
   const void* nccl_unique_id;      /* 128-byte ncclUniqueId, or NULL (see above)                */
@@ -137,8 +160,13 @@ typedef struct {
    *      the per-ticket costs of overlapped passes outweigh the barrier they
    *      save and the run uses 1 (measured).
    * host_loop = 1 or world_size > 1 imply one launch per pass.  Other values:
-   * CUSHA_EINVAL.                                                          */
+   * CUSHA_EINVAL.  One launch per pass is a fixed-count CUDA graph of 16
+   * passes per host check (passes past convergence exit at once).        */
   int pass_barrier;
+  /* 1 = keep arrays that only layout inspection (cusha_get_layout) reads:
+   * the input edge index of every shard entry and, for CW, the window
+   * table.  0 (default) = release them after the build.                    */
+  int keep_layout;
 } cusha_build_opts;
 
 typedef struct cusha_graph cusha_graph;   /* opaque; owns all device memory it allocates */
@@ -172,6 +200,16 @@ typedef struct {
   uint32_t host_shard;             /* first shard whose topology is host-resident (|S|: none)   */
   uint32_t mapper_form;            /* last run, CW: 1 = stage 4 used the Mapper in window form
                                       (u16 window index per entry + per-shard delta row), 0 = u32 Mapper */
+  uint64_t paper_bytes;            /* last run: algorithmic bytes in the paper's layout (4-byte
+                                      fields: stage 2 8/12/16 B per edge, stage 4
+                                      CW 12 / GS 8 B (+4 for 8-byte Vertex) per active edge,
+                                      2 x sizeof(Vertex) per vertex)                            */
+  uint64_t wb_entries;             /* last run: stage-4 entries visited (active shards' windows) */
+  uint64_t vertices_processed;     /* last run: vertices of the processed shards, over all passes */
+  uint64_t updated_total;          /* last run: committed updates, over all passes               */
+  uint32_t partitions;             /* partitions of the graph (row e); 1 = unpartitioned         */
+  uint32_t max_in_degree;          /* largest in-degree (fixed-point range check)                */
+  uint64_t max_part_device_bytes;  /* the largest partition's device_bytes (= device_bytes at 1)  */
 } cusha_stats;
 
 /* ---------------------------------------------------------------- build */
@@ -216,8 +254,8 @@ CUSHA_API int cusha_set_vertex_values(cusha_graph* g, cusha_algorithm alg, const
  * pass (Fig. 5) until a pass commits no update (L189) or max_iters passes ran.
  *   source     BFS/SSSP/SSWP start vertex (< |V|); ignored by the others.
  *   max_iters  upper bound on shard passes (R23); 0 = do nothing.
- * The iteration loop runs on the device (one CUDA-graph launch with a
- * conditional while node); the host waits once at the end.
+ * The iteration loop runs on the device (one launch of overlapped passes by
+ * default); the host waits once at the end.
  * Returns CUSHA_OK, CUSHA_NOT_CONVERGED, or CUSHA_EINVAL (bad source, NN/HS/CS
  * without initial values, EdgeValue needed but absent) / CUSHA_ECUDA.
  */
@@ -261,16 +299,37 @@ typedef enum {
   CUSHA_LAYOUT_CW_SRC_LOCAL = 8,    /* u16[Q]     SrcIndex - i*|N| per padded CW entry      */
   CUSHA_LAYOUT_MAPPER = 9,          /* u32[Q]     padded shard position (filler = trash P)  */
   CUSHA_LAYOUT_OUT_DEGREE = 10,     /* u32[|V|]   out-degree (PR NbrsNum, L318)            */
-  CUSHA_LAYOUT_RUN_K = 11,          /* u32[R]     CW position of each Mapper run's first entry (CW) */
+  CUSHA_LAYOUT_RUN_K = 11,          /* u32[R]     CW position of each Mapper run's first entry (CUSHA_RLE builds) */
   CUSHA_LAYOUT_RUN_T = 12,          /* u32[R]     its Mapper target; one run per non-empty W_ij      */
   CUSHA_LAYOUT_CW_WINDOW = 13,      /* u16[Q]     j of the window W_ij holding each CW_i entry (filler 0xFFFF) */
-  CUSHA_LAYOUT_CW_DELTA = 14        /* u32[|S|*|S|] Mapper in window form: Mapper[k] = delta[i*|S|+j] + k
+  CUSHA_LAYOUT_CW_DELTA = 14,       /* u32[|S|*|S|] Mapper in window form: Mapper[k] = delta[i*|S|+j] + k
                                                   (mod 2^32) for every real entry k of CW_i in W_ij  */
+  CUSHA_LAYOUT_CW_PARTITION_OFFSETS = 15 /* partitioned only: u32[Sl*(G+1)]: CW_i's entries aimed at
+                                                  partition q are [p[il*(G+1)+q], p[il*(G+1)+q+1])   */
 } cusha_layout_part;
 /* Returns the element count of `part` in *count (bytes = count * element size);
  * copies it to `out` (host) when out != NULL and out_bytes is large enough.
- * Parts not held by the representation return CUSHA_EUNSUPPORTED.          */
+ * Parts not held by the representation (or released after the build, see
+ * keep_layout) return CUSHA_EUNSUPPORTED.  Unpartitioned graphs only.      */
 CUSHA_API int cusha_get_layout(const cusha_graph* g, cusha_layout_part part, void* out, size_t out_bytes, uint64_t* count);
+
+/* The same for partition `p` of a partitioned graph (row e): p < G in the
+ * one-process simulation, p = 0 (this rank's) with one process per GPU.
+ * Sizes are the partition's: Sl = its shards, positions local to it; the
+ * Mapper holds positions in the OWNING partition's SrcValue; OUT_DEGREE and
+ * the window rows cover its own vertices / source shards.                  */
+CUSHA_API int cusha_get_part_layout(const cusha_graph* g, uint32_t p, cusha_layout_part part, void* out,
+                                    size_t out_bytes, uint64_t* count);
+
+/* Statistics of partition p (as cusha_get_stats, with device_bytes,
+ * entries_padded and the last run's byte / edge counts of that partition). */
+CUSHA_API int cusha_get_part_stats(const cusha_graph* g, uint32_t p, cusha_stats* s);
+
+/* Return the unused blocks of the library's private device-memory pool on
+ * `device` to the driver.  Freed graphs keep their memory in that pool (so
+ * repeated builds do not map HBM again); it is never shared with torch or
+ * NCCL.  Errors: CUSHA_ECUDA.                                              */
+CUSHA_API int cusha_trim_memory(int device);
 
 /* Diagnostic timeline (tools/timeline.py): only a library built with
  * -DCUSHA_TIMELINE=1 records it; the product build returns CUSHA_EUNSUPPORTED.

@@ -1,24 +1,21 @@
 // api.cu — the C ABI of include/cusha.h (row b) and the iteration driver (row a5).
 //
 // cusha_run replaces the paper's host loop (Fig. 5 lines 0-2 and 29; L189:
-// launch, cudaMemcpy(is_converged), decide) by ONE launch of a CUDA graph
-// whose body is the shard pass under a conditional while node; the shard
-// pass's last CTA decides whether the loop goes on (DESIGN.md "Iteration
-// control").  The host waits once, at the end.
+// launch, cudaMemcpy(is_converged), decide).  On one GPU the default is ONE
+// launch for the whole run (overlapped passes, kernels.cu); the per-pass mode
+// launches a fixed-count CUDA graph of passes and checks the device-resident
+// convergence flag once per graph.  A destination-range partitioned graph
+// (row e) runs one pass per partition, then decides global convergence from
+// every partition's "committed an update" word (NCCL all-reduce across GPUs,
+// or directly in the one-process simulation).
 #include <algorithm>
-#include <chrono>
 #include <cmath>
 #include <cstring>
 #include <string>
+#include <vector>
 
 #include "algorithms.cuh"
 #include "graph.hpp"
-
-struct cusha_graph {
-  cusha::Graph g;
-  cudaGraphExec_t exec[cusha::kNumAlgs] = {};
-  bool exec_failed[cusha::kNumAlgs] = {};
-};
 
 namespace cusha {
 
@@ -39,53 +36,149 @@ static int fail(int code, const std::string& msg) {
     }                                                                                              \
   } while (0)
 
-static void free_graph_memory(Graph& g) {
-  void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcloc, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
-                  g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_srcvalue, g.d_vv, g.d_ctl, g.d_trace,
-                  g.d_active, g.d_bounds, g.d_owner, g.d_cwp, g.d_gathered, g.d_run_k, g.d_run_t,
-                  g.d_run_unit, g.d_run_bits, g.d_run_d, g.d_dirty, g.d_shard_seq, g.d_cw_win, g.d_cw_delta};
-  nccl_destroy(g);
-  // device memory is stream-ordered (cudaMallocAsync on g.stream): released to
-  // the retained pool without unmapping or a device-wide synchronisation
-  for (void* p : ptrs)
-    if (p) cudaFreeAsync(p, g.stream);
-  for (void*& p : g.d_init)
-    if (p) { cudaFreeAsync(p, g.stream); p = nullptr; }
-  void* hosts[] = {g.h_dest, g.h_ev, g.h_srcloc, g.h_eid, g.h_cw_src, g.h_mapper, g.h_cw_win};
-  for (void* p : hosts)
-    if (p) cudaFreeHost(p);
-  delete g.h_ctl;
-  g.h_ctl = nullptr;
-  if (g.ev0) cudaEventDestroy(g.ev0);
-  if (g.ev1) cudaEventDestroy(g.ev1);
-  if (g.evm) cudaEventDestroy(g.evm);
-  if (g.own_stream && g.stream) {
-    cudaStreamSynchronize(g.stream);
-    cudaStreamDestroy(g.stream);
-  }
-}
+constexpr int kModeSingle = 0, kModeSim = 1, kModeNccl = 2;
+constexpr int kChunk = 16;  // passes per fixed-count graph / per host check (per-pass modes)
 
-// Keep freed device memory in the default pool so that repeated builds (the
-// e2e path) reuse it instead of mapping HBM again.
-static void retain_pool(int device) {
-  cudaMemPool_t pool;
-  if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
-    uint64_t keep = UINT64_MAX;
-    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
-  }
-}
+}  // namespace cusha
+
+// The handle: one partition on a single GPU or per rank (NCCL), or all G
+// partitions of the one-process simulation (same kernels and layout as the
+// per-rank mode; the "peer" SrcValue arrays are the sibling partitions').
+struct cusha_graph {
+  int mode = cusha::kModeSingle;
+  std::vector<cusha::Graph*> parts;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  int device = 0;
+  cudaGraphExec_t exec[cusha::kNumAlgs] = {};  // per-pass mode: kChunk passes per graph (single partition)
+  cusha::Ctl** d_ctls = nullptr;                // partitioned: device array of the partitions' Ctl (sim) / own (NCCL)
+  cusha_stats st{};
+  int last_alg = -1;
+  bool have_values = false;
+};
+
+namespace cusha {
 
 static uint64_t device_bytes(const Graph& g) {
-  uint64_t b = 4ull * (g.S + 1) * 2 + 4ull * g.S * 2;  // offsets + counts
-  b += 2 * g.P + 4 * g.P;                               // dest + eid
+  uint64_t b = 4ull * (g.Sl + 1) * 2 + 4ull * g.Sl * 2;  // shard / CW offsets + counts
+  // per-entry arrays count whole; their host-streamed tails (row f3) are subtracted below
+  b += 2 * g.P;                                          // DestIndex
+  if (g.d_eid || g.h_eid) b += 4 * g.P;
   if (g.has_ev) b += 4 * g.P;
-  if (g.d_srcloc) b += 2 * g.P;
-  if (g.d_win) b += 4ull * (g.S + 1) * g.S;
-  b += (2 + 4 + 2) * g.Q;                               // CW: SrcIndexCW, Mapper, window
-  if (g.d_cw_delta) b += 4ull * g.S * g.S;             // Mapper deltas per window
-  b += 4ull * g.V;                                      // outdeg
-  b += 4 * (g.P + 1) + 8ull * g.V;                      // SrcValue + VertexValues
-  return b - g.host_bytes;                              // minus the host-streamed part (row f3)
+  if (g.d_srcloc || g.h_srcloc) b += 2 * g.P;
+  if (g.d_win) b += 4ull * (g.Sl + 1) * g.S;
+  if (g.d_cw_src || g.h_cw_src) b += 2 * g.Q;
+  if (g.d_mapper || g.h_mapper) b += 4 * g.Q;
+  if (g.d_cw_win || g.h_cw_win) b += 2 * g.Q;
+  if (g.d_cw_delta) b += 4ull * g.Sl * g.S;
+  if (g.d_cwp) b += 4ull * g.Sl * (g.G + 1) + g.S;
+  b += 4ull * g.nvl;                                     // out-degrees
+  b += 4 * (g.P + 1) + 8ull * g.nvl;                     // SrcValue + VertexValues
+  return b - g.host_bytes;                               // minus the host-streamed part (row f3)
+}
+
+static void free_handle(cusha_graph* h) {
+  if (!h) return;
+  cudaSetDevice(h->device);
+  for (auto& e : h->exec)
+    if (e) cudaGraphExecDestroy(e);
+  for (Graph* g : h->parts) {
+    free_device_arrays(*g);
+    nccl_destroy(*g);
+    delete g->h_ctl;
+    delete g;
+  }
+  h->parts.clear();
+  if (h->d_ctls) cudaFreeAsync(h->d_ctls, h->stream);
+  if (h->own_stream && h->stream) {
+    cudaStreamSynchronize(h->stream);
+    cudaStreamDestroy(h->stream);
+  } else if (h->stream) {
+    cudaStreamSynchronize(h->stream);
+  }
+  delete h;
+}
+
+static Graph& g0(cusha_graph* h) { return *h->parts[0]; }
+static const Graph& g0(const cusha_graph* h) { return *h->parts[0]; }
+
+// Per-run arrays of a partition: SrcValue (P entries + 1), VertexValues
+// (8 B per owned vertex covers every Table-3 Vertex), the control block.
+// With one process per GPU, SrcValue and dirty[] are cudaMalloc'ed so the
+// other ranks can map them (CUDA IPC) and store into them over NVLink.
+static int alloc_run_state(Graph& g, bool ipc) {
+  g.srcvalue_ipc = ipc;
+  if (ipc) {
+    CKA(cudaMalloc(&g.d_srcvalue, 4 * (g.P + 1)));
+    if (g.skip_clean) {
+      if (g.d_dirty) cudaFreeAsync(g.d_dirty, g.stream);
+      g.d_dirty = nullptr;
+      CKA(cudaMalloc(&g.d_dirty, 4ull * std::max<uint32_t>(g.Sl, 1)));
+    }
+  } else {
+    CKA(dev_alloc((void**)&g.d_srcvalue, 4 * (g.P + 1), g.stream));
+  }
+  CKA(cudaMemsetAsync(g.d_srcvalue, 0, 4 * (g.P + 1), g.stream));
+  CKA(dev_alloc(&g.d_vv, 8ull * std::max<uint32_t>(g.nvl, 1), g.stream));
+  CKA(dev_alloc((void**)&g.d_ctl, sizeof(Ctl), g.stream));
+  CKA(cudaMemsetAsync(g.d_ctl, 0, sizeof(Ctl), g.stream));
+  g.h_ctl = new (std::nothrow) Ctl();
+  if (!g.h_ctl) return fail(CUSHA_ENOMEM, "host allocation");
+  return CUSHA_OK;
+}
+
+// Peer tables of the partitioned mode: SrcValue (and dirty[]) of every
+// partition, as device pointers valid on this device.
+static int set_peer_tables(Graph& g, const std::vector<uint32_t*>& sv, const std::vector<uint32_t*>& dirty) {
+  CKA(dev_alloc((void**)&g.d_sv_peer, sizeof(uint32_t*) * g.G, g.stream));
+  CKA(cudaMemcpyAsync(g.d_sv_peer, sv.data(), sizeof(uint32_t*) * g.G, cudaMemcpyHostToDevice, g.stream));
+  if (g.skip_clean) {
+    CKA(dev_alloc((void**)&g.d_dirty_peer, sizeof(uint32_t*) * g.G, g.stream));
+    CKA(cudaMemcpyAsync(g.d_dirty_peer, dirty.data(), sizeof(uint32_t*) * g.G, cudaMemcpyHostToDevice, g.stream));
+  }
+  CKA(cudaStreamSynchronize(g.stream));  // the host vectors go out of scope
+  return CUSHA_OK;
+}
+
+// One process per GPU: exchange the CUDA IPC handles of every rank's SrcValue
+// and dirty[] over NCCL (all-gather of 64-byte handles) and map the peers'.
+static int connect_ipc_peers(Graph& g) {
+  const uint32_t G = g.G;
+  cudaIpcMemHandle_t mine[2];
+  std::memset(mine, 0, sizeof(mine));
+  CKA(cudaIpcGetMemHandle(&mine[0], g.d_srcvalue));
+  if (g.skip_clean) CKA(cudaIpcGetMemHandle(&mine[1], g.d_dirty));
+  void* dsend = nullptr;
+  void* drecv = nullptr;
+  CKA(dev_alloc(&dsend, sizeof(mine), g.stream));
+  CKA(dev_alloc(&drecv, sizeof(mine) * G, g.stream));
+  CKA(cudaMemcpyAsync(dsend, mine, sizeof(mine), cudaMemcpyHostToDevice, g.stream));
+  std::string err;
+  const int rc = nccl_allgather_bytes(g, dsend, drecv, sizeof(mine), err);
+  if (rc) return fail(rc, "IPC handle exchange: " + err);
+  std::vector<cudaIpcMemHandle_t> all(2 * G);
+  CKA(cudaMemcpyAsync(all.data(), drecv, sizeof(mine) * G, cudaMemcpyDeviceToHost, g.stream));
+  CKA(cudaStreamSynchronize(g.stream));
+  cudaFreeAsync(dsend, g.stream);
+  cudaFreeAsync(drecv, g.stream);
+  std::vector<uint32_t*> sv(G), dirty(G, nullptr);
+  for (uint32_t q = 0; q < G; ++q) {
+    if (q == g.part) {
+      sv[q] = g.d_srcvalue;
+      dirty[q] = g.d_dirty;
+      continue;
+    }
+    void* p = nullptr;
+    CKA(cudaIpcOpenMemHandle(&p, all[2 * q], cudaIpcMemLazyEnablePeerAccess));
+    g.ipc_open.push_back(p);
+    sv[q] = static_cast<uint32_t*>(p);
+    if (g.skip_clean) {
+      CKA(cudaIpcOpenMemHandle(&p, all[2 * q + 1], cudaIpcMemLazyEnablePeerAccess));
+      g.ipc_open.push_back(p);
+      dirty[q] = static_cast<uint32_t*>(p);
+    }
+  }
+  return set_peer_tables(g, sv, dirty);
 }
 
 }  // namespace cusha
@@ -146,28 +239,22 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
     return fail(CUSHA_EUNSUPPORTED, "the partitioned (multi-GPU) mode uses the CW representation");
   if (o.world_size > 1 && o.nccl_unique_id && (o.rank < 0 || o.rank >= o.world_size))
     return fail(CUSHA_EINVAL, "rank out of range");
+  if (o.world_size > 1 && o.device_topology_budget)
+    return fail(CUSHA_EUNSUPPORTED, "host-streamed topology is for a single partition (row f3)");
   uint32_t N = o.vertices_per_shard ? o.vertices_per_shard : cusha_shard_size(V, E, o.smem_bytes_per_vertex, 0, 0);
   if (N > 65534) return fail(CUSHA_EINVAL, "vertices_per_shard must be <= 65534");
   if (o.pass_barrier < 0 || o.pass_barrier > 2) return fail(CUSHA_EINVAL, "pass_barrier must be 0, 1 or 2");
   if (N > V) N = V;
+  const uint32_t S = (V + N - 1) / N;
+  const int mode = o.world_size == 1 ? kModeSingle : (o.nccl_unique_id ? kModeNccl : kModeSim);
+  const uint32_t G = std::min<uint32_t>((uint32_t)o.world_size, S);  // never more partitions than shards
+  if (mode == kModeNccl && G != (uint32_t)o.world_size) return fail(CUSHA_EINVAL, "world_size exceeds the number of shards");
 
   cusha_graph* h = new (std::nothrow) cusha_graph();
   if (!h) return fail(CUSHA_ENOMEM, "host allocation");
-  Graph& g = h->g;
-  g.V = V; g.E = E; g.N = N; g.S = (V + N - 1) / N; g.repr = (int)o.repr; g.device = o.device;
-  g.host_loop = o.host_loop != 0;
-  g.skip_clean = o.skip_clean_shards != 0;
-  g.pass_barrier = o.pass_barrier;
-  g.topo_budget = o.device_topology_budget;
-  g.world_size = o.world_size;
-  g.rank = o.world_size > 1 && o.nccl_unique_id ? o.rank : 0;
-  g.simulate = o.world_size > 1 && !o.nccl_unique_id;
-  g.G = std::min<uint32_t>((uint32_t)o.world_size, g.S);  // never more partitions than shards
-  if (!g.simulate && g.G != (uint32_t)o.world_size) {
-    delete h;
-    return fail(CUSHA_EINVAL, "world_size exceeds the number of shards");
-  }
-  auto bail = [&](int code) { free_graph_memory(g); delete h; return code; };
+  h->mode = G > 1 ? mode : kModeSingle;
+  h->device = o.device;
+  auto bail = [&](int code) { free_handle(h); return code; };
   auto cu = [&](cudaError_t e, const char* what) -> int {
     if (e == cudaSuccess) return 0;
     set_error(std::string(what) + ": " + cudaGetErrorString(e));
@@ -175,133 +262,219 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   };
   int rc;
   if ((rc = cu(cudaSetDevice(o.device), "cudaSetDevice"))) return bail(rc);
-  retain_pool(o.device);
   if (o.stream) {
-    g.stream = (cudaStream_t)o.stream;
+    h->stream = (cudaStream_t)o.stream;
   } else {
-    if ((rc = cu(cudaStreamCreateWithFlags(&g.stream, cudaStreamNonBlocking), "cudaStreamCreate"))) return bail(rc);
-    g.own_stream = true;
+    if ((rc = cu(cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking), "cudaStreamCreate"))) return bail(rc);
+    h->own_stream = true;
   }
-  if ((rc = cu(cudaEventCreate(&g.ev0), "cudaEventCreate")) || (rc = cu(cudaEventCreate(&g.ev1), "cudaEventCreate")) ||
-      (rc = cu(cudaEventCreate(&g.evm), "cudaEventCreate")))
+  Graph* glob = new (std::nothrow) Graph();
+  if (!glob) return bail(fail(CUSHA_ENOMEM, "host allocation"));
+  h->parts.push_back(glob);  // freed with the handle on any failure
+  Graph& g = *glob;
+  g.V = V; g.E = E; g.N = N; g.S = S; g.repr = (int)o.repr; g.device = o.device; g.stream = h->stream;
+  g.host_loop = o.host_loop != 0;
+  g.skip_clean = o.skip_clean_shards != 0;
+  g.pass_barrier = o.pass_barrier;
+  g.topo_budget = o.device_topology_budget;
+  g.keep_ids = o.keep_layout != 0;
+  g.world_size = o.world_size;
+  g.rank = mode == kModeNccl ? o.rank : 0;
+  cudaEvent_t e0 = nullptr, eh = nullptr, e1 = nullptr;
+  if ((rc = cu(cudaEventCreate(&e0), "cudaEventCreate")) || (rc = cu(cudaEventCreate(&eh), "cudaEventCreate")) ||
+      (rc = cu(cudaEventCreate(&e1), "cudaEventCreate")))
     return bail(rc);
-  cudaEvent_t eh = nullptr;
-  if ((rc = cu(cudaEventCreate(&eh), "cudaEventCreate"))) return bail(rc);
+  struct EvGuard {
+    cudaEvent_t a, b, c;
+    ~EvGuard() { cudaEventDestroy(a); cudaEventDestroy(b); cudaEventDestroy(c); }
+  } evg{e0, eh, e1};
 
-  auto t0 = std::chrono::steady_clock::now();
-  CKA(cudaEventRecord(g.ev0, g.stream));
+  CKA(cudaEventRecord(e0, h->stream));
   const uint32_t *d_src = src, *d_dst = dst, *d_val = edge_values;
-  uint32_t* tmp = nullptr;
+  void* tmp = nullptr;
   uint64_t h2d = 0;
   if (o.input_location == CUSHA_INPUT_HOST && E) {
     const uint64_t nvals = edge_values ? 3 : 2;
-    if ((rc = cu(cudaMallocAsync(&tmp, nvals * E * 4, g.stream), "cudaMallocAsync(inputs)"))) {
-      cudaEventDestroy(eh);
+    if ((rc = cu(dev_alloc(&tmp, nvals * E * 4, h->stream), "cudaMallocAsync(inputs)"))) return bail(rc);
+    uint32_t* t = static_cast<uint32_t*>(tmp);
+    if ((rc = cu(cudaMemcpyAsync(t, src, E * 4, cudaMemcpyHostToDevice, h->stream), "H2D src")) ||
+        (rc = cu(cudaMemcpyAsync(t + E, dst, E * 4, cudaMemcpyHostToDevice, h->stream), "H2D dst")) ||
+        (edge_values &&
+         (rc = cu(cudaMemcpyAsync(t + 2 * E, edge_values, E * 4, cudaMemcpyHostToDevice, h->stream), "H2D values")))) {
+      cudaFreeAsync(tmp, h->stream);
       return bail(rc);
     }
-    cudaMemcpyAsync(tmp, src, E * 4, cudaMemcpyHostToDevice, g.stream);
-    cudaMemcpyAsync(tmp + E, dst, E * 4, cudaMemcpyHostToDevice, g.stream);
-    if (edge_values) cudaMemcpyAsync(tmp + 2 * E, edge_values, E * 4, cudaMemcpyHostToDevice, g.stream);
-    d_src = tmp; d_dst = tmp + E; d_val = edge_values ? tmp + 2 * E : nullptr;
+    d_src = t; d_dst = t + E; d_val = edge_values ? t + 2 * E : nullptr;
     h2d = nvals * E * 4;
   }
-  cudaEventRecord(eh, g.stream);
+  CKA(cudaEventRecord(eh, h->stream));
   std::string err;
   rc = build_layout(g, d_src, d_dst, d_val, err);
+  if (tmp) cudaFreeAsync(tmp, h->stream);
   if (rc) {
-    if (tmp) cudaFreeAsync(tmp, g.stream);
-    cudaEventDestroy(eh);
     set_error("build: " + err);
     return bail(rc);
   }
-  if (tmp) cudaFreeAsync(tmp, g.stream);
-  if (g.G > 1) {  // destination-range partition (row e)
-    rc = build_partition(g, err);
-    if (!rc && !g.simulate) rc = nccl_init(g, o.nccl_unique_id, err);
+  if (h->mode == kModeSingle) {
+    // CW reads no window table after the build (unless skipping clean shards or inspecting the layout)
+    if (g.repr == CUSHA_REPR_CW && !g.skip_clean && !g.keep_ids && g.d_win) {
+      cudaFreeAsync(g.d_win, h->stream);
+      g.d_win = nullptr;
+    }
+    g.h_bounds = {0u, S};
+    rc = offload_topology(g, err);  // row f3 (no-op without a budget)
     if (rc) {
-      cudaEventDestroy(eh);
+      set_error("host topology: " + err);
+      return bail(rc);
+    }
+    if ((rc = alloc_run_state(g, false))) return bail(rc);
+  } else {
+    // destination-range partition (row e): split by work, then keep per
+    // partition only its shards and the CW of its source shards
+    std::vector<uint64_t> work;
+    if ((rc = partition_work(g, work, err))) {
       set_error("partition: " + err);
       return bail(rc);
     }
+    std::vector<uint32_t> bounds(G + 1);
+    partition_bounds(S, work.data(), G, bounds.data());
+    std::vector<Graph*> parts;
+    const uint32_t r0 = h->mode == kModeNccl ? (uint32_t)o.rank : 0u, r1 = h->mode == kModeNccl ? r0 + 1 : G;
+    for (uint32_t r = r0; r < r1; ++r) {
+      Graph* p = new (std::nothrow) Graph();
+      if (!p) { for (Graph* x : parts) { free_device_arrays(*x); delete x; } return bail(fail(CUSHA_ENOMEM, "host")); }
+      parts.push_back(p);
+      p->device = o.device; p->stream = h->stream; p->skip_clean = g.skip_clean; p->host_loop = true;
+      p->pass_barrier = 1; p->world_size = o.world_size; p->rank = (int)r;
+      if ((rc = build_part(g, bounds, r, *p, h->mode == kModeNccl, err))) {
+        for (Graph* x : parts) { free_device_arrays(*x); delete x; }
+        set_error("partition: " + err);
+        return bail(rc);
+      }
+      if (!p->skip_clean && !p->keep_ids && p->d_win) {  // only the clean-shard marks read the window rows
+        cudaFreeAsync(p->d_win, h->stream);
+        p->d_win = nullptr;
+      }
+    }
+    // the global layout is released; the handle now holds the partitions
+    free_device_arrays(g);
+    delete glob;
+    h->parts = parts;
+    for (Graph* p : h->parts)
+      if ((rc = alloc_run_state(*p, h->mode == kModeNccl))) return bail(rc);
+    if (h->mode == kModeSim) {
+      std::vector<uint32_t*> sv(G), dirty(G);
+      std::vector<Ctl*> ctls(G);
+      for (uint32_t q = 0; q < G; ++q) {
+        sv[q] = h->parts[q]->d_srcvalue;
+        dirty[q] = h->parts[q]->d_dirty;
+        ctls[q] = h->parts[q]->d_ctl;
+      }
+      for (Graph* p : h->parts)
+        if ((rc = set_peer_tables(*p, sv, dirty))) return bail(rc);
+      CKA(dev_alloc((void**)&h->d_ctls, sizeof(Ctl*) * G, h->stream));
+      CKA(cudaMemcpyAsync(h->d_ctls, ctls.data(), sizeof(Ctl*) * G, cudaMemcpyHostToDevice, h->stream));
+      CKA(cudaStreamSynchronize(h->stream));
+    } else {
+      Graph& p = *h->parts[0];
+      if ((rc = nccl_init(p, o.nccl_unique_id, err))) {
+        set_error("NCCL: " + err);
+        return bail(rc);
+      }
+      if ((rc = connect_ipc_peers(p))) return bail(rc);
+      CKA(dev_alloc((void**)&h->d_ctls, sizeof(Ctl*), h->stream));
+      CKA(cudaMemcpyAsync(h->d_ctls, &p.d_ctl, sizeof(Ctl*), cudaMemcpyHostToDevice, h->stream));
+      CKA(cudaStreamSynchronize(h->stream));
+    }
   }
-  rc = offload_topology(g, err);  // row f3 (no-op without a budget)
-  if (rc) {
-    cudaEventDestroy(eh);
-    set_error("host topology: " + err);
-    return bail(rc);
-  }
-  // per-run state: SrcValue (P entries + trash slot), VertexValues (8 B/vertex covers every Table-3 Vertex)
-  g.h_ctl = new (std::nothrow) Ctl();
-  if ((rc = cu(cudaMallocAsync(&g.d_srcvalue, 4 * (g.P + 1), g.stream), "cudaMallocAsync(SrcValue)")) ||
-      (rc = cu(cudaMemsetAsync(g.d_srcvalue, 0, 4 * (g.P + 1), g.stream), "memset")) ||
-      (rc = cu(cudaMallocAsync(&g.d_vv, 8ull * V, g.stream), "cudaMallocAsync(VertexValues)")) ||
-      (rc = cu(cudaMallocAsync(&g.d_ctl, sizeof(Ctl), g.stream), "cudaMallocAsync(ctl)")) ||
-      (rc = g.h_ctl ? 0 : CUSHA_ENOMEM)) {
-    cudaEventDestroy(eh);
-    return bail(rc);
-  }
-  CKA(cudaEventRecord(g.ev1, g.stream));
-  CKA(cudaEventSynchronize(g.ev1));
+  CKA(cudaEventRecord(e1, h->stream));
+  CKA(cudaEventSynchronize(e1));
   float ms = 0, ms_h2d = 0;
-  cudaEventElapsedTime(&ms, g.ev0, g.ev1);
-  cudaEventElapsedTime(&ms_h2d, g.ev0, eh);
-  cudaEventDestroy(eh);
-  (void)t0;
-  g.st.num_vertices = V;
-  g.st.num_edges = E;
-  g.st.vertices_per_shard = N;
-  g.st.num_shards = g.S;
-  g.st.repr = (uint32_t)g.repr;
-  g.st.last_algorithm = -1;
-  g.st.build_ms = ms;
-  g.st.h2d_ms = ms_h2d;
-  g.st.h2d_bytes = h2d;
-  g.st.device_bytes = device_bytes(g);
-  g.st.entries_padded = g.P;
-  g.st.world_size = g.world_size;
-  g.st.rank = g.rank;
-  g.st.host_bytes = g.host_bytes;
-  g.st.host_shard = g.host_shard;
+  cudaEventElapsedTime(&ms, e0, e1);
+  cudaEventElapsedTime(&ms_h2d, e0, eh);
+  cusha_stats& st = h->st;
+  st.num_vertices = V;
+  st.num_edges = E;
+  st.vertices_per_shard = N;
+  st.num_shards = S;
+  st.repr = (uint32_t)o.repr;
+  st.last_algorithm = -1;
+  st.build_ms = ms;
+  st.h2d_ms = ms_h2d;
+  st.h2d_bytes = h2d;
+  st.world_size = o.world_size;
+  st.rank = h->mode == kModeNccl ? o.rank : 0;
+  st.partitions = h->mode == kModeSingle ? 1 : G;
+  st.max_in_degree = g0(h).max_indeg;
+  st.device_bytes = 0;
+  st.max_part_device_bytes = 0;
+  st.entries_padded = 0;
+  for (Graph* p : h->parts) {
+    p->st = cusha_stats{};
+    const uint64_t b = device_bytes(*p);
+    st.device_bytes += b;
+    st.max_part_device_bytes = std::max(st.max_part_device_bytes, b);
+    st.entries_padded += p->P;
+  }
+  st.host_bytes = g0(h).host_bytes;
+  st.host_shard = g0(h).host_shard;
   *out = h;
   set_error("");
   return CUSHA_OK;
 }
 
-void cusha_free_graph(cusha_graph* h) {
-  if (!h) return;
-  cudaSetDevice(h->g.device);
-  for (auto& e : h->exec)
-    if (e) cudaGraphExecDestroy(e);
-  free_graph_memory(h->g);
-  delete h;
+void cusha_free_graph(cusha_graph* h) { free_handle(h); }
+
+int cusha_trim_memory(int device) {
+  CKA(cudaSetDevice(device));
+  CKA(cudaDeviceSynchronize());
+  CKA(trim_pool(device));
+  return CUSHA_OK;
 }
 
 int cusha_set_vertex_values(cusha_graph* h, cusha_algorithm alg, const void* init, size_t bytes) {
   if (!h || !init) return fail(CUSHA_EINVAL, "null argument");
   if ((int)alg < 0 || (int)alg >= kNumAlgs) return fail(CUSHA_EINVAL, "bad algorithm");
-  Graph& g = h->g;
-  const size_t want = (size_t)g.V * value_bytes((int)alg);
+  const uint32_t V = h->st.num_vertices;
+  const size_t vb = value_bytes((int)alg);
+  const size_t want = (size_t)V * vb;
   if (bytes != want) return fail(CUSHA_EINVAL, "bytes must be |V| * value_bytes(alg)");
-  CKA(cudaSetDevice(g.device));
-  if (!g.d_init[alg]) CKA(cudaMallocAsync(&g.d_init[alg], want, g.stream));
-  CKA(cudaMemcpyAsync(g.d_init[alg], init, want, cudaMemcpyHostToDevice, g.stream));
-  CKA(cudaStreamSynchronize(g.stream));
+  // largest |value| of the field stage 2 reads (fixed-point range, include/cusha.h)
+  float mx = 0.f;
+  const float* f = static_cast<const float*>(init);
+  const size_t stride = vb / 4;
+  for (size_t v = 0; v < V; ++v) {
+    const float x = std::fabs(f[v * stride]);
+    if (!(x <= 3.0e38f)) { mx = INFINITY; break; }
+    mx = std::max(mx, x);
+  }
+  CKA(cudaSetDevice(h->device));
+  for (Graph* g : h->parts) {
+    const size_t n = (size_t)g->nvl * vb;
+    if (!g->d_init[alg]) CKA(dev_alloc(&g->d_init[alg], std::max<size_t>(n, 1), h->stream));
+    if (n) CKA(cudaMemcpyAsync(g->d_init[alg], static_cast<const char*>(init) + (size_t)g->v0 * vb, n,
+                               cudaMemcpyHostToDevice, h->stream));
+    g->init_max_abs[alg] = mx;
+  }
+  CKA(cudaStreamSynchronize(h->stream));
   return CUSHA_OK;
 }
 
+}  // extern "C"
+
+namespace cusha {
+
 // Persistent grid of the shard pass: as many CTAs as fit on the device at
-// once (occupancy x SMs), never more than there are shards.
+// once (occupancy x SMs), never more than the partition has shards.
 static uint32_t pass_grid(const Graph& g, const PassKernel& pk, size_t smem) {
-  // shards this process runs: its partition (multi-GPU) or all of them
-  const uint32_t mine = g.G > 1 && !g.simulate ? g.h_bounds[g.rank + 1] - g.h_bounds[g.rank] : g.S;
-  if (!pk.persistent) return std::max<uint32_t>(mine, 1);
+  if (!pk.persistent) return std::max<uint32_t>(g.Sl, 1);
   int sms = 148, per_sm = 1;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g.device);
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, pk.func, (int)pk.threads, smem) != cudaSuccess ||
       per_sm < 1)
     per_sm = 1;
   const uint64_t gsz = (uint64_t)sms * (uint64_t)per_sm;
-  return (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(gsz, mine));
+  return (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(gsz, g.Sl));
 }
 
 // Shared memory of the pass and the CW Mapper form (DESIGN.md "Mapper in
@@ -317,7 +490,12 @@ static uint32_t pass_grid(const Graph& g, const PassKernel& pk, size_t smem) {
 #ifndef CUSHA_STASH
 #define CUSHA_STASH 1  // 0: stage 3 of the integer algorithms re-reads VertexValues (tuning comparison)
 #endif
-static int pass_config(const Graph& g, const PassKernel& pk, size_t* smem, int* mapj, int* stash, uint32_t* nst) {
+struct PassCfg {
+  size_t smem = 0;
+  int mapj = 0, stash = 0;
+  uint32_t nst = 0;
+};
+static int pass_config(const Graph& g, const PassKernel& pk, PassCfg* c) {
   cudaFuncAttributes fa{};
   CKA(cudaFuncGetAttributes(&fa, pk.func));
   const size_t kMaxSmem = 227 * 1024 - fa.sharedSizeBytes;  // dynamic part of the 227 KB per-CTA limit
@@ -326,49 +504,51 @@ static int pass_config(const Graph& g, const PassKernel& pk, size_t* smem, int* 
     return fail(CUSHA_EINVAL, "vertices_per_shard too large for this algorithm's shared-memory state");
   CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem));
   CKA(cudaFuncSetAttribute(pk.func, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared));
-  *smem = sm_m;
-  *mapj = 0;
+  c->smem = sm_m;
+  c->mapj = 0;
   const size_t sm_j = pk.smem_bytes(g.N, g.S);
   // ... and only when the rows cost less traffic than they save: an active
   // shard reads its 4|S|-byte row, so |S| rows per pass (4|S|^2 bytes) against
   // 2 bytes per CW entry (|Q| entries) saved over the u32 Mapper
-  const bool row_pays = 4ull * g.S * g.S <= (uint64_t)g.Q;
+  const bool row_pays = 4ull * g.Sl * g.S <= (uint64_t)g.Q;
   if (CUSHA_MAPJ && row_pays && g.repr == CUSHA_REPR_CW && g.d_cw_win && g.d_cw_delta && !kernels_rle() &&
       g.S <= 0xFFFFu && sm_j <= kMaxSmem) {
     int occ_m = 0, occ_j = 0;
     CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_m, pk.func, (int)pk.threads, sm_m));
     CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_j, pk.func, (int)pk.threads, sm_j));
     if (occ_j >= occ_m && occ_j > 0) {
-      *smem = sm_j;
-      *mapj = 1;
+      c->smem = sm_j;
+      c->mapj = 1;
     }
   }
+  if (g.repr == CUSHA_REPR_CW && !c->mapj && !g.d_mapper && !g.h_mapper)
+    return fail(CUSHA_EUNSUPPORTED, "this graph keeps only the window-form Mapper, whose delta row does not fit");
   // integer algorithms: keep the shard's VertexValues from stage 1 in shared
   // memory for stage 3's update_condition (no second global read) whenever
   // that costs no CTAs per SM
-  *stash = 0;
-  const size_t sm_s = *smem + 4ull * g.N;
+  c->stash = 0;
+  const size_t sm_s = c->smem + 4ull * g.N;
   if (CUSHA_STASH && pk.monotone && sm_s <= kMaxSmem) {
     int occ_0 = 0, occ_s = 0;
-    CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_0, pk.func, (int)pk.threads, *smem));
+    CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_0, pk.func, (int)pk.threads, c->smem));
     CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_s, pk.func, (int)pk.threads, sm_s));
     if (occ_s >= occ_0 && occ_s > 0) {
-      *smem = sm_s;
-      *stash = 1;
+      c->smem = sm_s;
+      c->stash = 1;
     }
   }
   // a deeper TMA ring whenever another slot fits at the same CTAs per SM
   // (more bytes in flight per SM; e.g. C5 at one CTA per SM)
-  *nst = pk.ring_bytes / pk.slot_bytes;
+  c->nst = pk.ring_bytes / pk.slot_bytes;
   if (CUSHA_DEEP_RING) {
     int occ_0 = 0;
-    CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_0, pk.func, (int)pk.threads, *smem));
-    while (*nst < pk.max_stages && *smem + pk.slot_bytes <= kMaxSmem) {
+    CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_0, pk.func, (int)pk.threads, c->smem));
+    while (c->nst < pk.max_stages && c->smem + pk.slot_bytes <= kMaxSmem) {
       int occ_d = 0;
-      CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_d, pk.func, (int)pk.threads, *smem + pk.slot_bytes));
+      CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_d, pk.func, (int)pk.threads, c->smem + pk.slot_bytes));
       if (occ_d < occ_0 || occ_d == 0) break;
-      *smem += pk.slot_bytes;
-      ++*nst;
+      c->smem += pk.slot_bytes;
+      ++c->nst;
     }
   }
   return CUSHA_OK;
@@ -385,339 +565,422 @@ static int pass_ahead(const Graph& g, int alg) {
   return bytes > 2ull * (uint64_t)l2 ? 1 : 0;
 }
 
-#ifndef CUSHA_DIAG_FIXED_GRAPH
-#define CUSHA_DIAG_FIXED_GRAPH 0
-#endif
-#ifndef CUSHA_DIAG_COND_NODE
-#define CUSHA_DIAG_COND_NODE 0
-#endif
-#if CUSHA_DIAG_COND_NODE
-// sanitizer diagnostic only: the while condition set by a one-thread kernel
-// after the pass (the pass runs with use_cond = 0 and closes the iteration)
-__global__ void diag_set_cond(const Ctl* ctl, cudaGraphConditionalHandle h) {
-  const uint32_t more = !*reinterpret_cast<const volatile uint32_t*>(&ctl->converged) && ctl->iter < ctl->max_iters;
-  cudaGraphSetConditional(h, more ? 1u : 0u);
+static KParams pass_params(const Graph& g, uint32_t source, const PassCfg& c, int alg) {
+  KParams kp = make_params(g, source);
+  kp.mapj = c.mapj;
+  kp.stash = c.stash;
+  kp.nst = c.nst;
+  kp.ahead = pass_ahead(g, alg);
+  return kp;
 }
-#endif
-static int ensure_exec(cusha_graph* h, int alg) {
-  Graph& g = h->g;
+
+// Per-pass mode on one partition: a CUDA graph of kChunk pass launches (no
+// conditional node); a pass launched after convergence or max_iters exits at
+// once, so the host launches the graph until the flag says stop.
+static int ensure_exec(cusha_graph* h, int alg, const PassKernel& pk, const PassCfg& c) {
   if (h->exec[alg]) return CUSHA_OK;
-  const PassKernel& pk = pass_kernel(alg, g.repr);
-  size_t smem = 0;
-  int mapj = 0, stash = 0;
-  uint32_t nst = 0;
-  const int prc = pass_config(g, pk, &smem, &mapj, &stash, &nst);
-  if (prc) return prc;
+  Graph& g = g0(h);
   cudaGraph_t graph = nullptr;
   CKA(cudaGraphCreate(&graph, 0));
-#if CUSHA_DIAG_FIXED_GRAPH
-  // sanitizer diagnostic only (profiles/r1/sanitizer/README.md): a chain of
-  // CUSHA_DIAG_FIXED_GRAPH per-pass launches without the conditional node; a
-  // pass launched after convergence is a no-op, as in the host loop
-  {
-    KParams kp = make_params(g, 0);
-    kp.mapj = mapj;
-    kp.stash = stash;
-    kp.nst = nst;
-    kp.ahead = pass_ahead(g, alg);
-    void* args[] = {&kp};
-    cudaKernelNodeParams knp = {};
-    knp.func = const_cast<void*>(pk.func);
-    knp.gridDim = dim3(pass_grid(g, pk, smem));
-    knp.blockDim = dim3(pk.threads);
-    knp.sharedMemBytes = (unsigned)smem;
-    knp.kernelParams = args;
-    cudaGraphNode_t prev = nullptr, kn;
-    cudaError_t e = cudaSuccess;
-    for (int i = 0; i < CUSHA_DIAG_FIXED_GRAPH && e == cudaSuccess; ++i) {
-      e = cudaGraphAddKernelNode(&kn, graph, prev ? &prev : nullptr, prev ? 1 : 0, &knp);
-      prev = kn;
-    }
-    if (e == cudaSuccess) e = cudaGraphInstantiate(&h->exec[alg], graph, 0);
-    cudaGraphDestroy(graph);
-    if (e != cudaSuccess) { h->exec[alg] = nullptr; return fail(CUSHA_ECUDA, std::string("graph: ") + cudaGetErrorString(e)); }
-    return CUSHA_OK;
-  }
-#endif
-  cudaGraphConditionalHandle handle;
-  cudaError_t e = cudaGraphConditionalHandleCreate(&handle, graph, 1, cudaGraphCondAssignDefault);
-  if (e != cudaSuccess) { cudaGraphDestroy(graph); return fail(CUSHA_ECUDA, std::string("conditional handle: ") + cudaGetErrorString(e)); }
-  cudaGraphNodeParams cp = {};
-  cp.type = cudaGraphNodeTypeConditional;
-  cp.conditional.handle = handle;
-  cp.conditional.type = cudaGraphCondTypeWhile;
-  cp.conditional.size = 1;
-  cudaGraphNode_t cnode;
-  e = cudaGraphAddNode(&cnode, graph, nullptr, 0, &cp);
-  if (e != cudaSuccess) { cudaGraphDestroy(graph); return fail(CUSHA_ECUDA, std::string("conditional node: ") + cudaGetErrorString(e)); }
-  cudaGraph_t body = cp.conditional.phGraph_out[0];
-  KParams kp = make_params(g, 0);
-  kp.use_cond = CUSHA_DIAG_COND_NODE ? 0 : 1;
-  kp.mapj = mapj;
-  kp.stash = stash;
-  kp.nst = nst;
-  kp.ahead = pass_ahead(g, alg);
-  kp.cond_handle = handle;
+  KParams kp = pass_params(g, 0, c, alg);
   void* args[] = {&kp};
   cudaKernelNodeParams knp = {};
   knp.func = const_cast<void*>(pk.func);
-  knp.gridDim = dim3(pass_grid(g, pk, smem));
+  knp.gridDim = dim3(pass_grid(g, pk, c.smem));
   knp.blockDim = dim3(pk.threads);
-  knp.sharedMemBytes = (unsigned)smem;
+  knp.sharedMemBytes = (unsigned)c.smem;
   knp.kernelParams = args;
-  cudaGraphNode_t kn;
-  e = cudaGraphAddKernelNode(&kn, body, nullptr, 0, &knp);
-#if CUSHA_DIAG_COND_NODE
-  if (e == cudaSuccess) {
-    const Ctl* ctlp = g.d_ctl;
-    void* cargs[] = {&ctlp, &handle};
-    cudaKernelNodeParams cnp = {};
-    cnp.func = reinterpret_cast<void*>(diag_set_cond);
-    cnp.gridDim = dim3(1);
-    cnp.blockDim = dim3(1);
-    cnp.kernelParams = cargs;
-    cudaGraphNode_t sn;
-    e = cudaGraphAddKernelNode(&sn, body, &kn, 1, &cnp);
+  cudaGraphNode_t prev = nullptr, kn;
+  cudaError_t e = cudaSuccess;
+  for (int i = 0; i < kChunk && e == cudaSuccess; ++i) {
+    e = cudaGraphAddKernelNode(&kn, graph, prev ? &prev : nullptr, prev ? 1 : 0, &knp);
+    prev = kn;
   }
-#endif
   if (e == cudaSuccess) e = cudaGraphInstantiate(&h->exec[alg], graph, 0);
   cudaGraphDestroy(graph);
-  if (e != cudaSuccess) { h->exec[alg] = nullptr; return fail(CUSHA_ECUDA, std::string("graph: ") + cudaGetErrorString(e)); }
+  if (e != cudaSuccess) {
+    h->exec[alg] = nullptr;
+    return fail(CUSHA_ECUDA, std::string("graph: ") + cudaGetErrorString(e));
+  }
   return CUSHA_OK;
 }
 
-int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max_iters) {
-  if (!h) return fail(CUSHA_EINVAL, "graph is NULL");
-  if ((int)alg < 0 || (int)alg >= kNumAlgs) return fail(CUSHA_EINVAL, "bad algorithm");
-  Graph& g = h->g;
-  const int a = (int)alg;
-  if ((a == kBFS || a == kSSSP || a == kSSWP) && source >= g.V) return fail(CUSHA_EINVAL, "source >= num_vertices");
-  if (alg_needs_edge_values(a) && !g.has_ev) return fail(CUSHA_EINVAL, "algorithm needs edge_values");
-  if (alg_needs_init(a) && !g.d_init[a]) return fail(CUSHA_EINVAL, "NN/HS/CS need cusha_set_vertex_values first");
-  CKA(cudaSetDevice(g.device));
-  // trace buffer sized to min(max_iters, 2^20)
-  const uint32_t want_cap = std::min<uint32_t>(std::max<uint32_t>(max_iters, 1), 1u << 20);
-  if (g.trace_cap < want_cap) {
-    if (g.d_trace) cudaFreeAsync(g.d_trace, g.stream);
-    g.d_trace = nullptr;
-    g.trace_cap = 0;
-    CKA(cudaMallocAsync(&g.d_trace, sizeof(TraceRec) * (size_t)want_cap, g.stream));
-    CKA(cudaMemsetAsync(g.d_trace, 0, sizeof(TraceRec) * (size_t)want_cap, g.stream));
-    g.trace_cap = want_cap;
-    g.trace_dirty = 0;
-    for (auto& e : h->exec)  // kernel params captured the old trace pointer
-      if (e) { cudaGraphExecDestroy(e); e = nullptr; }
-  }
-  const PassKernel& pk = pass_kernel(a, g.repr);
-  size_t smem = 0;
-  int mapj = 0, stash = 0;
-  uint32_t nst = 0;
-  int rc = pass_config(g, pk, &smem, &mapj, &stash, &nst);
-  if (rc) return rc;
-  const bool host_loop = g.host_loop || g.G > 1;  // the partitioned mode exchanges between passes
-  // overlapped passes (default): one launch runs every pass; it needs a trace
-  // record per pass (<= 2^20), else the CUDA-graph loop runs one launch per pass
-  // automatic mode: many small shards per CTA favour one launch per pass
-  // (67_16 at |N| = 1536: 4.40 vs 5.48 ms)
-  bool barrier = g.pass_barrier == 1;
-  if (g.pass_barrier == 0 && g.S) {
-    const uint64_t grid = pass_grid(g, pk, smem);
-    barrier = (uint64_t)g.S >= 16 * grid && g.P <= 16384ull * g.S;
-  }
-  const bool multi = !host_loop && !barrier && max_iters <= g.trace_cap;
-  if (!host_loop && !multi) {
-    rc = ensure_exec(h, a);
-    if (rc) return rc;
-  }
-  // records a previous run may have written (the rest are still zero)
-  if (g.trace_dirty) CKA(cudaMemsetAsync(g.d_trace, 0, sizeof(TraceRec) * (size_t)g.trace_dirty, g.stream));
-  g.trace_dirty = g.trace_cap;  // until this run's extent is known
-  CKA(cudaEventRecord(g.ev0, g.stream));
-  CKA(launch_reset_ctl(g.d_ctl, max_iters, g.stream));
-  CKA(launch_init(g, a, source, g.stream));
-  CKA(cudaEventRecord(g.evm, g.stream));
-  if (max_iters > 0 && multi) {
-    KParams kp = make_params(g, source);
-    kp.multi = 1;
-    kp.mapj = mapj;
-    kp.stash = stash;
-    kp.nst = nst;
-    kp.ahead = pass_ahead(g, a);
-    void* args[] = {&kp};
-    CKA(cudaLaunchKernel(pk.func, dim3(pass_grid(g, pk, smem)), dim3(pk.threads), args, smem, g.stream));
-  } else if (max_iters > 0 && !host_loop) {
-    CKA(cudaGraphLaunch(h->exec[a], g.stream));
-  }
-  if (max_iters > 0 && host_loop) {
-    // passes launched by the host in chunks; a pass that finds the run
-    // converged (or at max_iters) exits at once, so over-launching is exact.
-    // Partitioned: pass -> exchange (NCCL, multi-GPU) -> refresh of remote
-    // windows + global convergence; every rank takes the same decisions
-    // from the same exchanged data, so all issue the same collectives.
-    KParams kp = make_params(g, source);
-    kp.mapj = mapj;
-    kp.stash = stash;
-    kp.nst = nst;
-    kp.ahead = pass_ahead(g, a);
-    void* args[] = {&kp};
-    const dim3 grid(pass_grid(g, pk, smem));
-    // 8 passes per host check, multi-GPU too: a pass launched after the run
-    // converged exits at once and the exchange / refresh after it change
-    // nothing, and every rank reads the same convergence flag after the same
-    // chunk, so all ranks issue the same collectives
-    const int chunk = 8;
-    std::string err;
-    for (;;) {
-      for (int k = 0; k < chunk; ++k) {
-        CKA(cudaLaunchKernel(pk.func, grid, dim3(pk.threads), args, smem, g.stream));
-        if (g.G > 1) {
-          if (!g.simulate && (rc = nccl_exchange(g, 0, false, err))) return fail(rc, "exchange: " + err);
-          CKA(launch_refresh(g, g.stream));
-        }
-      }
-      CKA(cudaMemcpyAsync(g.h_ctl, g.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g.stream));
-      CKA(cudaStreamSynchronize(g.stream));
-      if (g.h_ctl->converged || g.h_ctl->iter >= max_iters) break;
-    }
-    if (g.G > 1 && !g.simulate && (rc = nccl_exchange(g, (uint32_t)value_bytes(a), true, err)))
-      return fail(rc, "final exchange: " + err);
-  }
-  CKA(cudaEventRecord(g.ev1, g.stream));
-  CKA(cudaMemcpyAsync(g.h_ctl, g.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g.stream));
-  CKA(cudaStreamSynchronize(g.stream));
-  float ms = 0, lms = 0;
-  cudaEventElapsedTime(&ms, g.ev0, g.ev1);
-  cudaEventElapsedTime(&lms, g.evm, g.ev1);
-  Ctl c = *g.h_ctl;
-  {  // passes whose trace records this run touched: its iterations, or every drawn ticket's pass
-    const uint64_t drawn = multi && g.S ? c.ticket / g.S + 1 : 0;
-    g.trace_dirty = (uint32_t)std::min<uint64_t>(g.trace_cap, std::max<uint64_t>(c.iter, drawn) + 2);
-  }
-  if (multi && max_iters > 0) {  // the confirming pass that committed nothing, else max_iters passes ran
-    c.converged = c.conv_iter != 0xFFFFFFFFu;
-    c.iter = c.converged ? c.conv_iter : max_iters;
-  }
-  // statistics and algorithmic bytes
+// Fixed-point range of the float algorithms' stage-2 sums (include/cusha.h):
+// every |sum| must stay below 2^31.  PR: sum_{u->v} Rank_u/NbrsNum_u <=
+// sum_u Rank_u <= |V| < 2^31 at every pass (the total rank starts at |V| and
+// (1-d)|V| + d*(sum over non-dangling) keeps it there).  NN / HS / CS: a
+// bound from the initial values, the edge values and the largest in-degree.
+static int check_fixed_range(const Graph& g, int a) {
+  if (a != kNN && a != kHS && a != kCS) return CUSHA_OK;
+  const double w = g.max_abs_ev, x = g.init_max_abs[a], deg = std::max<uint32_t>(g.max_indeg, 1);
+  double term = 0;
+  if (a == kNN) term = std::max(x, 1.0) * w;       // |x_u * w|, |x_u| <= max(|x0|, 1) after tanh
+  else if (a == kHS) term = 2.0 * x * w;            // |(Q_u - Q_v) * coeff|
+  else term = std::max(x, 1.0) * std::max(w, 1.0);  // |V_u * G| and G itself
+  if (!(term * deg < 2147483648.0))
+    return fail(CUSHA_EINVAL, "values x edge values x in-degree reach the 2^31 fixed-point range of the stage-2 sums");
+  return CUSHA_OK;
+}
+
+static void account_run(const Graph& g, int a, const Ctl& c, bool multi, bool mapj, cusha_stats& st,
+                        std::vector<TraceRec>& tr) {
   const uint64_t vb = value_bytes(a);
   const uint64_t evb = alg_needs_edge_values(a) ? 4 : 0;
   const uint32_t n = std::min(c.iter, g.trace_cap);
-  TraceRec* tr = new TraceRec[n ? n : 1];
-  CKA(cudaMemcpy(tr, g.d_trace, sizeof(TraceRec) * n, cudaMemcpyDeviceToHost));
-  uint64_t bytes = 0, edges = 0;
+  uint64_t bytes = 0, paper = 0, edges = 0, wbe = 0, nvp = 0, upd = 0;
+  // paper-layout bytes: stage 2 per edge 8 (BFS, CC) / 12 (SSSP, SSWP, NN, PR) / 16 (HS, CS);
+  // stage 4 per active edge CW 12 / GS 8 (+4 for 8-byte vertices); stages 1+3 per vertex 2 * sizeof(Vertex)
+  const uint64_t p2 = (a == kBFS || a == kCC) ? 8 : (vb == 8 ? 16 : 12);
+  const uint64_t p4 = (g.repr == CUSHA_REPR_CW ? 12 : 8) + (vb == 8 ? 4 : 0);
   for (uint32_t i = 0; i < n; ++i) {
-    // vertices of the processed shards (all of V unless clean shards were skipped)
-    const uint64_t nv = std::min<uint64_t>(g.V, tr[i].shards * (uint64_t)g.N);
+    // vertices of the processed shards (all of the partition's unless clean shards were skipped)
+    const uint64_t nv = std::min<uint64_t>(g.nvl, tr[i].shards * (uint64_t)g.N);
     bytes += nv * vb + (a == kPR ? 4ull * nv : 0);                    // stages 1+3 reads
     bytes += (uint64_t)tr[i].updated * vb;                            // stage 3 commits
     bytes += tr[i].edges * (4 + 2 + evb);                             // stage 2
     edges += tr[i].edges;
+    wbe += tr[i].wb_entries;
+    nvp += nv;
+    upd += tr[i].updated;
     if (g.repr == CUSHA_REPR_CW)  // SrcIndexCW + window index (+ delta row) or u32 Mapper; SrcValue
       bytes += tr[i].wb_entries * (mapj ? 4 : 6) + tr[i].wb_stores * 4 +
                (mapj ? (uint64_t)tr[i].shards * 4ull * g.S : 0);
     else
       bytes += tr[i].wb_entries * 4 + tr[i].wb_stores * 4 + (uint64_t)tr[i].active_shards * 8ull * g.S;
+    paper += tr[i].edges * p2 + tr[i].wb_entries * p4 + nv * 2 * vb;
   }
-  delete[] tr;
-  g.st.iterations = c.iter;
-  g.st.converged = c.converged;
-  g.st.run_ms = ms;
-  g.st.loop_ms = lms;
-  g.st.last_algorithm = a;
-  g.st.algorithmic_bytes = bytes;
-  g.st.edges_processed = n == c.iter ? edges : (uint64_t)c.iter * g.E;
-  g.st.stage2_bytes_per_iter = g.E * (4 + 2 + evb);
-  g.st.wb_bytes_all_active = g.repr == CUSHA_REPR_CW ? g.E * (mapj ? 8 : 10) : g.E * 8;
-  g.st.mapper_form = (uint32_t)mapj;
-  g.st.device_loop = host_loop ? 0 : (multi ? 2 : 1);
-  g.last_alg = a;
-  g.have_values = true;
-  return c.converged ? CUSHA_OK : CUSHA_NOT_CONVERGED;
+  st.iterations = c.iter;
+  st.converged = c.converged;
+  st.algorithmic_bytes = bytes;
+  st.paper_bytes = paper;
+  st.edges_processed = n == c.iter ? edges : (uint64_t)c.iter * g.E_loc;
+  st.wb_entries = wbe;
+  st.vertices_processed = nvp;
+  st.updated_total = upd;
+  st.stage2_bytes_per_iter = g.E_loc * (4 + 2 + evb);
+  st.wb_bytes_all_active = g.repr == CUSHA_REPR_CW ? g.E_loc * (mapj ? 8 : 10) : g.E_loc * 8;
+  st.mapper_form = (uint32_t)mapj;
+  (void)multi;
+}
+
+static int read_trace(const Graph& g, uint32_t n, std::vector<TraceRec>& tr) {
+  tr.assign(std::max<uint32_t>(n, 1), TraceRec{});
+  if (n) {
+    CKA(cudaMemcpyAsync(tr.data(), g.d_trace, sizeof(TraceRec) * n, cudaMemcpyDeviceToHost, g.stream));
+    CKA(cudaStreamSynchronize(g.stream));
+  }
+  return CUSHA_OK;
+}
+
+}  // namespace cusha
+
+extern "C" {
+
+int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max_iters) {
+  if (!h) return fail(CUSHA_EINVAL, "graph is NULL");
+  if ((int)alg < 0 || (int)alg >= kNumAlgs) return fail(CUSHA_EINVAL, "bad algorithm");
+  Graph& g = g0(h);
+  const int a = (int)alg;
+  const uint32_t V = h->st.num_vertices;
+  if ((a == kBFS || a == kSSSP || a == kSSWP) && source >= V) return fail(CUSHA_EINVAL, "source >= num_vertices");
+  if (alg_needs_edge_values(a) && !g.has_ev) return fail(CUSHA_EINVAL, "algorithm needs edge_values");
+  if (alg_needs_init(a) && !g.d_init[a]) return fail(CUSHA_EINVAL, "NN/HS/CS need cusha_set_vertex_values first");
+  int rc = check_fixed_range(g, a);
+  if (rc) return rc;
+  CKA(cudaSetDevice(h->device));
+  cudaStream_t st = h->stream;
+  // trace buffer per partition, sized to min(max_iters, 2^20)
+  const uint32_t want_cap = std::min<uint32_t>(std::max<uint32_t>(max_iters, 1), 1u << 20);
+  for (Graph* p : h->parts) {
+    if (p->trace_cap >= want_cap) continue;
+    if (p->d_trace) cudaFreeAsync(p->d_trace, st);
+    p->d_trace = nullptr;
+    p->trace_cap = 0;
+    CKA(dev_alloc((void**)&p->d_trace, sizeof(TraceRec) * (size_t)want_cap, st));
+    CKA(cudaMemsetAsync(p->d_trace, 0, sizeof(TraceRec) * (size_t)want_cap, st));
+    p->trace_cap = want_cap;
+    p->trace_dirty = 0;
+    for (auto& e : h->exec)  // kernel params captured the old trace pointer
+      if (e) { cudaGraphExecDestroy(e); e = nullptr; }
+  }
+  const PassKernel& pk = pass_kernel(a, g.repr);
+  PassCfg cfg;
+  if ((rc = pass_config(g, pk, &cfg))) return rc;
+  const bool parted = h->mode != kModeSingle;
+  const bool host_loop = g.host_loop || parted;
+  // one launch for the whole run (overlapped passes) unless asked otherwise;
+  // the automatic mode takes one launch per pass for many small shards per
+  // CTA (67_16 at |N| = 1536: 4.40 vs 5.48 ms)
+  bool barrier = g.pass_barrier == 1;
+  if (g.pass_barrier == 0 && g.S) {
+    const uint64_t grid = pass_grid(g, pk, cfg.smem);
+    barrier = (uint64_t)g.S >= 16 * grid && g.P <= 16384ull * g.S;
+  }
+  const bool multi = !host_loop && !barrier && max_iters <= g.trace_cap;
+  if (!host_loop && !multi && (rc = ensure_exec(h, a, pk, cfg))) return rc;
+  // records a previous run may have written (the rest are still zero)
+  for (Graph* p : h->parts) {
+    if (p->trace_dirty) CKA(cudaMemsetAsync(p->d_trace, 0, sizeof(TraceRec) * (size_t)p->trace_dirty, st));
+    p->trace_dirty = p->trace_cap;  // until this run's extent is known
+  }
+  cudaEvent_t ev0, evm, ev1;
+  CKA(cudaEventCreate(&ev0));
+  CKA(cudaEventCreate(&evm));
+  CKA(cudaEventCreate(&ev1));
+  struct EvGuard {
+    cudaEvent_t a, b, c;
+    ~EvGuard() { cudaEventDestroy(a); cudaEventDestroy(b); cudaEventDestroy(c); }
+  } evg{ev0, evm, ev1};
+  std::string err;
+  CKA(cudaEventRecord(ev0, st));
+  for (Graph* p : h->parts) CKA(launch_reset_ctl(p->d_ctl, max_iters, st));
+  for (Graph* p : h->parts) CKA(launch_init(*p, a, source, st));
+  // every partition's SrcValue is initialised (R20) before any pass reads it
+  if (h->mode == kModeNccl && (rc = nccl_allreduce_max_u32(g, &g.d_ctl->lchanged, &g.d_ctl->gchanged, err)))
+    return fail(rc, "init barrier: " + err);
+  CKA(cudaEventRecord(evm, st));
+  if (max_iters > 0 && multi) {
+    KParams kp = pass_params(g, source, cfg, a);
+    kp.multi = 1;
+    void* args[] = {&kp};
+    CKA(cudaLaunchKernel(pk.func, dim3(pass_grid(g, pk, cfg.smem)), dim3(pk.threads), args, cfg.smem, st));
+  } else if (max_iters > 0) {
+    // passes in chunks; a pass that finds the run converged (or at max_iters)
+    // exits at once, so over-launching is exact.  Partitioned: every
+    // partition's pass, then the global convergence decision; every rank
+    // takes it from the same all-reduced word, so all issue the same collectives.
+    std::vector<KParams> kps;
+    std::vector<uint32_t> grids;
+    for (Graph* p : h->parts) {
+      kps.push_back(pass_params(*p, source, cfg, a));
+      grids.push_back(pass_grid(*p, pk, cfg.smem));
+    }
+    for (;;) {
+      if (host_loop) {
+        for (int k = 0; k < kChunk; ++k) {
+          for (size_t r = 0; r < h->parts.size(); ++r) {
+            void* args[] = {&kps[r]};
+            CKA(cudaLaunchKernel(pk.func, dim3(grids[r]), dim3(pk.threads), args, cfg.smem, st));
+          }
+          if (h->mode == kModeSim) {
+            CKA(launch_close_parts(h->d_ctls, (uint32_t)h->parts.size(), st));
+          } else if (h->mode == kModeNccl) {
+            if ((rc = nccl_allreduce_max_u32(g, &g.d_ctl->lchanged, &g.d_ctl->gchanged, err)))
+              return fail(rc, "convergence all-reduce: " + err);
+            CKA(launch_close_parts(h->d_ctls, 0, st));
+          }
+        }
+      } else {
+        CKA(cudaGraphLaunch(h->exec[a], st));
+      }
+      CKA(cudaMemcpyAsync(g.h_ctl, g.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, st));
+      CKA(cudaStreamSynchronize(st));
+      if (g.h_ctl->converged || g.h_ctl->iter >= max_iters) break;
+    }
+  }
+  CKA(cudaEventRecord(ev1, st));
+  CKA(cudaStreamSynchronize(st));
+  float ms = 0, lms = 0;
+  cudaEventElapsedTime(&ms, ev0, ev1);
+  cudaEventElapsedTime(&lms, evm, ev1);
+  // statistics and algorithmic bytes, per partition and summed
+  cusha_stats sum{};
+  Ctl c0{};
+  for (size_t r = 0; r < h->parts.size(); ++r) {
+    Graph& p = *h->parts[r];
+    CKA(cudaMemcpyAsync(p.h_ctl, p.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, st));
+    CKA(cudaStreamSynchronize(st));
+    Ctl c = *p.h_ctl;
+    {  // passes whose trace records this run touched: its iterations, or every drawn ticket's pass
+      const uint64_t drawn = multi && p.Sl ? c.ticket / p.Sl + 1 : 0;
+      p.trace_dirty = (uint32_t)std::min<uint64_t>(p.trace_cap, std::max<uint64_t>(c.iter, drawn) + 2);
+    }
+    if (multi && max_iters > 0) {  // the confirming pass that committed nothing, else max_iters passes ran
+      c.converged = c.conv_iter != 0xFFFFFFFFu;
+      c.iter = c.converged ? c.conv_iter : max_iters;
+    }
+    std::vector<TraceRec> tr;
+    if ((rc = read_trace(p, std::min(c.iter, p.trace_cap), tr))) return rc;
+    account_run(p, a, c, multi, cfg.mapj != 0, p.st, tr);
+    p.st.run_ms = ms;
+    p.st.loop_ms = lms;
+    if (r == 0) c0 = c;
+    sum.algorithmic_bytes += p.st.algorithmic_bytes;
+    sum.paper_bytes += p.st.paper_bytes;
+    sum.edges_processed += p.st.edges_processed;
+    sum.wb_entries += p.st.wb_entries;
+    sum.vertices_processed += p.st.vertices_processed;
+    sum.updated_total += p.st.updated_total;
+    sum.stage2_bytes_per_iter += p.st.stage2_bytes_per_iter;
+    sum.wb_bytes_all_active += p.st.wb_bytes_all_active;
+  }
+  cusha_stats& s = h->st;
+  s.iterations = c0.iter;
+  s.converged = c0.converged;
+  s.run_ms = ms;
+  s.loop_ms = lms;
+  s.last_algorithm = a;
+  s.algorithmic_bytes = sum.algorithmic_bytes;
+  s.paper_bytes = sum.paper_bytes;
+  s.edges_processed = sum.edges_processed;
+  s.wb_entries = sum.wb_entries;
+  s.vertices_processed = sum.vertices_processed;
+  s.updated_total = sum.updated_total;
+  s.stage2_bytes_per_iter = sum.stage2_bytes_per_iter;
+  s.wb_bytes_all_active = sum.wb_bytes_all_active;
+  s.mapper_form = (uint32_t)cfg.mapj;
+  s.device_loop = host_loop ? 0 : (multi ? 2 : 1);
+  h->last_alg = a;
+  h->have_values = true;
+  return c0.converged ? CUSHA_OK : CUSHA_NOT_CONVERGED;
+}
+
+// copy every partition's VertexValues slice to dst (host or device)
+static int copy_values(const cusha_graph* h, void* dst, bool to_host) {
+  const uint32_t V = h->st.num_vertices;
+  const size_t vb = value_bytes(h->last_alg);
+  const cudaMemcpyKind kind = to_host ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
+  if (h->mode == kModeNccl) {
+    Graph& g = *h->parts[0];
+    void* full = nullptr;
+    CKA(dev_alloc(&full, (size_t)V * vb, h->stream));
+    std::string err;
+    const int rc = nccl_gather_values(g, full, (uint32_t)vb, err);
+    if (rc) {
+      cudaFreeAsync(full, h->stream);
+      return fail(rc, "gather: " + err);
+    }
+    CKA(cudaMemcpyAsync(dst, full, (size_t)V * vb, kind, h->stream));
+    cudaFreeAsync(full, h->stream);
+  } else {
+    for (const Graph* g : h->parts)
+      if (g->nvl)
+        CKA(cudaMemcpyAsync(static_cast<char*>(dst) + (size_t)g->v0 * vb, g->d_vv, (size_t)g->nvl * vb, kind,
+                            h->stream));
+  }
+  CKA(cudaStreamSynchronize(h->stream));
+  return CUSHA_OK;
 }
 
 int cusha_get_values(const cusha_graph* h, void* out, size_t out_bytes) {
   if (!h || !out) return fail(CUSHA_EINVAL, "null argument");
-  const Graph& g = h->g;
-  if (!g.have_values) return fail(CUSHA_ESTATE, "no run yet");
-  const size_t want = (size_t)g.V * value_bytes(g.last_alg);
+  if (!h->have_values) return fail(CUSHA_ESTATE, "no run yet");
+  const size_t want = (size_t)h->st.num_vertices * value_bytes(h->last_alg);
   if (out_bytes != want) return fail(CUSHA_EINVAL, "out_bytes must be |V| * value_bytes(last algorithm)");
-  CKA(cudaSetDevice(g.device));
-  CKA(cudaMemcpyAsync(out, g.d_vv, want, cudaMemcpyDeviceToHost, g.stream));
-  CKA(cudaStreamSynchronize(g.stream));
-  return CUSHA_OK;
+  CKA(cudaSetDevice(h->device));
+  return copy_values(h, out, true);
 }
 
 int cusha_get_values_device(const cusha_graph* h, void* dptr, size_t out_bytes) {
   if (!h || !dptr) return fail(CUSHA_EINVAL, "null argument");
-  const Graph& g = h->g;
-  if (!g.have_values) return fail(CUSHA_ESTATE, "no run yet");
-  const size_t want = (size_t)g.V * value_bytes(g.last_alg);
+  if (!h->have_values) return fail(CUSHA_ESTATE, "no run yet");
+  const size_t want = (size_t)h->st.num_vertices * value_bytes(h->last_alg);
   if (out_bytes != want) return fail(CUSHA_EINVAL, "out_bytes must be |V| * value_bytes(last algorithm)");
-  CKA(cudaSetDevice(g.device));
-  CKA(cudaMemcpyAsync(dptr, g.d_vv, want, cudaMemcpyDeviceToDevice, g.stream));
-  CKA(cudaStreamSynchronize(g.stream));
-  return CUSHA_OK;
+  CKA(cudaSetDevice(h->device));
+  return copy_values(h, dptr, false);
 }
 
 int cusha_get_stats(const cusha_graph* h, cusha_stats* s) {
   if (!h || !s) return fail(CUSHA_EINVAL, "null argument");
-  *s = h->g.st;
+  *s = h->st;
+  return CUSHA_OK;
+}
+
+int cusha_get_part_stats(const cusha_graph* h, uint32_t part, cusha_stats* s) {
+  if (!h || !s) return fail(CUSHA_EINVAL, "null argument");
+  if (part >= h->parts.size()) return fail(CUSHA_EINVAL, "partition not held by this handle");
+  const Graph& g = *h->parts[part];
+  *s = h->st;
+  s->device_bytes = device_bytes(g);
+  s->max_part_device_bytes = s->device_bytes;
+  s->entries_padded = g.P;
+  s->rank = h->mode == kModeNccl ? h->st.rank : (int)part;
+  if (h->have_values) {
+    s->algorithmic_bytes = g.st.algorithmic_bytes;
+    s->paper_bytes = g.st.paper_bytes;
+    s->edges_processed = g.st.edges_processed;
+    s->wb_entries = g.st.wb_entries;
+    s->vertices_processed = g.st.vertices_processed;
+    s->updated_total = g.st.updated_total;
+    s->stage2_bytes_per_iter = g.st.stage2_bytes_per_iter;
+    s->wb_bytes_all_active = g.st.wb_bytes_all_active;
+  }
   return CUSHA_OK;
 }
 
 int cusha_get_trace(const cusha_graph* h, uint32_t* upd, uint32_t* act, uint32_t cap) {
   if (!h) return fail(CUSHA_EINVAL, "null argument");
-  const Graph& g = h->g;
-  if (!g.have_values || !g.d_trace) return 0;
-  const uint32_t n = std::min(std::min(g.st.iterations, g.trace_cap), cap);
+  if (!h->have_values) return 0;
+  const uint32_t n = std::min(std::min(h->st.iterations, g0(h).trace_cap), cap);
   if (!n) return 0;
-  TraceRec* tr = new TraceRec[n];
-  cudaSetDevice(g.device);
-  if (cudaMemcpy(tr, g.d_trace, sizeof(TraceRec) * n, cudaMemcpyDeviceToHost) != cudaSuccess) {
-    delete[] tr;
-    return fail(CUSHA_ECUDA, "trace copy");
+  cudaSetDevice(h->device);
+  std::vector<uint64_t> su(n, 0), sa(n, 0);
+  for (const Graph* g : h->parts) {  // summed over the partitions of this handle
+    std::vector<TraceRec> tr;
+    const int rc = read_trace(*g, n, tr);
+    if (rc) return rc;
+    for (uint32_t i = 0; i < n; ++i) {
+      su[i] += tr[i].updated;
+      sa[i] += tr[i].active_shards;
+    }
   }
   for (uint32_t i = 0; i < n; ++i) {
-    if (upd) upd[i] = tr[i].updated;
-    if (act) act[i] = tr[i].active_shards;
+    if (upd) upd[i] = (uint32_t)su[i];
+    if (act) act[i] = (uint32_t)sa[i];
   }
-  delete[] tr;
   return (int)n;
 }
 
-int cusha_get_layout(const cusha_graph* h, cusha_layout_part part, void* out, size_t out_bytes, uint64_t* count) {
-  if (!h) return fail(CUSHA_EINVAL, "graph is NULL");
-  const Graph& g = h->g;
+static int layout_of(const Graph& g, cusha_layout_part part, void* out, size_t out_bytes, uint64_t* count) {
   const void* src = nullptr;
   const void* tail = nullptr;  // host-resident part (row f3) from position `split`
   uint64_t n = 0, split = ~0ull;
   size_t es = 4;
   switch (part) {
-    case CUSHA_LAYOUT_SHARD_OFFSETS: src = g.d_shard_off; n = (uint64_t)g.S + 1; break;
-    case CUSHA_LAYOUT_SHARD_SIZES: src = g.d_shard_cnt; n = g.S; break;
+    case CUSHA_LAYOUT_SHARD_OFFSETS: src = g.d_shard_off; n = (uint64_t)g.Sl + 1; break;
+    case CUSHA_LAYOUT_SHARD_SIZES: src = g.d_shard_cnt; n = g.Sl; break;
     case CUSHA_LAYOUT_SRC_INDEX: src = g.d_srcloc; tail = g.h_srcloc; split = g.splitP; n = g.P; es = 2; break;
     case CUSHA_LAYOUT_DEST_LOCAL: src = g.d_dest; tail = g.h_dest; split = g.splitP; n = g.P; es = 2; break;
     case CUSHA_LAYOUT_EDGE_ID: src = g.d_eid; tail = g.h_eid; split = g.splitP; n = g.P; break;
-    case CUSHA_LAYOUT_WINDOWS: src = g.d_win; n = ((uint64_t)g.S + 1) * g.S; break;
-    case CUSHA_LAYOUT_CW_OFFSETS: src = g.d_cw_off; n = (uint64_t)g.S + 1; break;
-    case CUSHA_LAYOUT_CW_SIZES: src = g.d_cw_cnt; n = g.S; break;
+    case CUSHA_LAYOUT_WINDOWS: src = g.d_win; n = ((uint64_t)g.Sl + 1) * g.S; break;
+    case CUSHA_LAYOUT_CW_OFFSETS: src = g.d_cw_off; n = (uint64_t)g.Sl + 1; break;
+    case CUSHA_LAYOUT_CW_SIZES: src = g.d_cw_cnt; n = g.Sl; break;
     case CUSHA_LAYOUT_CW_SRC_LOCAL: src = g.d_cw_src; tail = g.h_cw_src; split = g.splitQ; n = g.Q; es = 2; break;
     case CUSHA_LAYOUT_MAPPER: src = g.d_mapper; tail = g.h_mapper; split = g.splitQ; n = g.Q; break;
-    case CUSHA_LAYOUT_OUT_DEGREE: src = g.d_outdeg; n = g.V; break;
+    case CUSHA_LAYOUT_OUT_DEGREE: src = g.d_outdeg; n = g.nvl; break;
     case CUSHA_LAYOUT_RUN_K: src = g.d_run_k; n = g.R; break;
     case CUSHA_LAYOUT_RUN_T: src = g.d_run_t; n = g.R; break;
     case CUSHA_LAYOUT_CW_WINDOW: src = g.d_cw_win; tail = g.h_cw_win; split = g.splitQ; n = g.Q; es = 2; break;
-    case CUSHA_LAYOUT_CW_DELTA: src = g.d_cw_delta; n = (uint64_t)g.S * g.S; break;
+    case CUSHA_LAYOUT_CW_DELTA: src = g.d_cw_delta; n = (uint64_t)g.Sl * g.S; break;
+    case CUSHA_LAYOUT_CW_PARTITION_OFFSETS: src = g.d_cwp; n = (uint64_t)g.Sl * (g.G + 1); break;
     default: return fail(CUSHA_EINVAL, "bad layout part");
   }
-  if (!src && !tail) return fail(CUSHA_EUNSUPPORTED, "part not held by this representation");
+  if (!src && !tail) return fail(CUSHA_EUNSUPPORTED, "part not held by this graph (representation / options)");
   if (count) *count = n;
   if (!out) return CUSHA_OK;
   if (out_bytes < n * es) return fail(CUSHA_EINVAL, "out_bytes too small");
   CKA(cudaSetDevice(g.device));
   const uint64_t nd = std::min(n, split);  // HBM part
-  if (nd) CKA(cudaMemcpy(out, src, nd * es, cudaMemcpyDeviceToHost));
+  if (nd) {
+    CKA(cudaMemcpyAsync(out, src, nd * es, cudaMemcpyDeviceToHost, g.stream));
+    CKA(cudaStreamSynchronize(g.stream));
+  }
   if (nd < n) std::memcpy(static_cast<char*>(out) + nd * es, tail, (n - nd) * es);
   return CUSHA_OK;
+}
+
+int cusha_get_layout(const cusha_graph* h, cusha_layout_part part, void* out, size_t out_bytes, uint64_t* count) {
+  if (!h) return fail(CUSHA_EINVAL, "graph is NULL");
+  if (h->mode != kModeSingle)
+    return fail(CUSHA_EUNSUPPORTED, "partitioned graph: use cusha_get_part_layout");
+  return layout_of(g0(h), part, out, out_bytes, count);
+}
+
+int cusha_get_part_layout(const cusha_graph* h, uint32_t p, cusha_layout_part part, void* out, size_t out_bytes,
+                          uint64_t* count) {
+  if (!h) return fail(CUSHA_EINVAL, "graph is NULL");
+  if (p >= h->parts.size()) return fail(CUSHA_EINVAL, "partition not held by this handle");
+  return layout_of(*h->parts[p], part, out, out_bytes, count);
 }
 
 int cusha_nccl_unique_id(void* out128) {
@@ -735,16 +998,11 @@ int cusha_partition_shards(uint32_t num_shards, const uint64_t* work, uint32_t p
 
 int cusha_get_partition(const cusha_graph* h, uint32_t* bounds, uint32_t cap) {
   if (!h || !bounds) return fail(CUSHA_EINVAL, "null argument");
-  const Graph& g = h->g;
-  if (g.G <= 1) {
-    if (cap < 2) return fail(CUSHA_EINVAL, "cap too small");
-    bounds[0] = 0;
-    bounds[1] = g.S;
-    return 1;
-  }
-  if (cap < g.G + 1) return fail(CUSHA_EINVAL, "cap too small");
-  for (uint32_t q = 0; q <= g.G; ++q) bounds[q] = g.h_bounds[q];
-  return (int)g.G;
+  const std::vector<uint32_t>& b = g0(h).h_bounds;
+  const uint32_t G = (uint32_t)b.size() - 1;
+  if (cap < G + 1) return fail(CUSHA_EINVAL, "cap too small");
+  for (uint32_t q = 0; q <= G; ++q) bounds[q] = b[q];
+  return (int)G;
 }
 
 int cusha_diag_timeline(void* out, size_t out_bytes) {

@@ -18,6 +18,7 @@
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
+#include <cstring>
 #include <string>
 #include <vector>
 
@@ -91,7 +92,7 @@ __global__ void k_fill_shard_pads(const uint32_t* off, const uint32_t* cnt, uint
     if (pos < off[s + 1]) {
       dest[pos] = (uint16_t)N;
       srcidx[pos] = 0;
-      eid[pos] = 0xFFFFFFFFu;
+      if (eid) eid[pos] = 0xFFFFFFFFu;
       if (ev) ev[pos] = 0;
     }
   }
@@ -108,7 +109,7 @@ __global__ void k_scatter_gs(const uint64_t* __restrict__ keys, const uint32_t* 
     dest[pp] = (uint16_t)(k & mn);
     srcidx[pp] = (uint16_t)(((k >> bn) & ms) % N);  // SrcIndex local to its source shard
     const uint32_t id = ids[p];
-    eid[pp] = id;
+    if (eid) eid[pp] = id;
     if (ev) ev[pp] = val[id];
   }
 }
@@ -139,6 +140,28 @@ __global__ void k_windows_tail(const uint64_t* __restrict__ keys, const uint32_t
 
 __global__ void k_outdeg(const uint32_t* __restrict__ src, uint64_t E, uint32_t* outdeg) {
   GRID_STRIDE(e, E) atomicAdd(&outdeg[src[e]], 1u);
+}
+// largest in-degree: the shard entries of one destination are consecutive
+// within its shard only after sorting by dst, so count with atomics instead
+__global__ void k_indeg(const uint32_t* __restrict__ dst, uint64_t E, uint32_t* indeg) {
+  GRID_STRIDE(e, E) atomicAdd(&indeg[dst[e]], 1u);
+}
+__global__ void k_max_u32(const uint32_t* __restrict__ a, uint64_t n, uint32_t* out) {
+  uint32_t m = 0;
+  GRID_STRIDE(i, n) m = max(m, a[i]);
+  for (int o = 16; o; o >>= 1) m = max(m, __shfl_xor_sync(0xFFFFFFFFu, m, o));
+  if ((threadIdx.x & 31) == 0 && m) atomicMax(out, m);
+}
+// largest |x| of raw 4-byte values read as f32 (non-finite: +inf bits)
+__global__ void k_max_abs_f32(const uint32_t* __restrict__ a, uint64_t n, uint32_t* out) {
+  uint32_t m = 0;
+  GRID_STRIDE(i, n) {
+    uint32_t b = a[i] & 0x7FFFFFFFu;
+    if (b > 0x7F800000u) b = 0x7F800000u;  // NaN counts as infinite
+    m = max(m, b);                          // non-negative floats order like their bits
+  }
+  for (int o = 16; o; o >>= 1) m = max(m, __shfl_xor_sync(0xFFFFFFFFu, m, o));
+  if ((threadIdx.x & 31) == 0 && m) atomicMax(out, m);
 }
 
 // |CW_i| = sum of out-degrees over shard i's vertex range
@@ -253,7 +276,7 @@ struct PhaseTimer {
 
 template <class T>
 cudaError_t dalloc(T** p, uint64_t n) {
-  return cudaMallocAsync(reinterpret_cast<void**>(p), (n ? n : 1) * sizeof(T), t_alloc_stream);
+  return dev_alloc(reinterpret_cast<void**>(p), (n ? n : 1) * sizeof(T), t_alloc_stream);
 }
 
 // ---- run-length form of Mapper
@@ -319,10 +342,10 @@ int build_runs(Graph& g, std::string& err) {
   CK(cudaGetLastError());
   size_t b1 = 0, b2 = 0;
   CK(cub::DeviceScan::ExclusiveSum(nullptr, b1, (uint32_t*)len.p, (uint32_t*)pos.p, (int64_t)S2, st));
-  CK(cudaMallocAsync(&t1.p, b1 ? b1 : 1, st));
+  CK(dev_alloc(&t1.p, b1 ? b1 : 1, st));
   CK(cub::DeviceScan::ExclusiveSum(t1.p, b1, (uint32_t*)len.p, (uint32_t*)pos.p, (int64_t)S2, st));
   CK(cub::DeviceScan::InclusiveSum(nullptr, b2, (uint32_t*)nonempty.p, (uint32_t*)ridx.p + 1, (int64_t)S2, st));
-  CK(cudaMallocAsync(&t2.p, b2 ? b2 : 1, st));
+  CK(dev_alloc(&t2.p, b2 ? b2 : 1, st));
   CK(cudaMemsetAsync(ridx.p, 0, 4, st));
   CK(cub::DeviceScan::InclusiveSum(t2.p, b2, (uint32_t*)nonempty.p, (uint32_t*)ridx.p + 1, (int64_t)S2, st));
   uint32_t R = 0;
@@ -353,6 +376,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   cudaStream_t st = g.stream;
   const uint64_t E = g.E;
   const uint32_t V = g.V, N = g.N, S = g.S;
+  g.s0 = 0; g.Sl = S; g.v0 = 0; g.nvl = V; g.E_loc = E;
   const int bn = bits_for(N - 1) ? bits_for(N - 1) : 1, bsrc = bits_for(V - 1) ? bits_for(V - 1) : 1,
             bsh = bits_for(S - 1);
   const int total = bsh + bsrc + bn;
@@ -383,7 +407,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   size_t tbytes = 0;
   if (E) {
     CK(cub::DeviceRadixSort::SortPairs(nullptr, tbytes, kb, vb, (int64_t)E, 0, total, st));
-    CK(cudaMallocAsync(&temp.p, tbytes, st));
+    CK(dev_alloc(&temp.p, tbytes, st));
     CK(cub::DeviceRadixSort::SortPairs(temp.p, tbytes, kb, vb, (int64_t)E, 0, total, st));
   }
   pt.mark("G-Shards sort");
@@ -403,7 +427,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
     size_t b2 = 0;
     CK(dalloc((uint64_t**)&scan.p, (uint64_t)S + 1));
     CK(cub::DeviceScan::ExclusiveSum(nullptr, b2, (uint64_t*)padded.p, (uint64_t*)scan.p, (int64_t)S + 1, st));
-    CK(cudaMallocAsync(&t2.p, b2 ? b2 : 1, st));
+    CK(dev_alloc(&t2.p, b2 ? b2 : 1, st));
     CK(cub::DeviceScan::ExclusiveSum(t2.p, b2, (uint64_t*)padded.p, (uint64_t*)scan.p, (int64_t)S + 1, st));
     uint64_t P = 0;
     CK(cudaMemcpyAsync(&P, (uint64_t*)scan.p + S, 8, cudaMemcpyDeviceToHost, st));
@@ -416,7 +440,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   const uint64_t P = g.P;
   CK(dalloc(&g.d_dest, P));
   CK(dalloc(&g.d_srcloc, P));
-  CK(dalloc(&g.d_eid, P));
+  if (g.keep_ids) CK(dalloc(&g.d_eid, P));  // layout inspection only (no kernel reads it)
   if (d_val) { CK(dalloc(&g.d_ev, P)); g.has_ev = true; }
   pt.mark("offsets + alloc shard arrays");
   k_fill_shard_pads<<<grid_for((uint64_t)S * kPad), 256, 0, st>>>(g.d_shard_off, g.d_shard_cnt, S, N, g.d_dest,
@@ -440,6 +464,21 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   CK(dalloc(&g.d_outdeg, V));
   CK(cudaMemsetAsync(g.d_outdeg, 0, (size_t)V * 4, st));
   if (E) k_outdeg<<<grid_for(E), 256, 0, st>>>(d_src, E, g.d_outdeg);
+  {  // range of the float algorithms' fixed-point sums (include/cusha.h "Fixed-point range")
+    DevBuf indeg, mx;
+    CK(dalloc((uint32_t**)&indeg.p, V));
+    CK(dalloc((uint32_t**)&mx.p, 2));
+    CK(cudaMemsetAsync(indeg.p, 0, (size_t)V * 4, st));
+    CK(cudaMemsetAsync(mx.p, 0, 8, st));
+    if (E) k_indeg<<<grid_for(E), 256, 0, st>>>(d_dst, E, (uint32_t*)indeg.p);
+    k_max_u32<<<grid_for(V), 256, 0, st>>>((uint32_t*)indeg.p, V, (uint32_t*)mx.p);
+    if (d_val && E) k_max_abs_f32<<<grid_for(E), 256, 0, st>>>(d_val, E, (uint32_t*)mx.p + 1);
+    uint32_t h[2] = {0, 0};
+    CK(cudaMemcpyAsync(h, mx.p, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    g.max_indeg = h[0];
+    std::memcpy(&g.max_abs_ev, &h[1], 4);
+  }
   CK(dalloc(&g.d_cw_cnt, S));
   k_cw_counts<<<S, 256, 0, st>>>(g.d_outdeg, V, N, g.d_cw_cnt);
   CK(cudaGetLastError());
@@ -459,7 +498,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
     CK(cudaGetLastError());
     size_t b4 = 0;
     CK(cub::DeviceScan::ExclusiveSum(nullptr, b4, (uint64_t*)cpad.p, (uint64_t*)cscan.p, (int64_t)S + 1, st));
-    CK(cudaMallocAsync(&t4.p, b4 ? b4 : 1, st));
+    CK(dev_alloc(&t4.p, b4 ? b4 : 1, st));
     CK(cub::DeviceScan::ExclusiveSum(t4.p, b4, (uint64_t*)cpad.p, (uint64_t*)cscan.p, (int64_t)S + 1, st));
     uint64_t Q = 0;
     CK(cudaMemcpyAsync(&Q, (uint64_t*)cscan.p + S, 8, cudaMemcpyDeviceToHost, st));
@@ -483,8 +522,10 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
     cudaFreeAsync(g.d_srcloc, st);
     g.d_srcloc = nullptr;
     pt.mark("CW offsets + scatter");
-    const int rc = build_runs(g, err);
-    if (rc) return rc;
+    if (kernels_rle()) {  // the run-length Mapper only serves builds with CUSHA_RLE stage 4
+      const int rc = build_runs(g, err);
+      if (rc) return rc;
+    }
   }
   pt.mark("Mapper runs");
   CK(cudaStreamSynchronize(st));
@@ -542,8 +583,8 @@ int offload_topology(Graph& g, std::string& err) {
   CK(cudaMemcpyAsync(so.data(), g.d_shard_off, 4ull * (S + 1), cudaMemcpyDeviceToHost, st));
   if (g.d_cw_off) CK(cudaMemcpyAsync(co.data(), g.d_cw_off, 4ull * (S + 1), cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
-  const uint64_t bP = 2 + 4 + (g.has_ev ? 4 : 0) + (g.d_srcloc ? 2 : 0);  // DestIndex, edge id, EdgeValue, SrcIndex
-  const uint64_t bQ = g.d_cw_src ? 8 : 0;                                  // SrcIndexCW, Mapper, window
+  const uint64_t bP = 2 + (g.d_eid ? 4 : 0) + (g.has_ev ? 4 : 0) + (g.d_srcloc ? 2 : 0);  // DestIndex, edge id, EdgeValue, SrcIndex
+  const uint64_t bQ = g.d_cw_src ? 8 : 0;                                                 // SrcIndexCW, Mapper, window
   uint32_t h = 0;
   while (h < S && (uint64_t)so[h + 1] * bP + (uint64_t)co[h + 1] * bQ <= g.topo_budget) ++h;
   g.host_shard = h;
@@ -580,52 +621,225 @@ void partition_bounds(uint32_t S, const uint64_t* work, uint32_t G, uint32_t* bo
   bounds[G] = S;
 }
 
+// ------------------------------------------------ destination-range partition (row e)
+// Work per shard for the split: stage-2 entries (its in-edges) + stage-4
+// entries (|CW_s|, the out-edges of its vertices).
+int partition_work(const Graph& glob, std::vector<uint64_t>& work, std::string& err) {
+  const uint32_t S = glob.S;
+  std::vector<uint32_t> cnt(S), ccnt(S, 0);
+  CK(cudaMemcpyAsync(cnt.data(), glob.d_shard_cnt, 4ull * S, cudaMemcpyDeviceToHost, glob.stream));
+  CK(cudaMemcpyAsync(ccnt.data(), glob.d_cw_cnt, 4ull * S, cudaMemcpyDeviceToHost, glob.stream));
+  CK(cudaStreamSynchronize(glob.stream));
+  work.resize(S);
+  for (uint32_t s = 0; s < S; ++s) work[s] = (uint64_t)cnt[s] + ccnt[s];
+  return CUSHA_OK;
+}
+
 namespace {
-// cwp[i][q] = first CW_i position whose Mapper target lies in partition q:
-// CW_i lists W_i0, W_i1, ... in shard order (L175), so that is cw_off[i] plus
-// the sizes of W_ij for j < bounds[q].
-__global__ void k_cwp(const uint32_t* __restrict__ win, const uint32_t* cw_off, const uint32_t* cw_cnt,
-                      const uint32_t* bounds, uint32_t S, uint32_t G, uint32_t* cwp) {
-  GRID_STRIDE(t, (uint64_t)S * (G + 1)) {
-    const uint32_t i = (uint32_t)(t / (G + 1)), q = (uint32_t)(t % (G + 1));
+__global__ void k_rebase(const uint32_t* __restrict__ in, uint64_t n, uint32_t sub, uint32_t* out) {
+  GRID_STRIDE(i, n) out[i] = in[i] - sub;
+}
+// partition owning global padded shard position m: pb[q] <= m < pb[q+1]
+__device__ __forceinline__ uint32_t part_of_pos(const uint32_t* pb, uint32_t G, uint32_t m) {
+  uint32_t lo = 0, hi = G;
+  while (hi - lo > 1) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (pb[mid] <= m) lo = mid;
+    else hi = mid;
+  }
+  return lo;
+}
+// Mapper of the partition's CW_i: the target position local to the partition
+// that owns it (filler entries: 0xFFFFFFFF; no kernel reads them)
+__global__ void k_mapper_local(const uint32_t* __restrict__ m, uint64_t n, const uint32_t* __restrict__ pb, uint32_t G,
+                               uint32_t trash, uint32_t* out) {
+  GRID_STRIDE(k, n) {
+    const uint32_t t = m[k];
+    out[k] = t == trash ? 0xFFFFFFFFu : t - pb[part_of_pos(pb, G, t)];
+  }
+}
+// window-form Mapper of the partition: Mapper_loc[k_loc] = delta_loc[il][j] + k_loc with
+// k_loc = k - c0 and targets local to owner(j):  delta_loc = delta + c0 - pb[owner(j)]  (mod 2^32)
+__global__ void k_delta_local(const uint32_t* __restrict__ delta, uint32_t Sl, uint32_t S, uint32_t c0,
+                              const uint32_t* __restrict__ pb, const uint8_t* __restrict__ owner, uint32_t* out) {
+  GRID_STRIDE(t, (uint64_t)Sl * S) {
+    const uint32_t j = (uint32_t)(t % S);
+    out[t] = delta[t] + c0 - pb[owner[j]];
+  }
+}
+// cwp[il][q] = first CW_i position (local) whose target lies in partition q:
+// CW_i lists W_i0, W_i1, ... in shard order (L175), so that is the start of
+// CW_i plus the sizes of W_ij for j < bounds[q]; cwp[il][G] = end of CW_i.
+__global__ void k_cwp_local(const uint32_t* __restrict__ win_rows, const uint32_t* __restrict__ cw_off_loc,
+                            const uint32_t* __restrict__ cw_cnt, const uint32_t* __restrict__ bounds, uint32_t Sl,
+                            uint32_t S, uint32_t G, uint32_t* cwp) {
+  GRID_STRIDE(t, (uint64_t)Sl * (G + 1)) {
+    const uint32_t il = (uint32_t)(t / (G + 1)), q = (uint32_t)(t % (G + 1));
     uint32_t acc = 0;
     if (q == G) {
-      acc = cw_cnt[i];
+      acc = cw_cnt[il];
     } else {
-      const uint32_t* r0 = win + (size_t)i * S;
+      const uint32_t* r0 = win_rows + (size_t)il * S;
       const uint32_t* r1 = r0 + S;
       for (uint32_t j = 0; j < bounds[q]; ++j) acc += r1[j] - r0[j];
     }
-    cwp[t] = cw_off[i] + acc;
+    cwp[t] = cw_off_loc[il] + acc;
   }
+}
+template <class T>
+int dcopy(T** dst, const T* src, uint64_t n, cudaStream_t st, std::string& err) {
+  CK(dalloc(dst, n));
+  if (n) CK(cudaMemcpyAsync(*dst, src, n * sizeof(T), cudaMemcpyDeviceToDevice, st));
+  return CUSHA_OK;
 }
 }  // namespace
 
-int build_partition(Graph& g, std::string& err) {
+int build_part(const Graph& glob, const std::vector<uint32_t>& bounds, uint32_t r, Graph& g, bool srcvalue_ipc,
+               std::string& err) {
+  (void)srcvalue_ipc;
   cudaStream_t st = g.stream;
   t_alloc_stream = st;
-  const uint32_t S = g.S, G = g.G;
-  std::vector<uint32_t> cnt(S), ccnt(S);
-  CK(cudaMemcpyAsync(cnt.data(), g.d_shard_cnt, 4ull * S, cudaMemcpyDeviceToHost, st));
-  CK(cudaMemcpyAsync(ccnt.data(), g.d_cw_cnt, 4ull * S, cudaMemcpyDeviceToHost, st));
+  const uint32_t S = glob.S, N = glob.N, V = glob.V, G = (uint32_t)bounds.size() - 1;
+  const uint32_t s0 = bounds[r], s1 = bounds[r + 1], Sl = s1 - s0;
+  std::vector<uint32_t> so(S + 1), co(S + 1), cnt(S);
+  CK(cudaMemcpyAsync(so.data(), glob.d_shard_off, 4ull * (S + 1), cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(co.data(), glob.d_cw_off, 4ull * (S + 1), cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(cnt.data(), glob.d_shard_cnt, 4ull * S, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
-  std::vector<uint64_t> work(S);
-  for (uint32_t s = 0; s < S; ++s) work[s] = (uint64_t)cnt[s] + ccnt[s];  // stage-2 + stage-4 entries
-  g.h_bounds.assign(G + 1, 0);
-  partition_bounds(S, work.data(), G, g.h_bounds.data());
+  g.V = V; g.N = N; g.S = S; g.E = glob.E; g.repr = CUSHA_REPR_CW; g.has_ev = glob.has_ev;
+  g.keep_ids = glob.keep_ids; g.max_indeg = glob.max_indeg; g.max_abs_ev = glob.max_abs_ev;
+  g.G = G; g.part = r; g.h_bounds = bounds;
+  g.s0 = s0; g.Sl = Sl; g.v0 = s0 * N; g.nvl = std::min<uint64_t>(V, (uint64_t)s1 * N) - g.v0;
+  const uint32_t pos0 = so[s0], c0 = co[s0];
+  g.P = so[s1] - pos0;
+  g.Q = co[s1] - c0;
+  g.E_loc = 0;
+  for (uint32_t s = s0; s < s1; ++s) g.E_loc += cnt[s];
+  // host tables: bounds, owner, position bounds of the partitions
   std::vector<uint8_t> owner(S);
-  for (uint32_t q = 0; q < G; ++q)
-    for (uint32_t s = g.h_bounds[q]; s < g.h_bounds[q + 1]; ++s) owner[s] = (uint8_t)q;
+  std::vector<uint32_t> pb(G + 1);
+  for (uint32_t q = 0; q < G; ++q) {
+    pb[q] = so[bounds[q]];
+    for (uint32_t s = bounds[q]; s < bounds[q + 1]; ++s) owner[s] = (uint8_t)q;
+  }
+  pb[G] = so[S];
+  DevBuf dpb;
+  CK(dalloc((uint32_t**)&dpb.p, G + 1));
   CK(dalloc(&g.d_bounds, G + 1));
   CK(dalloc(&g.d_owner, S));
-  CK(dalloc(&g.d_cwp, (uint64_t)S * (G + 1)));
-  CK(dalloc(&g.d_gathered, g.V));
-  CK(cudaMemcpyAsync(g.d_bounds, g.h_bounds.data(), 4ull * (G + 1), cudaMemcpyHostToDevice, st));
+  CK(cudaMemcpyAsync(dpb.p, pb.data(), 4ull * (G + 1), cudaMemcpyHostToDevice, st));
+  CK(cudaMemcpyAsync(g.d_bounds, bounds.data(), 4ull * (G + 1), cudaMemcpyHostToDevice, st));
   CK(cudaMemcpyAsync(g.d_owner, owner.data(), S, cudaMemcpyHostToDevice, st));
-  k_cwp<<<grid_for((uint64_t)S * (G + 1)), 256, 0, st>>>(g.d_win, g.d_cw_off, g.d_cw_cnt, g.d_bounds, S, G, g.d_cwp);
+  // the partition's shards: in-edges of its vertices (positions rebased to 0)
+  CK(dalloc(&g.d_shard_off, (uint64_t)Sl + 1));
+  k_rebase<<<grid_for((uint64_t)Sl + 1), 256, 0, st>>>(glob.d_shard_off + s0, (uint64_t)Sl + 1, pos0, g.d_shard_off);
+  int rc;
+  if ((rc = dcopy(&g.d_shard_cnt, glob.d_shard_cnt + s0, Sl, st, err)) ||
+      (rc = dcopy(&g.d_dest, glob.d_dest + pos0, g.P, st, err)))
+    return rc;
+  if (glob.d_ev && (rc = dcopy(&g.d_ev, glob.d_ev + pos0, g.P, st, err))) return rc;
+  if (glob.d_eid && (rc = dcopy(&g.d_eid, glob.d_eid + pos0, g.P, st, err))) return rc;
+  // window-table rows of its source shards (emptiness tests; positions stay global)
+  if ((rc = dcopy(&g.d_win, glob.d_win + (size_t)s0 * S, ((uint64_t)Sl + 1) * S, st, err))) return rc;
+  // the Concatenated Windows of its source shards, every target partition
+  CK(dalloc(&g.d_cw_off, (uint64_t)Sl + 1));
+  k_rebase<<<grid_for((uint64_t)Sl + 1), 256, 0, st>>>(glob.d_cw_off + s0, (uint64_t)Sl + 1, c0, g.d_cw_off);
+  if ((rc = dcopy(&g.d_cw_cnt, glob.d_cw_cnt + s0, Sl, st, err)) ||
+      (rc = dcopy(&g.d_cw_src, glob.d_cw_src + c0, g.Q, st, err)) ||
+      (rc = dcopy(&g.d_cw_win, glob.d_cw_win + c0, g.Q, st, err)))
+    return rc;
+  CK(dalloc(&g.d_mapper, g.Q));
+  if (g.Q)
+    k_mapper_local<<<grid_for(g.Q), 256, 0, st>>>(glob.d_mapper + c0, g.Q, (const uint32_t*)dpb.p, G, (uint32_t)glob.P,
+                                                  g.d_mapper);
+  CK(dalloc(&g.d_cw_delta, (uint64_t)Sl * S));
+  k_delta_local<<<grid_for((uint64_t)Sl * S), 256, 0, st>>>(glob.d_cw_delta + (size_t)s0 * S, Sl, S, c0,
+                                                             (const uint32_t*)dpb.p, g.d_owner, g.d_cw_delta);
+  CK(dalloc(&g.d_cwp, (uint64_t)Sl * (G + 1)));
+  k_cwp_local<<<grid_for((uint64_t)Sl * (G + 1)), 256, 0, st>>>(g.d_win, g.d_cw_off, g.d_cw_cnt, g.d_bounds, Sl, S, G,
+                                                                  g.d_cwp);
+  if ((rc = dcopy(&g.d_outdeg, glob.d_outdeg + g.v0, g.nvl, st, err))) return rc;
+  CK(dalloc(&g.d_active, Sl));
+  if (g.skip_clean) CK(dalloc(&g.d_dirty, Sl));
+  CK(dalloc(&g.d_shard_seq, Sl));
   CK(cudaGetLastError());
   CK(cudaStreamSynchronize(st));
+  g.splitP = g.P;
+  g.splitQ = g.Q;
+  g.host_shard = Sl;
   return CUSHA_OK;
+}
+
+void free_device_arrays(Graph& g) {
+  void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcloc, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
+                  g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_vv, g.d_ctl, g.d_trace,
+                  g.d_active, g.d_bounds, g.d_owner, g.d_cwp, g.d_run_k, g.d_run_t, g.d_sv_peer, g.d_dirty_peer,
+                  g.d_run_unit, g.d_run_bits, g.d_run_d, g.d_shard_seq, g.d_cw_win, g.d_cw_delta};
+  for (void* p : ptrs)
+    if (p) cudaFreeAsync(p, g.stream);
+  if (g.d_dirty) {
+    if (g.srcvalue_ipc) cudaFree(g.d_dirty);
+    else cudaFreeAsync(g.d_dirty, g.stream);
+  }
+  if (g.d_srcvalue) {
+    if (g.srcvalue_ipc) cudaFree(g.d_srcvalue);  // IPC-exported allocations are not stream-ordered
+    else cudaFreeAsync(g.d_srcvalue, g.stream);
+  }
+  for (void*& p : g.d_init)
+    if (p) { cudaFreeAsync(p, g.stream); p = nullptr; }
+  for (void* p : g.ipc_open) cudaIpcCloseMemHandle(p);
+  g.ipc_open.clear();
+  void* hosts[] = {g.h_dest, g.h_ev, g.h_srcloc, g.h_eid, g.h_cw_src, g.h_mapper, g.h_cw_win};
+  for (void* p : hosts)
+    if (p) cudaFreeHost(p);
+  g.d_shard_off = g.d_shard_cnt = g.d_win = g.d_cw_off = g.d_cw_cnt = g.d_mapper = g.d_outdeg = nullptr;
+  g.d_dest = g.d_srcloc = g.d_cw_src = g.d_cw_win = nullptr;
+  g.d_eid = g.d_ev = g.d_bounds = g.d_cwp = g.d_run_k = g.d_run_t = g.d_run_unit = g.d_run_bits = g.d_run_d = nullptr;
+  g.d_shard_seq = g.d_cw_delta = g.d_dirty = g.d_srcvalue = nullptr;
+  g.d_vv = nullptr; g.d_ctl = nullptr; g.d_trace = nullptr; g.d_active = nullptr; g.d_owner = nullptr;
+  g.d_sv_peer = nullptr; g.d_dirty_peer = nullptr;
+  g.h_dest = nullptr; g.h_ev = nullptr; g.h_srcloc = nullptr; g.h_eid = nullptr; g.h_cw_src = nullptr;
+  g.h_mapper = nullptr; g.h_cw_win = nullptr;
+}
+
+// The library's device memory comes from a private stream-ordered pool per
+// device whose release threshold keeps freed blocks mapped, so that repeated
+// builds (the e2e path) reuse them.  It is private: torch's caching allocator,
+// NCCL and other cudaMalloc users of the process keep the default pool's
+// behaviour.  cusha_trim_memory() returns the unused blocks to the device.
+static cudaError_t pool_of(int dev, cudaMemPool_t* out) {
+  static cudaMemPool_t pools[64] = {};
+  static bool made[64] = {};
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+  if (!made[dev]) {
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    const cudaError_t e = cudaMemPoolCreate(&pools[dev], &props);
+    if (e != cudaSuccess) return e;
+    uint64_t keep = UINT64_MAX;
+    cudaMemPoolSetAttribute(pools[dev], cudaMemPoolAttrReleaseThreshold, &keep);
+    made[dev] = true;
+  }
+  *out = pools[dev];
+  return cudaSuccess;
+}
+
+cudaError_t dev_alloc(void** p, size_t bytes, cudaStream_t s) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  cudaMemPool_t pool;
+  if (e == cudaSuccess) e = pool_of(dev, &pool);
+  if (e != cudaSuccess) return e;
+  return cudaMallocFromPoolAsync(p, bytes ? bytes : 1, pool, s);
+}
+
+cudaError_t trim_pool(int dev) {
+  cudaMemPool_t pool;
+  cudaError_t e = pool_of(dev, &pool);
+  if (e == cudaSuccess) e = cudaMemPoolTrimTo(pool, 0);
+  return e;
 }
 
 }  // namespace cusha

@@ -20,8 +20,8 @@ struct Ctl {
   uint32_t max_iters;
   uint32_t converged;   // 1 once a pass committed nothing
   uint32_t next_shard;  // dynamic shard queue of the persistent pass
-  uint32_t gchanged;    // partitioned mode: some shard of any partition was active (refresh kernel)
-  uint32_t rctas_done;  // partitioned mode: refresh-kernel arrival counter
+  uint32_t lchanged;    // partitioned mode: this partition's last pass committed an update
+  uint32_t gchanged;    // partitioned mode: OR of lchanged over the partitions (NCCL all-reduce / simulation)
   // overlapped passes (one launch per run)
   unsigned long long ticket;  // shard tickets drawn: ticket t = shard t % |S| of pass t / |S|
   uint32_t stop;              // two consecutive passes committed nothing: draw no more tickets
@@ -41,42 +41,45 @@ struct TraceRec {
 };
 
 // Everything a shard-pass launch needs (passed by value).
+// Arrays of one partition are indexed by the LOCAL shard index sl = s - s0
+// (shard s is global; partition = shards [s0, s0 + Sl), vertices [s0*N,
+// min(V, (s0+Sl)*N))); a single GPU is the partition s0 = 0, Sl = S.
 struct KParams {
   uint32_t V, N, S, source;
-  const uint32_t* shard_off;   // S+1 padded start positions
-  const uint32_t* shard_cnt;   // S real entry counts
+  uint32_t s0, Sl;             // first shard and number of shards of this partition
+  const uint32_t* shard_off;   // Sl+1 padded start positions (local positions)
+  const uint32_t* shard_cnt;   // Sl real entry counts
   const uint16_t* dest;        // P local DestIndex (filler = N)
   const uint32_t* ev;          // P EdgeValue or null
-  uint32_t* srcvalue;          // P+1 (slot P = trash for CW filler)
+  uint32_t* srcvalue;          // P+1 SrcValue of this partition's shard entries
+  uint32_t* const* sv_peer;    // G: SrcValue of every partition (sv_peer[own] = srcvalue); stage 4 of a
+                               // source shard stores into the partition that owns each window's target
   const uint16_t* srcloc;      // GS: P SrcIndex - (source shard)*N
-  const uint32_t* win;         // GS: (S+1)*S window starts
-  const uint32_t* cw_off;      // CW: S+1 padded CW_i starts
-  const uint32_t* cw_cnt;      // S real |CW_i| (both reprs; = entries stage 4 of shard i visits)
-  uint8_t* active;             // S: shard ran stage 4 in the last pass (stage-4 prefetch predictor; exchanged)
+  const uint32_t* win;         // (Sl+1)*S window starts: rows s0..s0+Sl of the window table (GS walk, skip marks)
+  const uint32_t* cw_off;      // CW: Sl+1 padded CW_i starts (own source shards i)
+  const uint32_t* cw_cnt;      // Sl real |CW_i| (both reprs; = entries stage 4 of shard i visits)
+  uint8_t* active;             // Sl: shard ran stage 4 in the last pass (stage-4 prefetch predictor)
   const uint16_t* cw_src;      // CW: Q local SrcIndex
-  const uint32_t* mapper;      // CW: Q padded shard positions
+  const uint32_t* mapper;      // CW: Q target positions in the owning partition's SrcValue
   const uint16_t* cw_win;      // CW: Q target shard j of each entry (filler: 0xFFFF)
-  const uint32_t* cw_delta;    // CW: S*S, Mapper[k] = cw_delta[i*S + j] + k for k in W_ij's part of CW_i
-  void* vv;                    // VertexValues
-  const uint32_t* outdeg;      // V out-degrees (PR NbrsNum)
+  const uint32_t* cw_delta;    // CW: Sl*S, Mapper[k] = cw_delta[il*S + j] + k for k in W_ij's part of CW_i
+  void* vv;                    // VertexValues of the partition's vertices (local index (s - s0)*N + v)
+  const uint32_t* outdeg;      // out-degrees of the partition's vertices (PR NbrsNum)
   Ctl* ctl;
   TraceRec* trace;
   uint32_t trace_cap;
-  int use_cond;
-  unsigned long long cond_handle;
   int multi;                   // 1: one launch runs every pass (overlapped passes)
   int mapj;                    // 1: CW stage 4 uses the Mapper in window form (cw_win + delta row in smem)
   int stash;                   // 1: integer algorithms keep stage 1's VertexValues in smem for stage 3
   int ahead;                   // 1: the producer prefetches stage-2 tiles into L2 beyond the ring (HBM-resident passes)
   uint32_t nst;                // ring slots of this run (kStages, or more when shared memory has room)
-  uint32_t* shard_seq;         // S: passes of shard s completed (overlapped passes)
+  uint32_t* shard_seq;         // Sl: passes of shard s completed (overlapped passes)
   // destination-range partition (row e); G = 1: single partition
   uint32_t G;                  // partitions
-  int part;                    // partition this launch processes (-1: all, the single-process simulation)
   const uint32_t* bounds;      // G+1 shard bounds of the partitions
-  const uint8_t* owner;        // S: partition owning shard s
-  const uint32_t* cwp;         // S*(G+1): CW_i entries whose targets lie in partition p = [cwp[i][p], cwp[i][p+1])
-  uint32_t* gathered;          // V: write-back value of every vertex after its last pass (exchanged)
+  const uint8_t* owner;        // S: partition owning shard j
+  const uint32_t* cwp;         // Sl*(G+1): CW_i entries whose targets lie in partition q = [cwp[il][q], cwp[il][q+1])
+  uint32_t* const* dirty_peer; // G: dirty[] of every partition (clean-shard skipping marks remote shards)
   // Mapper in run-length form (CW): one run per non-empty window
   const uint32_t* run_k;       // R (+pad): CW position of each run's first entry (sorted)
   const uint32_t* run_t;       // R (+pad): target shard position of that entry
@@ -86,7 +89,7 @@ struct KParams {
   uint32_t R;
   // opt-in exact work skipping
   int skip;                    // 1: a shard none of whose windows was written since its last pass is skipped
-  uint32_t* dirty;             // S: some window of shard j written since j's last pass (set by writers)
+  uint32_t* dirty;             // Sl: some window of shard j written since j's last pass (set by writers)
   // host-streamed topology (row f3): entries at shard
   // positions >= splitP / CW positions >= splitQ live in pinned host memory
   // (x_h[i - split]); below the split, in HBM (x[i]).  splitP = P, splitQ = Q: all in HBM.
@@ -118,28 +121,37 @@ struct PassKernel {
   size_t smem_bytes(uint32_t N, uint32_t delta_row = 0) const;  // delta_row: words of the window-form row
 };
 
+// One partition's device state (row a0 layout + per-run arrays).  A single
+// GPU holds one partition covering every shard (s0 = 0, Sl = S); the
+// destination-range partition of row e gives each rank (or, in the one-process
+// simulation, each sub-graph) shards [s0, s0 + Sl) and their in-edges, plus the
+// Concatenated Windows of its own SOURCE shards, whose Mapper targets are
+// positions in the SrcValue array of the partition that owns each window.
 struct Graph {
   // topology
-  uint32_t V = 0, N = 0, S = 0;
-  uint64_t E = 0, P = 0, Q = 0;
+  uint32_t V = 0, N = 0, S = 0;     // global |V|, |N|, |S|
+  uint64_t E = 0, P = 0, Q = 0;     // E: global |E|; P, Q: this partition's padded shard / CW entries
+  uint32_t s0 = 0, Sl = 0;          // owned shards [s0, s0 + Sl)
+  uint32_t v0 = 0, nvl = 0;         // owned vertices [v0, v0 + nvl)
+  uint64_t E_loc = 0;               // real in-edges of the owned shards
   int repr = 0, device = 0;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
   bool has_ev = false;
-  uint32_t* d_shard_off = nullptr;  // S+1
-  uint32_t* d_shard_cnt = nullptr;  // S
+  bool keep_ids = false;            // keep the input edge index per entry (layout inspection only)
+  uint32_t* d_shard_off = nullptr;  // Sl+1
+  uint32_t* d_shard_cnt = nullptr;  // Sl
   uint16_t* d_dest = nullptr;       // P
   uint16_t* d_srcloc = nullptr;     // P (GS): SrcIndex local to its source shard
-  uint32_t* d_eid = nullptr;        // P
+  uint32_t* d_eid = nullptr;        // P (only with keep_ids)
   uint32_t* d_ev = nullptr;         // P (if has_ev)
-  uint32_t* d_win = nullptr;        // (S+1)*S (GS)
-  uint32_t* d_cw_off = nullptr;     // S+1
-  uint32_t* d_cw_cnt = nullptr;     // S
-  uint8_t* d_active = nullptr;      // S: stage-4 prefetch predictor
-  uint32_t* d_dirty = nullptr;      // S: clean-shard skipping flags
-  uint32_t* d_shard_seq = nullptr;  // S: overlapped passes, per-shard pass order
-  int pass_barrier = 0;             // 0: automatic, 1: one launch per pass (CUDA-graph while loop), 2: overlapped
-  int mapj = -1;                    // per-run choice of the Mapper form (-1: not chosen yet)
+  uint32_t* d_win = nullptr;        // (Sl+1)*S: rows s0..s0+Sl of the window table
+  uint32_t* d_cw_off = nullptr;     // Sl+1
+  uint32_t* d_cw_cnt = nullptr;     // Sl
+  uint8_t* d_active = nullptr;      // Sl: stage-4 prefetch predictor
+  uint32_t* d_dirty = nullptr;      // Sl: clean-shard skipping flags
+  uint32_t* d_shard_seq = nullptr;  // Sl: overlapped passes, per-shard pass order
+  int pass_barrier = 0;             // 0: automatic, 1: one launch per pass, 2: overlapped
   bool skip_clean = false;
   // host-streamed topology (row f3): shards >= host_shard keep their entry
   // arrays (and CW_i arrays) in pinned, mapped host memory
@@ -156,19 +168,23 @@ struct Graph {
   uint16_t* d_cw_src = nullptr;     // Q (CW)
   uint32_t* d_mapper = nullptr;     // Q (CW)
   uint16_t* d_cw_win = nullptr;     // Q (CW): target shard of each entry (Mapper in window form)
-  uint32_t* d_cw_delta = nullptr;   // S*S (CW): Mapper - CW position, per window
+  uint32_t* d_cw_delta = nullptr;   // Sl*S (CW): Mapper - CW position, per window
   uint16_t* h_cw_win = nullptr;     // Q - splitQ (row f3)
-  uint32_t R = 0;                   // Mapper runs (non-empty windows)
+  uint32_t R = 0;                   // Mapper runs (non-empty windows; CUSHA_RLE builds only)
   uint32_t* d_run_k = nullptr;      // R+pad
   uint32_t* d_run_t = nullptr;      // R+pad
   uint32_t* d_run_unit = nullptr;   // Q/kRunUnit+2
   uint32_t* d_run_bits = nullptr;   // Q/32 + pad
   uint32_t* d_run_d = nullptr;      // R+pad
-  uint32_t* d_outdeg = nullptr;     // V
+  uint32_t* d_outdeg = nullptr;     // nvl
+  uint32_t max_indeg = 0;           // largest in-degree (fixed-point range check)
+  float max_abs_ev = 0.f;           // largest |EdgeValue| read as f32 (fixed-point range check)
   // per-run state
   uint32_t* d_srcvalue = nullptr;   // P+1
-  void* d_vv = nullptr;             // V * 8 bytes
-  void* d_init[8] = {};             // user initial values per algorithm
+  bool srcvalue_ipc = false;        // allocated with cudaMalloc (exported to the other ranks)
+  void* d_vv = nullptr;             // nvl * 8 bytes
+  void* d_init[8] = {};             // user initial values per algorithm (this partition's slice)
+  float init_max_abs[8] = {};       // largest |initial value| given per algorithm
   Ctl* d_ctl = nullptr;
   TraceRec* d_trace = nullptr;
   uint32_t trace_cap = 0;
@@ -177,13 +193,15 @@ struct Graph {
   cudaEvent_t ev0 = nullptr, ev1 = nullptr, evm = nullptr;
   // destination-range partition (row e)
   int world_size = 1, rank = 0;
-  bool simulate = false;            // all partitions in this process, exchange through device memory
-  uint32_t G = 1;
+  uint32_t G = 1;                   // partitions (1: unpartitioned)
+  uint32_t part = 0;                // this partition's index
   std::vector<uint32_t> h_bounds;   // G+1 shard bounds
-  uint32_t* d_bounds = nullptr;
+  uint32_t* d_bounds = nullptr;     // G+1
   uint8_t* d_owner = nullptr;       // S
-  uint32_t* d_cwp = nullptr;        // S*(G+1)
-  uint32_t* d_gathered = nullptr;   // V
+  uint32_t* d_cwp = nullptr;        // Sl*(G+1)
+  uint32_t** d_sv_peer = nullptr;   // G: SrcValue of every partition (device pointers valid on this device)
+  uint32_t** d_dirty_peer = nullptr;// G: dirty[] of every partition (skip_clean only)
+  std::vector<void*> ipc_open;      // peer allocations mapped with cudaIpcOpenMemHandle
   void* nccl_comm = nullptr;        // ncclComm_t (real multi-GPU)
   // stats
   cusha_stats st{};
@@ -196,7 +214,7 @@ struct Graph {
 const PassKernel& pass_kernel(int alg, int repr);
 cudaError_t launch_init(const Graph& g, int alg, uint32_t source, cudaStream_t s);
 cudaError_t launch_reset_ctl(Ctl* ctl, uint32_t max_iters, cudaStream_t s);
-cudaError_t launch_refresh(const Graph& g, cudaStream_t s);
+cudaError_t launch_close_parts(Ctl* const* ctls, uint32_t G, cudaStream_t s);  // partitioned: global convergence
 KParams make_params(const Graph& g, uint32_t source);
 size_t value_bytes(int alg);
 int timeline_copy(void* out, size_t bytes);  // CUSHA_TIMELINE builds: per-ticket stamps (else -1)
@@ -207,18 +225,27 @@ bool alg_needs_init(int alg);
 
 // builder.cu
 int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const uint32_t* d_val, std::string& err);
-int build_partition(Graph& g, std::string& err);  // bounds, owner, cwp, gathered (G > 1)
-int build_runs(Graph& g, std::string& err);       // Mapper runs (CW)
+int build_runs(Graph& g, std::string& err);       // Mapper runs (CW, CUSHA_RLE builds)
 int offload_topology(Graph& g, std::string& err); // row f3: move shards >= host_shard to pinned host memory
 void partition_bounds(uint32_t S, const uint64_t* work, uint32_t G, uint32_t* bounds);
+int partition_work(const Graph& glob, std::vector<uint64_t>& work, std::string& err);
+// the partition r of a global layout (bounds: G+1 shard bounds); srcvalue_ipc:
+// SrcValue by cudaMalloc (exportable) instead of the stream-ordered pool
+int build_part(const Graph& glob, const std::vector<uint32_t>& bounds, uint32_t r, Graph& part, bool srcvalue_ipc,
+               std::string& err);
+void free_device_arrays(Graph& g);  // every device / pinned array of g (not its stream or events)
+cudaError_t dev_alloc(void** p, size_t bytes, cudaStream_t s);  // the library's private stream-ordered pool
+cudaError_t trim_pool(int dev);                                  // release its unused blocks
 
 // api.cu
 void set_error(const std::string& msg);
 
-// nccl.cpp (loaded at run time; no link-time NCCL dependency)
+// nccl.cu (loaded at run time; no link-time NCCL dependency)
 int nccl_unique_id(void* out128, std::string& err);
 int nccl_init(Graph& g, const void* id128, std::string& err);
-int nccl_exchange(Graph& g, uint32_t value_bytes_vv, bool final_values, std::string& err);
+int nccl_allgather_bytes(Graph& g, const void* dsend, void* drecv, size_t bytes, std::string& err);
+int nccl_allreduce_max_u32(Graph& g, const uint32_t* dsend, uint32_t* drecv, std::string& err);
+int nccl_gather_values(Graph& g, void* dfull, uint32_t value_bytes, std::string& err);  // every rank's vv slice
 void nccl_destroy(Graph& g);
 
 }  // namespace cusha

@@ -7,6 +7,10 @@
 // while-condition, instead of the paper's
 // per-iteration cudaMemcpy of is_converged (L189).
 //
+// Arrays of the partition (a single GPU is one partition, s0 = 0, Sl = S) are
+// indexed by the local shard index sl; shard s0 + sl owns global vertices
+// [(s0 + sl)*N, ...), held locally at sl*N.
+//
 // B200 structure: a persistent grid (a few CTAs per
 // SM).  In each CTA one producer thread takes shards from a global queue in
 // shard order and streams, with the TMA engine (cp.async.bulk), every tile
@@ -184,7 +188,7 @@ enum : uint32_t { kFlagLast = 1, kFlagSpec4 = 2 };
 // copied into the slot; [lo, hi) = the entries the consumers use; base = CW
 // position of entry 0 of the slot; nruns = runs in the slot (kDescStage4R).
 struct __align__(16) TileDesc {
-  uint32_t shard, kind, n, flags, lo, hi, base, nruns, pass;
+  uint32_t shard, kind, n, flags, lo, hi, base, nruns, pass, tgt;  // tgt: partition receiving a stage-4 tile's stores
 };
 
 // ------------------------------------------------ overlapped passes (row a5)
@@ -211,13 +215,22 @@ __device__ __forceinline__ uint32_t ld_vol(const uint32_t* a) { return *reinterp
 __device__ __forceinline__ void st_vol(uint32_t* a, uint32_t v) { *reinterpret_cast<volatile uint32_t*>(a) = v; }
 __device__ __forceinline__ void fence_sc_gpu() { asm volatile("fence.sc.gpu;" ::: "memory"); }
 
-// the producer's waits before ticket (s, pass) may read anything
-__device__ __forceinline__ void ticket_wait(const KParams& p, uint32_t s, uint32_t pass, uint32_t Sloc) {
-  while (ld_vol(&p.shard_seq[s]) < pass) __nanosleep(64);
+// the producer's waits before ticket (s, pass) may read anything; false: the
+// run stopped meanwhile (the ticket is abandoned - every waiting ticket polls
+// stop, so an abandoned ticket never leaves another one waiting for it)
+__device__ __forceinline__ bool ticket_wait(const KParams& p, uint32_t s, uint32_t pass, uint32_t Sloc) {
+  while (ld_vol(&p.shard_seq[s]) < pass) {
+    if (ld_vol(&p.ctl->stop)) return false;
+    __nanosleep(64);
+  }
   if (pass >= 2)
-    while (ld_vol(&p.trace[pass - 2].done) < Sloc) __nanosleep(64);
+    while (ld_vol(&p.trace[pass - 2].done) < Sloc) {
+      if (ld_vol(&p.ctl->stop)) return false;
+      __nanosleep(64);
+    }
   __threadfence();                                      // acquire the completed passes' stores ...
   asm volatile("fence.proxy.async.global;" ::: "memory");  // ... for the TMA (async-proxy) reads too
+  return true;
 }
 
 // ticket (s, pass) finished (its stores ordered before by the caller's
@@ -230,7 +243,9 @@ __device__ __forceinline__ void ticket_done(const KParams& p, uint32_t s, uint32
   fence_sc_gpu();  // pairs with the other neighbour's completer: at least one of two sees both complete
   if (ld_vol(&p.trace[pass].active_shards) != 0) return;
   auto clean = [&](uint32_t r) {
-    return ld_vol(&p.trace[r].done) == Sloc && ld_vol(&p.trace[r].active_shards) == 0;
+    if (ld_vol(&p.trace[r].done) != Sloc) return false;
+    __threadfence();  // acquire: the completers' active_shards increments precede their done increments
+    return ld_vol(&p.trace[r].active_shards) == 0;
   };
   uint32_t conv = 0xFFFFFFFFu;
   if (pass >= 1 && clean(pass - 1)) conv = pass + 1;
@@ -367,6 +382,10 @@ __device__ __forceinline__ void gs_walk(const KParams& p, uint32_t s, uint32_t l
 // Per shard: its stage-2 tiles, then — for CW — its stage-4 tiles, either
 // right away (shard predicted active: prefetch overlaps stage 3) or once the
 // consumers' stage 3 has decided values_updated (decide_bar / s_any).
+// Stage-4 tiles are cut per target partition q (CW_s lists W_s0, W_s1, ... in
+// j order, L175, and partitions are contiguous j ranges, so the entries aimed
+// at partition q are one contiguous segment): a tile's stores all go to
+// sv_peer[q], the partition that owns its windows (one segment on one GPU).
 template <class A, int REPR>
 __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDesc* desc, uint64_t* full_bar,
                                          uint64_t* empty_bar, uint64_t* decide_bar, const volatile int* s_any) {
@@ -378,9 +397,9 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
   auto push = [&](uint32_t shard, uint32_t kind, uint32_t n, uint32_t flags, const void* g0, uint32_t b0,
                   const void* g1, uint32_t o1, uint32_t b1, const void* g2, uint32_t o2, uint32_t b2,
                   uint32_t lo = 0, uint32_t hi = 0xFFFFFFFFu, uint32_t base = 0, uint32_t nruns = 0,
-                  const void* g3 = nullptr, uint32_t o3 = 0, uint32_t b3 = 0) {
+                  const void* g3 = nullptr, uint32_t o3 = 0, uint32_t b3 = 0, uint32_t tgt = 0) {
     mbar_wait(&empty_bar[slot], ph ^ 1);
-    desc[slot] = TileDesc{shard, kind, n, flags, lo, hi == 0xFFFFFFFFu ? n : hi, base, nruns, cur_pass};
+    desc[slot] = TileDesc{shard, kind, n, flags, lo, hi == 0xFFFFFFFFu ? n : hi, base, nruns, cur_pass, tgt};
     uint8_t* buf = ring + slot * SLOT;
     const uint32_t bytes = b0 + b1 + b2 + b3;
     if (bytes) {
@@ -406,9 +425,7 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     }
     if (++slot == p.nst) { slot = 0; ph ^= 1; }
   };
-  // shards of this launch: one partition's range (multi-GPU) or all of them
-  const uint32_t q_lo = p.part >= 0 ? p.bounds[p.part] : 0u, q_hi = p.part >= 0 ? p.bounds[p.part + 1] : p.S;
-  const uint32_t Sloc = q_hi - q_lo;
+  const uint32_t Sloc = p.Sl;
   // L2 prefetch of stage-2 tile [t0, t0 + kTile) of a shard ending at e (device-resident parts only)
   auto pf2 = [&](uint32_t t0, uint32_t e) {
     if (t0 >= e) return;
@@ -427,34 +444,47 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     if (p.mapj) bulk_prefetch_l2(p.cw_win + k0, n * 2);
     else bulk_prefetch_l2(p.mapper + k0, n * 4);
   };
+  // CW_s's segment aimed at partition q: [*a, *b)
+  auto segment = [&](uint32_t s, uint32_t q, uint32_t* a, uint32_t* b) {
+    if (p.G > 1) {
+      const uint32_t* row = p.cwp + (size_t)s * (p.G + 1);
+      *a = row[q];
+      *b = row[q + 1];
+    } else {
+      *a = p.cw_off[s];
+      *b = *a + p.cw_cnt[s];
+    }
+  };
   // tiles prefetched into L2 beyond the ring, when the pass streams from HBM (KParams::ahead)
   const uint32_t ahead = p.ahead ? CUSHA_AHEAD : 0u;
   for (uint32_t round = 0;; ++round) {
-    uint32_t s;
+    uint32_t s;  // local shard index
     if (p.multi) {
       // overlapped passes: the next ticket, whatever pass it belongs to
       bool over = ld_vol(&p.ctl->stop) != 0;
       if (!over) {
         const unsigned long long t = atomicAdd(&p.ctl->ticket, 1ull);
         cur_pass = (uint32_t)(t / Sloc);
-        s = q_lo + (uint32_t)(t - (unsigned long long)cur_pass * Sloc);
+        s = (uint32_t)(t - (unsigned long long)cur_pass * Sloc);
         over = cur_pass >= p.ctl->max_iters || ld_vol(&p.ctl->stop) != 0;
         if (CUSHA_TIMELINE && !over) tl_mark((uint32_t)t, 0);
+      }
+      if (!over) {
+        // the shard's first stage-2 tiles start towards L2 while the producer
+        // waits (a prefetch reads nothing into the CTA, so it needs no ordering)
+        if (CUSHA_AHEAD_WAIT && ahead)
+          for (uint32_t j = 0; j <= ahead; ++j) pf2(p.shard_off[s] + j * kTile, p.shard_off[s + 1]);
+        over = !ticket_wait(p, s, cur_pass, Sloc);
       }
       if (over) {
         push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
         return;
       }
-      // the shard's first stage-2 tiles start towards L2 while the producer
-      // waits (a prefetch reads nothing into the CTA, so it needs no ordering)
-      if (CUSHA_AHEAD_WAIT && ahead)
-        for (uint32_t j = 0; j <= ahead; ++j) pf2(p.shard_off[s] + j * kTile, p.shard_off[s + 1]);
-      ticket_wait(p, s, cur_pass, Sloc);
-      if (CUSHA_TIMELINE) tl_mark(cur_pass * Sloc + (s - q_lo), 1);
+      if (CUSHA_TIMELINE) tl_mark(cur_pass * Sloc + s, 1);
     } else {
-      // persistent grid: shards from the global queue; otherwise CTA b runs shard q_lo + b only
-      s = q_lo + (kPersistent ? atomicAdd(&p.ctl->next_shard, 1u) : (round == 0 ? blockIdx.x : q_hi));
-      if (s >= q_hi) {
+      // persistent grid: shards from the global queue; otherwise CTA b runs shard b only
+      s = kPersistent ? atomicAdd(&p.ctl->next_shard, 1u) : (round == 0 ? blockIdx.x : Sloc);
+      if (s >= Sloc) {
         push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
         return;
       }
@@ -478,26 +508,24 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     if (CUSHA_PF == 1) {
       // the consumers' global reads of this shard (stage 1/3 VertexValues and
       // NbrsNum, the stage-4 delta row) become L2 hits: one TMA prefetch each
-      const uint32_t off = s * p.N, nv = min(p.N, p.V - off);
+      const uint32_t off = s * p.N, nv = min(p.N, p.V - (p.s0 + s) * p.N);
       bulk_prefetch_l2(reinterpret_cast<const typename A::Value*>(p.vv) + off, nv * (uint32_t)sizeof(typename A::Value));
       if (A::kOutDeg) bulk_prefetch_l2(p.outdeg + off, nv * 4);
       if (REPR == CUSHA_REPR_CW && p.mapj) bulk_prefetch_l2(p.cw_delta + (size_t)s * p.S, p.S * 4);
     }
-    // CW_s entries whose targets lie in the shard's own partition: all of CW_s
-    // on one GPU; with G partitions the other windows are refreshed after the
-    // exchange.  Stage-4 tiles are 8-entry aligned for TMA.
-    uint32_t a = 0, b2 = 0;
+    // first / last non-empty stage-4 segment of CW_s (stage-4 tiles are 8-entry aligned for TMA)
+    uint32_t qa = 0, qz = 0, a0 = 0, b0 = 0;
     if (REPR == CUSHA_REPR_CW) {
-      if (p.G > 1) {
-        const uint32_t o = p.owner[s];
-        a = p.cwp[(size_t)s * (p.G + 1) + o];
-        b2 = p.cwp[(size_t)s * (p.G + 1) + o + 1];
-      } else {
-        a = p.cw_off[s];
-        b2 = a + p.cw_cnt[s];
+      for (uint32_t q = 0; q < p.G; ++q) {
+        uint32_t x, y;
+        segment(s, q, &x, &y);
+        if (x < y) {
+          if (qz == 0) { qa = q; a0 = x; }
+          qz = q + 1;
+          b0 = y;
+        }
       }
     }
-    const uint32_t kb = a & ~7u, ke = (b2 + 7u) & ~7u;
     if (b == e) push(s, kDescStage2, 0, kFlagLast | (spec ? kFlagSpec4 : 0u), nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
     if (!(CUSHA_AHEAD_WAIT && p.multi))
       for (uint32_t j = 1; j <= ahead; ++j) pf2(b + j * kTile, e);
@@ -509,7 +537,7 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
            A::kEdge ? n * 4 : 0u);
       if (ahead) {
         if (t0 + (ahead + 1) * kTile < e) pf2(t0 + (ahead + 1) * kTile, e);
-        else if (CUSHA_AHEAD4 && spec && t0 + kTile >= e && a < b2) pf4(kb, ke);  // the first stage-4 tile
+        else if (CUSHA_AHEAD4 && spec && t0 + kTile >= e && qz) pf4(a0 & ~7u, (b0 + 7u) & ~7u);  // the first stage-4 tile
       }
     }
     bool send4 = spec;
@@ -521,11 +549,16 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     if (send4) {
       // [lo, hi) marks the valid part of each tile
       const uint32_t kT4 = p.mapj ? tile4j_of<A>() : tile4m_of<A>();
-      if (a >= b2) push(s, kDescStage4, 0, kFlagLast, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
-      else
+      if (qz == 0) push(s, kDescStage4, 0, kFlagLast, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
+      for (uint32_t q = qa; q < qz; ++q) {
+        uint32_t a, b2;
+        segment(s, q, &a, &b2);
+        if (a >= b2) continue;
+        const uint32_t kb = a & ~7u, ke = (b2 + 7u) & ~7u;
         for (uint32_t k0 = kb; k0 < ke; k0 += kT4) {
           const uint32_t n = min(kT4, ke - k0);
-          const uint32_t fl = k0 + n >= ke ? kFlagLast : 0u, lo = a > k0 ? a - k0 : 0u, hi = min(b2 - k0, n);
+          const uint32_t fl = (k0 + n >= ke && q + 1 == qz) ? kFlagLast : 0u, lo = a > k0 ? a - k0 : 0u,
+                         hi = min(b2 - k0, n);
           if (kRle) {
             // runs from the one containing position k0/128*128 (the slot's first
             // bitmap position) through the last starting inside the tile; the
@@ -538,18 +571,21 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
               const uint32_t wa = k0 / 128 * 4, wz = (k0 + n + 127) / 128 * 4;
               push(s, kDescStage4R, n, fl | ((ra - ra4) << 8), topo_at(p.cw_src, p.cw_src_h, p.splitQ, k0), n * 2,
                    p.run_d + ra4, 2 * kTile,
-                   nr * 4, p.run_bits + wa, 2 * kTile + 4 * kRunCap, (wz - wa) * 4, lo, hi, k0, nr);
+                   nr * 4, p.run_bits + wa, 2 * kTile + 4 * kRunCap, (wz - wa) * 4, lo, hi, k0, nr, nullptr, 0, 0, q);
               continue;
             }
           }
           if (p.mapj)
             push(s, kDescStage4, n, fl, topo_at(p.cw_src, p.cw_src_h, p.splitQ, k0), n * 2,
-                 topo_at(p.cw_win, p.cw_win_h, p.splitQ, k0), 2 * kT4, n * 2, nullptr, 0, 0, lo, hi, k0, 0);
+                 topo_at(p.cw_win, p.cw_win_h, p.splitQ, k0), 2 * kT4, n * 2, nullptr, 0, 0, lo, hi, k0, 0,
+                 nullptr, 0, 0, q);
           else
             push(s, kDescStage4, n, fl, topo_at(p.cw_src, p.cw_src_h, p.splitQ, k0), n * 2,
-                 topo_at(p.mapper, p.mapper_h, p.splitQ, k0), 2 * kT4, n * 4, nullptr, 0, 0, lo, hi, k0, 0);
+                 topo_at(p.mapper, p.mapper_h, p.splitQ, k0), 2 * kT4, n * 4, nullptr, 0, 0, lo, hi, k0, 0,
+                 nullptr, 0, 0, q);
           if (CUSHA_AHEAD4 && ahead) pf4(k0 + kT4, ke);
         }
+      }
     }
   }
 }
@@ -610,7 +646,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
   const uint32_t it0 = *reinterpret_cast<volatile uint32_t*>(&p.ctl->iter);
   // a pass launched after the run converged / hit max_iters is a no-op (host-loop mode)
   if (*reinterpret_cast<volatile uint32_t*>(&p.ctl->converged) || it0 >= p.ctl->max_iters) return;
-  const uint32_t Sloc = p.part >= 0 ? p.bounds[p.part + 1] - p.bounds[p.part] : p.S;
+  const uint32_t Sloc = p.Sl;
   if (tid == 0) {
     for (uint32_t i = 0; i < nst; ++i) {
       mbar_init(&full_bar[i], 1);                // the producer's arrive(.expect_tx)
@@ -635,13 +671,13 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
       mbar_wait(&full_bar[slot], ph);
       TileDesc d = desc[slot];
       if (d.kind == kDescDone) break;
-      const uint32_t s = d.shard;
+      const uint32_t s = d.shard;                  // local shard index (global p.s0 + s)
       const uint32_t it = p.multi ? d.pass : it0;  // the pass this shard belongs to
       const bool spec4 = d.flags & kFlagSpec4;
-      const uint32_t off = s * N;
-      const uint32_t nv = min(N, p.V - off);
+      const uint32_t off = s * N;                  // local vertex offset of the shard
+      const uint32_t nv = min(N, p.V - (p.s0 + s) * N);
       V_t* vv = reinterpret_cast<V_t*>(p.vv) + off;
-      const uint32_t tk = it * Sloc + (s - (p.part >= 0 ? p.bounds[p.part] : 0u));  // timeline ticket
+      const uint32_t tk = it * Sloc + s;            // timeline ticket
       if (CUSHA_TIMELINE && ct == 0) { tl_mark(tk, 2); tl_mark(tk, 8, blockIdx.x); tl_mark(tk, 9, spec4 ? 1u : 0u); }
 
       // ---- stage 1: local_vertices <- init_compute(VertexValues) (Fig. 5 lines 8-10, L267)
@@ -741,8 +777,6 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
             up = A::update(sm, st, v, x[u], &out, &wbv, od[u]);
             if (up) vv[v] = out;
             if (!A::kMonotone) aux[v] = wbv;
-            // partitioned mode: publish the value stage 4 writes (the exchange payload)
-            if (p.gathered) p.gathered[off + v] = A::kMonotone ? sm[v] : wbv;
           }
           const uint32_t m = __ballot_sync(kFull, up);
           if (lane == 0 && m) atomicAdd(&s_upd, (uint32_t)__popc(m));
@@ -760,7 +794,6 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
         // thread per CW_s entry: SrcValue[Mapper[k]] = local[SrcIndex[k]] (L177, Fig. 4b);
         // consecutive threads take consecutive entries, so the stores of one
         // window (consecutive Mapper targets) coalesce into whole sectors
-        const uint32_t trash = p.shard_off[p.S];
         if (!spec4 && ct == 0) {  // tell the producer whether CW_s's tiles are needed
           s_any = any;
           mbar_arrive(&decide_bar);
@@ -769,6 +802,9 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
           for (;;) {
             mbar_wait(&full_bar[slot], ph);
             d = desc[slot];
+            // the partition owning this tile's windows (this one on a single GPU):
+            // in the multi-GPU mode the stores below go over NVLink to its SrcValue
+            uint32_t* const svq = p.G > 1 ? p.sv_peer[d.tgt] : p.srcvalue;
             if (any && d.kind == kDescStage4R) {
               // Mapper from runs: target(k) = k + D[r], D = RunT - RunK, for the run r
               // containing CW position k.  Runs start where the run-start bitmap has
@@ -801,7 +837,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
                   const uint32_t k = sp + lane;
                   uint32_t val;
                   if (k >= alo && k < ahi && wb_get<A>(sm, aux, L[k - d.base], val)) {
-                    st_u32(p.srcvalue + (k + D[ri]), val);
+                    st_u32(svq + (k + D[ri]), val);
                     ++stores;
                   }
                   r += __popc(word);
@@ -824,7 +860,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
                 }
 #pragma unroll
                 for (uint32_t u = 0; u < kS4U; ++u)
-                  if (ok[u]) { st_u32(p.srcvalue + tg[u], val[u]); ++stores; }
+                  if (ok[u]) { st_u32(svq + tg[u], val[u]); ++stores; }
               }
             } else if (any) {
               const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
@@ -835,16 +871,16 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
 #pragma unroll
                 for (uint32_t u = 0; u < kS4U; ++u) {
                   const uint32_t i = i0 + u * kConsumers;
-                  tg[u] = i < d.hi ? M[i] : trash;
-                  ok[u] = tg[u] != trash && wb_get<A>(sm, aux, L[i], val[u]);
+                  tg[u] = i < d.hi ? M[i] : 0u;
+                  ok[u] = i < d.hi && wb_get<A>(sm, aux, L[i], val[u]);
                 }
 #pragma unroll
                 for (uint32_t u = 0; u < kS4U; ++u)
                   if (ok[u]) {
                     if (kDiag & 4) {
-                      if (val[u] == 0x9e3779b9u && tg[u] == 7u) st_u32(p.srcvalue + tg[u], val[u]);  // keep the loads
+                      if (val[u] == 0x9e3779b9u && tg[u] == 7u) st_u32(svq + tg[u], val[u]);  // keep the loads
                     } else {
-                      st_u32(p.srcvalue + tg[u], val[u]);
+                      st_u32(svq + tg[u], val[u]);
                     }
                     ++stores;
                   }
@@ -878,7 +914,14 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
         const uint32_t* w0 = p.win + (size_t)s * p.S;
         const uint32_t* w1 = w0 + p.S;
         for (uint32_t j = ct; j < p.S; j += kConsumers)
-          if (__ldg(w1 + j) > __ldg(w0 + j) && (p.G == 1 || p.owner[j] == p.owner[s])) p.dirty[j] = 1u;
+          if (__ldg(w1 + j) > __ldg(w0 + j)) {
+            if (p.G == 1) {
+              p.dirty[j] = 1u;
+            } else {  // shard j of partition q: its flag lives with q (over NVLink on another GPU)
+              const uint32_t q = p.owner[j];
+              st_u32(p.dirty_peer[q] + (j - p.bounds[q]), 1u);
+            }
+          }
         if (A::kId == kHS && ct == 0) p.dirty[s] = 1u;
         if (p.multi) bar_sync(kConsumerBar, kConsumers);  // the marks precede the ticket's completion
       }
@@ -914,88 +957,78 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
         const BkRec r = bk[b];
         if (r.s == 0xFFFFFFFFu) break;
         ticket_bookkeeping(p, r.s, r.it, r.any != 0, r.upd, r.stores, Sloc);
-        if (CUSHA_TIMELINE) tl_mark(r.it * Sloc + (r.s - (p.part >= 0 ? p.bounds[p.part] : 0u)), 7);
+        if (CUSHA_TIMELINE) tl_mark(r.it * Sloc + r.s, 7);
         mbar_arrive(&bk_empty[b]);
       }
     }
   }
   __syncthreads();
+  if (tid == 0) {  // every mbarrier is done with: invalidate before the shared memory is reused (PTX)
+    for (uint32_t i = 0; i < nst; ++i) {
+      mbar_inval(&full_bar[i]);
+      mbar_inval(&empty_bar[i]);
+    }
+    mbar_inval(&decide_bar);
+    for (uint32_t i = 0; i < 2; ++i) {
+      mbar_inval(&bk_full[i]);
+      mbar_inval(&bk_empty[i]);
+    }
+  }
   if (p.multi) return;  // overlapped passes: the last ticket of a pass closed it (ticket_done)
 
   // ---- iteration close (L189): the last CTA to finish decides whether another pass follows
   if (tid == 0) {
-    __threadfence();
+    if (p.G > 1) __threadfence_system();  // stage-4 stores into other GPUs' SrcValue / dirty before the arrival
+    else __threadfence();
     const uint32_t t = atomicAdd(&p.ctl->ctas_done, 1u);
     if (t == gridDim.x - 1) {
       __threadfence();
       const uint32_t changed = *reinterpret_cast<volatile uint32_t*>(&p.ctl->changed);
-      const uint32_t nit = it0 + 1;
-      p.ctl->iter = nit;
+      p.ctl->iter = it0 + 1;
       p.ctl->changed = 0;
       p.ctl->ctas_done = 0;
       p.ctl->next_shard = 0;
-      // with G partitions only the refresh after the exchange knows the global answer
+      // with G partitions the global answer is the OR over partitions (close_parts)
       if (p.G == 1) p.ctl->converged = changed ? 0u : 1u;
+      else p.ctl->lchanged = changed;
       __threadfence();
-      if (p.use_cond) cudaGraphSetConditional(p.cond_handle, (changed && nit < p.ctl->max_iters) ? 1u : 0u);
     }
   }
 }
 
-// ------------------------------------------------- remote-window refresh (row e)
-// After a partitioned pass and the exchange of gathered[] (write-back values)
-// and active[] (which shards ran stage 4): for every active source shard i,
-// rewrite its windows in the partitions other than its owner's —
-// SrcValue[Mapper[k]] = gathered[i*N + SrcIndexCW[k]] over CW_i's sub-range
-// for that partition — then decide global convergence (no shard of any
-// partition active).  BSP across partitions, asynchronous within one.
-__global__ void __launch_bounds__(256) refresh_remote(const KParams p) {
-  __shared__ int s_act;
-  if (*reinterpret_cast<volatile uint32_t*>(&p.ctl->converged)) return;  // past convergence (host loop)
-  const uint32_t i = blockIdx.x;
-  if (threadIdx.x == 0) s_act = p.active[i];
-  __syncthreads();
-  if (s_act) {
-    const uint32_t oi = p.owner[i];
-    const uint32_t* row = p.cwp + (size_t)i * (p.G + 1);
-    const uint32_t* vals = p.gathered + (size_t)i * p.N;
-    for (uint32_t q = 0; q < p.G; ++q) {
-      if (q == oi || (p.part >= 0 && (int)q != p.part)) continue;
-      for (uint32_t k = row[q] + threadIdx.x; k < row[q + 1]; k += blockDim.x)
-        st_u32(p.srcvalue + __ldg(topo_at(p.mapper, p.mapper_h, p.splitQ, k)),
-               __ldg(vals + __ldg(topo_at(p.cw_src, p.cw_src_h, p.splitQ, k))));
-      if (p.skip)  // the refreshed shards of partition q have new inputs
-        for (uint32_t j = p.bounds[q] + threadIdx.x; j < p.bounds[q + 1]; j += blockDim.x)
-          if (__ldg(p.win + (size_t)(i + 1) * p.S + j) > __ldg(p.win + (size_t)i * p.S + j)) p.dirty[j] = 1u;
-    }
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    if (s_act) *reinterpret_cast<volatile uint32_t*>(&p.ctl->gchanged) = 1u;
-    __threadfence();
-    const uint32_t t = atomicAdd(&p.ctl->rctas_done, 1u);
-    if (t == gridDim.x - 1) {
-      __threadfence();
-      const uint32_t any = *reinterpret_cast<volatile uint32_t*>(&p.ctl->gchanged);
-      p.ctl->converged = any ? 0u : 1u;
-      p.ctl->gchanged = 0;
-      p.ctl->rctas_done = 0;
-      __threadfence();
-    }
+// -------------------------------------------- global convergence (row e)
+// After every partition's pass (and, with one process per GPU, the NCCL
+// all-reduce of the partitions' lchanged words into gchanged): the run has
+// converged when no partition committed an update in that pass (L189).  The
+// pass is BSP across partitions - the all-reduce (or, simulated, the stream
+// order) separates consecutive passes - so a pass in which nothing committed
+// anywhere read a state no stage 4 changed during it: the fixed point.
+//   sim = 1: ctls[0..G) are the partitions of this process; gchanged = OR lchanged.
+//   sim = 0: ctls[0] is this rank's, gchanged already holds the all-reduce.
+__global__ void close_parts(Ctl* const* ctls, uint32_t G, int sim) {
+  if (threadIdx.x != 0) return;
+  uint32_t any = 0;
+  if (sim)
+    for (uint32_t q = 0; q < G; ++q) any |= *reinterpret_cast<volatile uint32_t*>(&ctls[q]->lchanged);
+  else
+    any = *reinterpret_cast<volatile uint32_t*>(&ctls[0]->gchanged);
+  for (uint32_t q = 0; q < (sim ? G : 1u); ++q) {
+    Ctl* c = ctls[q];
+    if (!c->converged && c->iter >= 1 && !any) c->converged = 1u;
   }
 }
 
 // ------------------------------------------------------------ init kernels
-// VertexValues <- Table-3 start state (L327) or the user's initial values;
-// every shard predicted active for the first pass.
+// VertexValues <- Table-3 start state (L327) or the user's initial values for
+// the partition's vertices; every shard predicted active for the first pass.
 template <class A>
-__global__ void init_vertex_values(const KParams p, const void* user) {
+__global__ void init_vertex_values(const KParams p, const void* user, uint32_t v0, uint32_t nvl) {
   using V_t = typename A::Value;
   V_t* vv = reinterpret_cast<V_t*>(p.vv);
   const V_t* u = reinterpret_cast<const V_t*>(user);
-  for (size_t v = blockIdx.x * (size_t)blockDim.x + threadIdx.x; v < p.V; v += (size_t)gridDim.x * blockDim.x)
-    vv[v] = u ? u[v] : A::start((uint32_t)v, p.source);
-  for (size_t s = blockIdx.x * (size_t)blockDim.x + threadIdx.x; s < p.S; s += (size_t)gridDim.x * blockDim.x) {
+  for (size_t v = blockIdx.x * (size_t)blockDim.x + threadIdx.x; v < nvl; v += (size_t)gridDim.x * blockDim.x)
+    vv[v] = u ? u[v] : A::start((uint32_t)(v0 + v), p.source);
+  for (size_t s = blockIdx.x * (size_t)blockDim.x + threadIdx.x; s < p.Sl; s += (size_t)gridDim.x * blockDim.x) {
     p.active[s] = 1;
     if (p.dirty) p.dirty[s] = 1u;  // every shard runs the first pass
     p.shard_seq[s] = 0;
@@ -1003,15 +1036,16 @@ __global__ void init_vertex_values(const KParams p, const void* user) {
 }
 
 // SrcValue[e] <- VertexValues[SrcIndex[e]] for every entry (R20: a full
-// write-back at t = 0), one CTA per source shard i.  Every source of shard i's
-// windows lies in shard i, so the CTA first stages the write-back values of
+// write-back at t = 0), one CTA per own source shard i.  Every source of shard
+// i's windows lies in shard i, so the CTA first stages the write-back values of
 // its |N| vertices in shared memory (coalesced) and then streams its windows
-// (G-Shards) or CW_i (CW) against them, as stage 4 of a pass does.
+// (G-Shards) or CW_i (CW) against them, as stage 4 of a pass does - into every
+// partition's SrcValue when the graph is partitioned.
 template <class A>
 __device__ __forceinline__ void stage_wb_values(const KParams& p, uint32_t i, uint32_t* wb) {
   using V_t = typename A::Value;
   const V_t* vv = reinterpret_cast<const V_t*>(p.vv);
-  const uint32_t off = i * p.N, nv = min(p.N, p.V - off);
+  const uint32_t off = i * p.N, nv = min(p.N, p.V - (p.s0 + i) * p.N);
   for (uint32_t v = threadIdx.x; v < nv; v += blockDim.x)
     wb[v] = A::wb_value(vv[off + v], A::kOutDeg ? __ldg(p.outdeg + off + v) : 0u);
   __syncthreads();
@@ -1026,11 +1060,24 @@ __global__ void __launch_bounds__(512) init_srcvalue_gs(const KParams p) {
 template <class A>
 __global__ void __launch_bounds__(512) init_srcvalue_cw(const KParams p) {
   extern __shared__ uint32_t wb[];
-  const uint32_t i = blockIdx.x, trash = p.shard_off[p.S];
+  const uint32_t i = blockIdx.x;
   stage_wb_values<A>(p, i, wb);
-  for (uint32_t k = p.cw_off[i] + threadIdx.x; k < p.cw_off[i + 1]; k += blockDim.x) {
-    const uint32_t m = __ldg(topo_at(p.mapper, p.mapper_h, p.splitQ, k));
-    if (m != trash) p.srcvalue[m] = wb[__ldg(topo_at(p.cw_src, p.cw_src_h, p.splitQ, k))];
+  for (uint32_t q = 0; q < p.G; ++q) {
+    uint32_t a, b;
+    if (p.G > 1) {
+      a = p.cwp[(size_t)i * (p.G + 1) + q];
+      b = p.cwp[(size_t)i * (p.G + 1) + q + 1];
+    } else {
+      a = p.cw_off[i];
+      b = a + p.cw_cnt[i];
+    }
+    uint32_t* const svq = p.G > 1 ? p.sv_peer[q] : p.srcvalue;
+    for (uint32_t k = a + threadIdx.x; k < b; k += blockDim.x) {
+      uint32_t m;
+      if (p.mapper) m = __ldg(topo_at(p.mapper, p.mapper_h, p.splitQ, k));
+      else m = __ldg(p.cw_delta + (size_t)i * p.S + __ldg(topo_at(p.cw_win, p.cw_win_h, p.splitQ, k))) + k;
+      svq[m] = wb[__ldg(topo_at(p.cw_src, p.cw_src_h, p.splitQ, k))];
+    }
   }
 }
 
@@ -1041,8 +1088,8 @@ __global__ void reset_ctl(Ctl* ctl, uint32_t max_iters) {
   ctl->max_iters = max_iters;
   ctl->converged = 0;
   ctl->next_shard = 0;
+  ctl->lchanged = 0;
   ctl->gchanged = 0;
-  ctl->rctas_done = 0;
   ctl->ticket = 0;
   ctl->stop = 0;
   ctl->conv_iter = 0xFFFFFFFFu;
@@ -1101,19 +1148,20 @@ bool alg_needs_init(int alg) { return alg == kNN || alg == kHS || alg == kCS; }
 KParams make_params(const Graph& g, uint32_t source) {
   KParams p{};
   p.V = g.V; p.N = g.N; p.S = g.S; p.source = source;
+  p.s0 = g.s0; p.Sl = g.Sl;
   p.shard_off = g.d_shard_off; p.shard_cnt = g.d_shard_cnt; p.dest = g.d_dest; p.ev = g.d_ev; p.srcvalue = g.d_srcvalue;
+  p.sv_peer = g.d_sv_peer;
   p.srcloc = g.d_srcloc; p.win = g.d_win; p.cw_off = g.d_cw_off; p.cw_cnt = g.d_cw_cnt; p.active = g.d_active;
   p.cw_src = g.d_cw_src; p.mapper = g.d_mapper; p.vv = g.d_vv; p.outdeg = g.d_outdeg;
   p.cw_win = g.d_cw_win; p.cw_delta = g.d_cw_delta; p.cw_win_h = g.h_cw_win;
   p.ctl = g.d_ctl; p.trace = g.d_trace; p.trace_cap = g.trace_cap;
-  p.G = g.G; p.part = g.G > 1 && !g.simulate ? g.rank : -1;
-  p.bounds = g.d_bounds; p.owner = g.d_owner; p.cwp = g.d_cwp; p.gathered = g.G > 1 ? g.d_gathered : nullptr;
+  p.G = g.G;
+  p.bounds = g.d_bounds; p.owner = g.d_owner; p.cwp = g.d_cwp; p.dirty_peer = g.d_dirty_peer;
   p.run_k = g.d_run_k; p.run_t = g.d_run_t; p.run_unit = g.d_run_unit; p.run_bits = g.d_run_bits; p.run_d = g.d_run_d;
   p.R = g.R;
   p.skip = g.skip_clean ? 1 : 0; p.dirty = g.d_dirty;
   p.splitP = (uint32_t)g.splitP; p.splitQ = (uint32_t)g.splitQ;
   p.dest_h = g.h_dest; p.ev_h = g.h_ev; p.srcloc_h = g.h_srcloc; p.cw_src_h = g.h_cw_src; p.mapper_h = g.h_mapper;
-  p.use_cond = 0; p.cond_handle = 0;
   p.multi = 0; p.shard_seq = g.d_shard_seq;
   p.mapj = 0;
   p.stash = 0;
@@ -1125,15 +1173,15 @@ KParams make_params(const Graph& g, uint32_t source) {
 template <class A>
 static cudaError_t launch_init_t(const Graph& g, uint32_t source, cudaStream_t s) {
   KParams p = make_params(g, source);
-  const uint32_t vb = (uint32_t)((g.V + 255) / 256);
-  init_vertex_values<A><<<vb < 148 * 16 ? vb : 148 * 16, 256, 0, s>>>(p, g.d_init[A::kId]);
-  if (g.S) {
+  const uint32_t vb = (uint32_t)((g.nvl + 255) / 256);
+  init_vertex_values<A><<<vb < 148 * 16 ? (vb ? vb : 1) : 148 * 16, 256, 0, s>>>(p, g.d_init[A::kId], g.v0, g.nvl);
+  if (g.Sl) {
     const size_t sm = 4ull * g.N;  // the shard's write-back values (|N| <= 65534: at most 256 KB)
     const void* fn = g.repr == CUSHA_REPR_CW ? (const void*)&init_srcvalue_cw<A> : (const void*)&init_srcvalue_gs<A>;
     cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;  // |N| beyond the shared-memory limit cannot run the pass either
-    if (g.repr == CUSHA_REPR_CW) init_srcvalue_cw<A><<<g.S, 512, sm, s>>>(p);
-    else init_srcvalue_gs<A><<<g.S, 512, sm, s>>>(p);
+    if (g.repr == CUSHA_REPR_CW) init_srcvalue_cw<A><<<g.Sl, 512, sm, s>>>(p);
+    else init_srcvalue_gs<A><<<g.Sl, 512, sm, s>>>(p);
   }
   return cudaGetLastError();
 }
@@ -1152,9 +1200,9 @@ cudaError_t launch_init(const Graph& g, int alg, uint32_t source, cudaStream_t s
   return cudaErrorInvalidValue;
 }
 
-cudaError_t launch_refresh(const Graph& g, cudaStream_t s) {
-  const KParams p = make_params(g, 0);
-  refresh_remote<<<g.S, 256, 0, s>>>(p);
+cudaError_t launch_close_parts(Ctl* const* ctls, uint32_t G, cudaStream_t s) {
+  // ctls: device array; G > 0: all partitions of this process (simulation); G == 0: one rank after its all-reduce
+  close_parts<<<1, 32, 0, s>>>(ctls, G ? G : 1u, G ? 1 : 0);
   return cudaGetLastError();
 }
 

@@ -2,10 +2,13 @@
 //
 // libnccl.so.2 is opened at run time (dlopen), so single-GPU use has no NCCL
 // dependency; torch ships the library and has normally loaded it already.
-// Per iteration every rank broadcasts, in one NCCL group, its slice of the
-// write-back values (gathered[], 4 B per owned vertex) and of active[] (1 B
-// per owned shard); after convergence the VertexValues slices are broadcast
-// once so that cusha_get_values returns |V| values on every rank.
+// The write-back values themselves never go through NCCL: stage 4 stores them
+// straight into the owning rank's SrcValue over NVLink (CUDA IPC mappings,
+// api.cu).  NCCL carries (1) at build time the 64-byte IPC handles of every
+// rank's SrcValue / dirty arrays (all-gather), (2) once per pass the
+// partition's "committed an update" word (all-reduce MAX), which is both the
+// global convergence test of L189 and the barrier between passes, and (3) at
+// cusha_get_values every rank's VertexValues slice (grouped broadcasts).
 #include <dlfcn.h>
 #include <nccl.h>
 
@@ -25,6 +28,8 @@ struct NcclApi {
   decltype(&ncclCommInitRank) commInitRank = nullptr;
   decltype(&ncclCommDestroy) commDestroy = nullptr;
   decltype(&ncclBroadcast) broadcast = nullptr;
+  decltype(&ncclAllGather) allGather = nullptr;
+  decltype(&ncclAllReduce) allReduce = nullptr;
   decltype(&ncclGroupStart) groupStart = nullptr;
   decltype(&ncclGroupEnd) groupEnd = nullptr;
   decltype(&ncclGetErrorString) errorString = nullptr;
@@ -43,11 +48,13 @@ const NcclApi& api() {
     x.commInitRank = reinterpret_cast<decltype(x.commInitRank)>(dlsym(h, "ncclCommInitRank"));
     x.commDestroy = reinterpret_cast<decltype(x.commDestroy)>(dlsym(h, "ncclCommDestroy"));
     x.broadcast = reinterpret_cast<decltype(x.broadcast)>(dlsym(h, "ncclBroadcast"));
+    x.allGather = reinterpret_cast<decltype(x.allGather)>(dlsym(h, "ncclAllGather"));
+    x.allReduce = reinterpret_cast<decltype(x.allReduce)>(dlsym(h, "ncclAllReduce"));
     x.groupStart = reinterpret_cast<decltype(x.groupStart)>(dlsym(h, "ncclGroupStart"));
     x.groupEnd = reinterpret_cast<decltype(x.groupEnd)>(dlsym(h, "ncclGroupEnd"));
     x.errorString = reinterpret_cast<decltype(x.errorString)>(dlsym(h, "ncclGetErrorString"));
     x.ok = x.getUniqueId && x.commInitRank && x.commDestroy && x.broadcast && x.groupStart && x.groupEnd &&
-           x.errorString;
+           x.errorString && x.allGather && x.allReduce;
     if (!x.ok) x.why = "libnccl.so.2 lacks a required symbol";
     return x;
   }();
@@ -83,21 +90,27 @@ int nccl_init(Graph& g, const void* id128, std::string& err) {
   return CUSHA_OK;
 }
 
-// Each rank r broadcasts its owned slices from the same device buffers (in
-// place), so after the group every rank holds every slice.
-int nccl_exchange(Graph& g, uint32_t vb, bool final_values, std::string& err) {
+int nccl_allgather_bytes(Graph& g, const void* dsend, void* drecv, size_t bytes, std::string& err) {
+  NC(api().allGather(dsend, drecv, bytes, ncclUint8, static_cast<ncclComm_t>(g.nccl_comm), g.stream));
+  return CUSHA_OK;
+}
+
+int nccl_allreduce_max_u32(Graph& g, const uint32_t* dsend, uint32_t* drecv, std::string& err) {
+  NC(api().allReduce(dsend, drecv, 1, ncclUint32, ncclMax, static_cast<ncclComm_t>(g.nccl_comm), g.stream));
+  return CUSHA_OK;
+}
+
+// Rank r broadcasts its VertexValues slice (its vertices [v0, v0 + nvl)) into
+// the same place of every rank's |V|-element buffer dfull.
+int nccl_gather_values(Graph& g, void* dfull, uint32_t vb, std::string& err) {
   ncclComm_t comm = static_cast<ncclComm_t>(g.nccl_comm);
+  char* full = static_cast<char*>(dfull);
   NC(api().groupStart());
-  for (int r = 0; r < g.world_size; ++r) {
-    const uint64_t s0 = g.h_bounds[r], s1 = g.h_bounds[r + 1];
-    const uint64_t v0 = std::min<uint64_t>(s0 * g.N, g.V), v1 = std::min<uint64_t>(s1 * g.N, g.V);
-    if (final_values) {
-      char* vv = static_cast<char*>(g.d_vv);
-      NC(api().broadcast(vv + v0 * vb, vv + v0 * vb, (v1 - v0) * vb, ncclUint8, r, comm, g.stream));
-    } else {
-      NC(api().broadcast(g.d_gathered + v0, g.d_gathered + v0, v1 - v0, ncclUint32, r, comm, g.stream));
-      NC(api().broadcast(g.d_active + s0, g.d_active + s0, s1 - s0, ncclUint8, r, comm, g.stream));
-    }
+  for (uint32_t r = 0; r < g.G; ++r) {
+    const uint64_t v0 = std::min<uint64_t>((uint64_t)g.h_bounds[r] * g.N, g.V);
+    const uint64_t v1 = std::min<uint64_t>((uint64_t)g.h_bounds[r + 1] * g.N, g.V);
+    const void* send = r == g.part ? g.d_vv : full + v0 * vb;
+    NC(api().broadcast(send, full + v0 * vb, (v1 - v0) * vb, ncclUint8, (int)r, comm, g.stream));
   }
   NC(api().groupEnd());
   return CUSHA_OK;

@@ -31,7 +31,7 @@ LAYOUT = {
     "dest_local": (3, np.uint16), "edge_id": (4, np.uint32), "windows": (5, np.uint32),
     "cw_offsets": (6, np.uint32), "cw_sizes": (7, np.uint32), "cw_src_local": (8, np.uint16),
     "mapper": (9, np.uint32), "out_degree": (10, np.uint32), "run_k": (11, np.uint32), "run_t": (12, np.uint32),
-    "cw_window": (13, np.uint16), "cw_delta": (14, np.uint32),
+    "cw_window": (13, np.uint16), "cw_delta": (14, np.uint32), "cw_partition_offsets": (15, np.uint32),
 }
 
 
@@ -50,6 +50,7 @@ class BuildOpts(ctypes.Structure):
         ("skip_clean_shards", ctypes.c_int),
         ("device_topology_budget", ctypes.c_uint64),
         ("pass_barrier", ctypes.c_int),
+        ("keep_layout", ctypes.c_int),
     ]
 
 
@@ -80,6 +81,13 @@ class Stats(ctypes.Structure):
         ("host_bytes", ctypes.c_uint64),
         ("host_shard", ctypes.c_uint32),
         ("mapper_form", ctypes.c_uint32),
+        ("paper_bytes", ctypes.c_uint64),
+        ("wb_entries", ctypes.c_uint64),
+        ("vertices_processed", ctypes.c_uint64),
+        ("updated_total", ctypes.c_uint64),
+        ("partitions", ctypes.c_uint32),
+        ("max_in_degree", ctypes.c_uint32),
+        ("max_part_device_bytes", ctypes.c_uint64),
     ]
 
 
@@ -105,6 +113,9 @@ def lib():
             "cusha_get_stats": (i32, [P, ctypes.POINTER(Stats)]),
             "cusha_get_trace": (i32, [P, P, P, u32]),
             "cusha_get_layout": (i32, [P, i32, P, sz, ctypes.POINTER(u64)]),
+            "cusha_get_part_layout": (i32, [P, u32, i32, P, sz, ctypes.POINTER(u64)]),
+            "cusha_get_part_stats": (i32, [P, u32, ctypes.POINTER(Stats)]),
+            "cusha_trim_memory": (i32, [i32]),
             "cusha_shard_size": (u32, [u32, u64, u32, u32, u32]),
             "cusha_value_bytes": (sz, [i32]),
             "cusha_last_error": (ctypes.c_char_p, []),
@@ -152,6 +163,19 @@ def _ptr(x):
 
 def _is_device(x) -> bool:
     return hasattr(x, "is_cuda") and bool(x.is_cuda)
+
+
+def _check_device_tensor(name, t, device, float_ok=False):
+    """A CUDA tensor passed to the C ABI is read as packed 4-byte values on
+    `device`: int32 / uint32 (float32 too for edge values), contiguous."""
+    import torch
+    ok = (torch.int32, torch.uint32) + ((torch.float32,) if float_ok else ())
+    if t.dtype not in ok:
+        raise TypeError(f"{name}: dtype {t.dtype} is not one of {ok} (the C ABI reads packed 4-byte values)")
+    if not t.is_contiguous():
+        raise ValueError(f"{name}: tensor must be contiguous")
+    if t.device.index != device:
+        raise ValueError(f"{name}: tensor is on cuda:{t.device.index}, the graph is built on cuda:{device}")
 
 
 class Graph:
@@ -218,7 +242,7 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
                 smem_bytes_per_vertex: int = 0, device: int = 0, stream: Optional[int] = None,
                 host_loop: bool = False, world_size: int = 1, rank: int = 0,
                 nccl_id: Optional[bytes] = None, skip_clean_shards: bool = False,
-                device_topology_budget: int = 0, pass_barrier: int = 0) -> Graph:
+                device_topology_budget: int = 0, pass_barrier: int = 0, keep_layout: bool = False) -> Graph:
     """cusha_build_graph.  src/dst/edge_values: numpy (host, copied in) or CUDA tensors (device).
     world_size > 1: destination-range partition; nccl_id = None simulates all
     partitions on this device, else one process per GPU over NCCL.
@@ -226,9 +250,24 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
     device_topology_budget: HBM bytes for per-entry topology; the rest is streamed from pinned host memory.
     pass_barrier: True / 1 = one launch per pass with a device-wide barrier between passes (Fig. 5);
     2 = always overlapped passes (one launch per run); False / 0 = automatic (overlapped unless the
-    graph has many small shards per CTA, include/cusha.h)."""
+    graph has many small shards per CTA, include/cusha.h).
+    keep_layout: keep the arrays only get_layout reads (input edge index per entry, CW window table).
+    CUDA tensors must be int32/uint32 (edge_values also float32), contiguous and on `device`; with
+    stream=None they are read on torch's current stream."""
     on_dev = _is_device(src)
-    if not on_dev:
+    if on_dev:
+        import torch
+        if not (_is_device(dst) and (edge_values is None or _is_device(edge_values))):
+            raise ValueError("src, dst and edge_values must all be CUDA tensors or all host arrays")
+        _check_device_tensor("src", src, device)
+        _check_device_tensor("dst", dst, device)
+        if edge_values is not None:
+            _check_device_tensor("edge_values", edge_values, device, float_ok=True)
+        if stream is None:
+            # build (and run) on torch's current stream: stream order covers the
+            # kernels that produced the tensors
+            stream = torch.cuda.current_stream(device).cuda_stream
+    else:
         src = np.ascontiguousarray(src, dtype=np.uint32)
         dst = np.ascontiguousarray(dst, dtype=np.uint32)
         if edge_values is not None:
@@ -250,6 +289,7 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
     o.skip_clean_shards = int(skip_clean_shards)
     o.device_topology_budget = int(device_topology_budget)
     o.pass_barrier = int(pass_barrier)
+    o.keep_layout = int(keep_layout)
     idbuf = None
     if nccl_id is not None:
         if len(nccl_id) != 128:
@@ -314,13 +354,28 @@ def get_trace(g: Graph):
     return upd[:k], act[:k]
 
 
-def get_layout(g: Graph, part: str) -> np.ndarray:
+def get_layout(g: Graph, part: str, partition: Optional[int] = None) -> np.ndarray:
+    """cusha_get_layout, or cusha_get_part_layout for partition p of a partitioned graph."""
     code, dt = LAYOUT[part]
     cnt = ctypes.c_uint64(0)
-    _check(lib().cusha_get_layout(g.handle, code, None, 0, ctypes.byref(cnt)), "cusha_get_layout")
+    if partition is None:
+        call = lambda out, n: lib().cusha_get_layout(g.handle, code, out, n, ctypes.byref(cnt))  # noqa: E731
+    else:
+        call = lambda out, n: lib().cusha_get_part_layout(g.handle, partition, code, out, n, ctypes.byref(cnt))  # noqa: E731
+    _check(call(None, 0), "cusha_get_layout")
     out = np.empty(cnt.value, dt)
-    _check(lib().cusha_get_layout(g.handle, code, _ptr(out), out.nbytes, ctypes.byref(cnt)), "cusha_get_layout")
+    _check(call(_ptr(out), out.nbytes), "cusha_get_layout")
     return out
+
+
+def get_part_stats(g: Graph, partition: int) -> dict:
+    s = Stats()
+    _check(lib().cusha_get_part_stats(g.handle, partition, ctypes.byref(s)), "cusha_get_part_stats")
+    return {name: getattr(s, name) for name, _ in Stats._fields_}
+
+
+def trim_memory(device: int = 0):
+    _check(lib().cusha_trim_memory(device), "cusha_trim_memory")
 
 
 def shard_size(num_vertices: int, num_edges: int, vertex_bytes: int = 4, smem_per_sm: int = 0,

@@ -42,3 +42,29 @@ def test_reference_arm_under_torchrun_rank0_only(tmp_path):
     assert len(lines) == 1
     d = json.loads(lines[0])
     assert d["impl"] == "reference" and d["n_gpus"] == 2
+
+
+def test_reference_arm_config_is_the_cuda_arms(tmp_path):
+    """Both arms print the same `config` (bench.static_config), so the driver's
+    ratio compares the same workload; PR's step is the cpu_baseline sample."""
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--workload", "C1",
+                          "--steps", "1", "--warmup", "0", "--cache-dir", str(tmp_path)],
+                         capture_output=True, text=True, timeout=600, cwd=ROOT)
+    d = json.loads([ln for ln in out.stdout.splitlines() if ln.startswith("{")][0])
+    sys.path.insert(0, ROOT)
+    import bench
+    import graphgen
+    wl = graphgen.workload("C1")
+    assert d["config"] == bench.static_config("C1", wl, "bfs", "gs")
+
+
+def test_multi_gpu_bench_without_devices_refuses():
+    """`bench.py --gpus 2` launches its own ranks; with fewer visible GPUs it
+    exits non-zero and prints no JSON line (never a silent 1-GPU number)."""
+    env = dict(os.environ, CUDA_VISIBLE_DEVICES="")
+    env.pop("WORLD_SIZE", None)
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--workload", "C1"],
+                         capture_output=True, text=True, timeout=600, cwd=ROOT, env=env)
+    assert out.returncode != 0
+    assert not [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
+    assert "refusing" in out.stderr

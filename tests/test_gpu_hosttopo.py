@@ -36,13 +36,13 @@ def _layout(g, repr):
 @pytest.mark.parametrize("budget_frac", [1e-9, 0.5])
 def test_host_topology_layout_and_results(rm, repr, budget_frac):
     V, s, d, w = rm
-    with cusha.build_graph(V, s, d, edge_values=w, repr=repr, vertices_per_shard=500) as g0:
+    with cusha.build_graph(V, s, d, edge_values=w, repr=repr, vertices_per_shard=500, keep_layout=True) as g0:
         want_layout = _layout(g0, repr)
         st0 = cusha.get_stats(g0)
     # topology bytes per entry of the all-HBM build, to place the split
     budget = max(1, int(budget_frac * st0["entries_padded"] * (14 if repr == "gs" else 16)))
     with cusha.build_graph(V, s, d, edge_values=w, repr=repr, vertices_per_shard=500,
-                           device_topology_budget=budget) as g:
+                           device_topology_budget=budget, keep_layout=True) as g:
         st = cusha.get_stats(g)
         assert st["host_bytes"] > 0 and st["host_shard"] < st["num_shards"]
         if budget_frac < 1e-6:
@@ -69,12 +69,15 @@ def test_host_topology_zero_budget_is_all_hbm(rm):
         assert st["host_bytes"] == 0 and st["host_shard"] == st["num_shards"]
 
 
-def test_host_topology_partitioned(rm):
+def test_host_topology_is_for_one_partition(rm):
+    """Host-streamed topology (row f3) and the destination-range partition
+    (row e) are alternatives for a graph larger than one GPU's HBM; combined
+    they are refused (include/cusha.h)."""
     V, s, d, w = rm
-    with cusha.build_graph(V, s, d, edge_values=w, repr="cw", vertices_per_shard=500, world_size=4,
-                           device_topology_budget=1) as g:
-        assert cusha.run("sssp", g) == cusha.OK
-        np.testing.assert_array_equal(cusha.get_values(g), oracle.sssp(V, s, d, w, 0))
+    with pytest.raises(cusha.CushaError) as e:
+        cusha.build_graph(V, s, d, edge_values=w, repr="cw", vertices_per_shard=500, world_size=4,
+                          device_topology_budget=1)
+    assert e.value.code == cusha.EUNSUPPORTED
 
 
 def test_host_topology_mesh_many_passes():

@@ -160,7 +160,7 @@ def test_layout_matches_oracle(repr, V, E, N):
     ev = np.arange(len(s), dtype=np.uint32) * 7 + 3
     ref = oracle.build_shards(V, s, d, N)
     S = ref["S"]
-    with cusha.build_graph(V, s, d, edge_values=ev, repr=repr, vertices_per_shard=N) as g:
+    with cusha.build_graph(V, s, d, edge_values=ev, repr=repr, vertices_per_shard=N, keep_layout=True) as g:
         off = cusha.get_layout(g, "shard_offsets").astype(np.int64)
         cnt = cusha.get_layout(g, "shard_sizes").astype(np.int64)
         dest = cusha.get_layout(g, "dest_local")
@@ -175,8 +175,6 @@ def test_layout_matches_oracle(repr, V, E, N):
             cw_off = cusha.get_layout(g, "cw_offsets").astype(np.int64)
             cw_src = cusha.get_layout(g, "cw_src_local")
             mapper = cusha.get_layout(g, "mapper").astype(np.int64)
-            run_k = cusha.get_layout(g, "run_k").astype(np.int64)
-            run_t = cusha.get_layout(g, "run_t").astype(np.int64)
             cw_win = cusha.get_layout(g, "cw_window").astype(np.int64)
             cw_delta = cusha.get_layout(g, "cw_delta").astype(np.int64).reshape(S, S)
     assert st["num_shards"] == S and st["vertices_per_shard"] == N
@@ -206,13 +204,6 @@ def test_layout_matches_oracle(repr, V, E, N):
         np.testing.assert_array_equal(cw_src[creal].astype(np.int64) + src_shard * N, ref["cw_src"])
         cfill = np.setdiff1d(np.arange(len(mapper)), creal)
         assert (mapper[cfill] == off[-1]).all()
-        # Mapper runs: one per non-empty window, and expanding them gives Mapper exactly
-        Wlen = np.diff(ref["win"].astype(np.int64), axis=0)
-        assert len(run_k) == int((Wlen > 0).sum())
-        assert (np.diff(run_k) > 0).all()
-        if E:
-            r = np.searchsorted(run_k, creal, side="right") - 1
-            np.testing.assert_array_equal(run_t[r] + (creal - run_k[r]), mapper[creal])
         # Mapper in window form: j = the shard the oracle's Mapper target lies in, and
         # delta[i][j] + k reproduces Mapper exactly; filler entries carry j = 0xFFFF
         tgt_shard = np.searchsorted(ref_off, ref["mapper"].astype(np.int64), side="right") - 1

@@ -79,3 +79,71 @@ def test_partition_max_iters(rm):
     V, s, d, _ = rm
     rc, got, st, _ = run_part("bfs", V, s, d, 4, N=300, max_iters=2)
     assert rc == cusha.NOT_CONVERGED and st["iterations"] == 2
+
+
+# ------------------------------------------------ per-partition layout (row e)
+@pytest.mark.parametrize("G", [2, 3, 8])
+def test_partition_layout_is_the_global_layout_sliced(rm, G):
+    """Each partition holds exactly its shards' entries (the global layout's
+    slice, positions rebased) and the CW of its source shards, whose Mapper
+    points into the OWNING partition's SrcValue: target + that partition's
+    first position = the global Mapper, and the segment of CW_i aimed at
+    partition q holds exactly the entries whose target shard q owns."""
+    V, s, d, w = rm
+    N = 300
+    with cusha.build_graph(V, s, d, edge_values=w, repr="cw", vertices_per_shard=N, keep_layout=True) as g1:
+        off = cusha.get_layout(g1, "shard_offsets").astype(np.int64)
+        cnt = cusha.get_layout(g1, "shard_sizes").astype(np.int64)
+        dest = cusha.get_layout(g1, "dest_local")
+        coff = cusha.get_layout(g1, "cw_offsets").astype(np.int64)
+        ccnt = cusha.get_layout(g1, "cw_sizes").astype(np.int64)
+        csrc = cusha.get_layout(g1, "cw_src_local")
+        mapper = cusha.get_layout(g1, "mapper").astype(np.int64)
+        cwin = cusha.get_layout(g1, "cw_window").astype(np.int64)
+        outdeg = cusha.get_layout(g1, "out_degree")
+        single = cusha.get_stats(g1)
+    S = single["num_shards"]
+    with cusha.build_graph(V, s, d, edge_values=w, repr="cw", vertices_per_shard=N, world_size=G,
+                           keep_layout=True) as g:
+        b = cusha.get_partition(g).astype(np.int64)
+        assert len(b) == G + 1 and b[0] == 0 and b[-1] == S
+        pb = off[b]                                           # first global position of each partition
+        owner = np.repeat(np.arange(G), np.diff(b))
+        total_bytes = 0
+        for q in range(G):
+            s0, s1 = b[q], b[q + 1]
+            lo = cusha.get_layout(g, "shard_offsets", partition=q).astype(np.int64)
+            np.testing.assert_array_equal(lo, off[s0:s1 + 1] - off[s0])
+            np.testing.assert_array_equal(cusha.get_layout(g, "shard_sizes", partition=q), cnt[s0:s1])
+            np.testing.assert_array_equal(cusha.get_layout(g, "dest_local", partition=q), dest[off[s0]:off[s1]])
+            lc = cusha.get_layout(g, "cw_offsets", partition=q).astype(np.int64)
+            np.testing.assert_array_equal(lc, coff[s0:s1 + 1] - coff[s0])
+            np.testing.assert_array_equal(cusha.get_layout(g, "cw_src_local", partition=q), csrc[coff[s0]:coff[s1]])
+            np.testing.assert_array_equal(cusha.get_layout(g, "out_degree", partition=q),
+                                          outdeg[s0 * N:min(V, s1 * N)])
+            lm = cusha.get_layout(g, "mapper", partition=q).astype(np.int64)
+            cwp = cusha.get_layout(g, "cw_partition_offsets", partition=q).astype(np.int64).reshape(s1 - s0, G + 1)
+            for il in range(s1 - s0):
+                i = s0 + il
+                assert cwp[il, 0] == lc[il] and cwp[il, G] == lc[il] + ccnt[i]
+                assert (np.diff(cwp[il]) >= 0).all()
+                for t in range(G):
+                    seg = np.arange(cwp[il, t], cwp[il, t + 1])
+                    glob_k = seg + coff[s0]
+                    assert (owner[cwin[glob_k]] == t).all()                     # aimed at partition t
+                    np.testing.assert_array_equal(lm[seg] + pb[t], mapper[glob_k])
+            st = cusha.get_part_stats(g, q)
+            total_bytes += st["device_bytes"]
+        assert cusha.get_stats(g)["partitions"] == G
+    # per-partition memory is the global layout split, not replicated
+    assert total_bytes < 1.25 * single["device_bytes"] + G * 4 * (S + 1) * S
+
+
+def test_partition_device_bytes_shrink_with_G():
+    wl = graphgen.workload("rmat:200000:3200000:64")
+    sizes = {}
+    for G in (1, 2, 4, 8):
+        with cusha.build_graph(wl.V, wl.src, wl.dst, repr="cw", world_size=G) as g:
+            sizes[G] = cusha.get_stats(g)["max_part_device_bytes"]
+    for G in (2, 4, 8):
+        assert sizes[G] < 1.6 * sizes[1] / G, sizes
