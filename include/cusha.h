@@ -167,7 +167,18 @@ typedef struct {
    * the input edge index of every shard entry and, for CW, the window
    * table.  0 (default) = release them after the build.                    */
   int keep_layout;
+  /* Schedule of SrcValue visibility (SURVEY.md §8(b) cusha_mode; L45, L433).
+   * CUSHA_MODE_ASYNC (0, default, the paper's): a shard's stage-4 write-back
+   *   is visible to shards processed after it in the same pass.
+   * CUSHA_MODE_BSP (1, two-phase): every pass reads the SrcValues as they were
+   *   at the end of the previous pass (stage 4 writes a second copy that the
+   *   next pass reads); the pass sequence is then deterministic and matches
+   *   the oracle's mode T pass for pass (tests/test_gpu_bsp.py).  Single
+   *   partition only; one launch per pass plus a copy of SrcValue.         */
+  int mode;
 } cusha_build_opts;
+
+enum { CUSHA_MODE_ASYNC = 0, CUSHA_MODE_BSP = 1 };
 
 typedef struct cusha_graph cusha_graph;   /* opaque; owns all device memory it allocates */
 

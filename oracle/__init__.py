@@ -51,6 +51,7 @@ def _L():
             "or_cs": [u64, u64, P, P, P, P, P, dbl, u64, P, P],
             "or_build_shards": [u64, u64, P, P, u32, P, P, P, P, P, P, P, P],
             "or_pagerank_residual": [u64, u64, P, P, dbl, P, P],
+            "or_trajectory": [ctypes.c_int, u64, u64, P, P, P, u32, u32, P, u64, dbl, P, P, P, P, P],
         }
         for name, args in sig.items():
             f = getattr(lib, name)
@@ -171,3 +172,32 @@ def build_shards(V, src, dst, N):
          "build_shards")
     r["win"] = r["win"].reshape(S + 1, S)
     return r
+
+
+ALGS = {"bfs": 0, "sssp": 1, "pr": 2, "cc": 3, "sswp": 4, "nn": 5, "hs": 6, "cs": 7}
+
+
+def trajectory(alg, V, src, dst, N, ev=None, source=0, init=None, max_passes=100000, tol=1e-5):
+    """Mode T (oracle.c or_trajectory): the paper's Fig. 5 pass, shard by shard
+    with |N| = N, under the two-phase BSP schedule.  ev: raw 4-byte EdgeValue
+    per input edge (u32 or f32 array); init: NN x0 / HS Q0 (f32[V]) or CS
+    {V0, GsumOrA0} (f32[V, 2]).  Returns dict(values, passes, updated,
+    active_shards, converged): values u32[V] (integer algorithms) or f64[V]
+    (PR Rank, NN x, HS Q, CS V)."""
+    a = ALGS[alg] if isinstance(alg, str) else int(alg)
+    src, dst = _u32(src), _u32(dst)
+    evb = None if ev is None else np.ascontiguousarray(ev).view(np.uint32)
+    ini = None if init is None else np.ascontiguousarray(init, dtype=np.float32).reshape(-1)
+    integer = a in (0, 1, 3, 4)
+    ou = np.empty(V, np.uint32) if integer else None
+    of = None if integer else np.empty(V, np.float64)
+    cap = int(max_passes)
+    upd = np.zeros(cap, np.uint32)
+    act = np.zeros(cap, np.uint32)
+    n = ctypes.c_uint64(0)
+    rc = _L().or_trajectory(a, V, len(src), _p(src), _p(dst), _p(evb), N, source, _p(ini), cap, tol, _p(ou), _p(of),
+                            _p(upd), _p(act), ctypes.byref(n))
+    _chk(rc, "trajectory", allow_notconv=True)
+    k = int(n.value)
+    return {"values": ou if integer else of, "passes": k, "updated": upd[:k], "active_shards": act[:k],
+            "converged": rc == OK}

@@ -73,7 +73,7 @@ static uint64_t device_bytes(const Graph& g) {
   if (g.d_cw_delta) b += 4ull * g.Sl * g.S;
   if (g.d_cwp) b += 4ull * g.Sl * (g.G + 1) + g.S;
   b += 4ull * g.nvl;                                     // out-degrees
-  b += 4 * (g.P + 1) + 8ull * g.nvl;                     // SrcValue + VertexValues
+  b += 4 * (g.P + 1) * (g.bsp ? 2 : 1) + 8ull * g.nvl;  // SrcValue (two copies in BSP mode) + VertexValues
   return b - g.host_bytes;                               // minus the host-streamed part (row f3)
 }
 
@@ -119,6 +119,10 @@ static int alloc_run_state(Graph& g, bool ipc) {
     CKA(dev_alloc((void**)&g.d_srcvalue, 4 * (g.P + 1), g.stream));
   }
   CKA(cudaMemsetAsync(g.d_srcvalue, 0, 4 * (g.P + 1), g.stream));
+  if (g.bsp) {
+    CKA(dev_alloc((void**)&g.d_srcvalue2, 4 * (g.P + 1), g.stream));
+    CKA(cudaMemsetAsync(g.d_srcvalue2, 0, 4 * (g.P + 1), g.stream));
+  }
   CKA(dev_alloc(&g.d_vv, 8ull * std::max<uint32_t>(g.nvl, 1), g.stream));
   CKA(dev_alloc((void**)&g.d_ctl, sizeof(Ctl), g.stream));
   CKA(cudaMemsetAsync(g.d_ctl, 0, sizeof(Ctl), g.stream));
@@ -244,6 +248,9 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   uint32_t N = o.vertices_per_shard ? o.vertices_per_shard : cusha_shard_size(V, E, o.smem_bytes_per_vertex, 0, 0);
   if (N > 65534) return fail(CUSHA_EINVAL, "vertices_per_shard must be <= 65534");
   if (o.pass_barrier < 0 || o.pass_barrier > 2) return fail(CUSHA_EINVAL, "pass_barrier must be 0, 1 or 2");
+  if (o.mode != CUSHA_MODE_ASYNC && o.mode != CUSHA_MODE_BSP) return fail(CUSHA_EINVAL, "mode must be ASYNC or BSP");
+  if (o.mode == CUSHA_MODE_BSP && o.world_size > 1)
+    return fail(CUSHA_EUNSUPPORTED, "the two-phase BSP mode runs one partition");
   if (N > V) N = V;
   const uint32_t S = (V + N - 1) / N;
   const int mode = o.world_size == 1 ? kModeSingle : (o.nccl_unique_id ? kModeNccl : kModeSim);
@@ -278,6 +285,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   g.pass_barrier = o.pass_barrier;
   g.topo_budget = o.device_topology_budget;
   g.keep_ids = o.keep_layout != 0;
+  g.bsp = o.mode == CUSHA_MODE_BSP;
   g.world_size = o.world_size;
   g.rank = mode == kModeNccl ? o.rank : 0;
   cudaEvent_t e0 = nullptr, eh = nullptr, e1 = nullptr;
@@ -707,7 +715,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   PassCfg cfg;
   if ((rc = pass_config(g, pk, &cfg))) return rc;
   const bool parted = h->mode != kModeSingle;
-  const bool host_loop = g.host_loop || parted;
+  const bool host_loop = g.host_loop || parted || g.bsp;
   // one launch for the whole run (overlapped passes) unless asked otherwise;
   // the automatic mode takes one launch per pass for many small shards per
   // CTA (67_16 at |N| = 1536: 4.40 vs 5.48 ms)
@@ -755,9 +763,19 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
       kps.push_back(pass_params(*p, source, cfg, a));
       grids.push_back(pass_grid(*p, pk, cfg.smem));
     }
+    uint32_t* cur = g.d_srcvalue;  // BSP: the copy this pass reads (init wrote d_srcvalue)
+    uint32_t* nxt = g.d_srcvalue2;
     for (;;) {
       if (host_loop) {
         for (int k = 0; k < kChunk; ++k) {
+          if (g.bsp) {
+            // two-phase BSP: stage 4 writes the copy the NEXT pass reads, which
+            // starts as this pass's input (entries no shard writes carry over)
+            CKA(cudaMemcpyAsync(nxt, cur, 4 * (g.P + 1), cudaMemcpyDeviceToDevice, st));
+            kps[0].srcvalue = cur;
+            kps[0].sv_write = nxt;
+            std::swap(cur, nxt);
+          }
           for (size_t r = 0; r < h->parts.size(); ++r) {
             void* args[] = {&kps[r]};
             CKA(cudaLaunchKernel(pk.func, dim3(grids[r]), dim3(pk.threads), args, cfg.smem, st));

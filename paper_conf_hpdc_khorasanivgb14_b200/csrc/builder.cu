@@ -785,6 +785,8 @@ void free_device_arrays(Graph& g) {
     if (g.srcvalue_ipc) cudaFree(g.d_srcvalue);  // IPC-exported allocations are not stream-ordered
     else cudaFreeAsync(g.d_srcvalue, g.stream);
   }
+  if (g.d_srcvalue2) cudaFreeAsync(g.d_srcvalue2, g.stream);
+  g.d_srcvalue2 = nullptr;
   for (void*& p : g.d_init)
     if (p) { cudaFreeAsync(p, g.stream); p = nullptr; }
   for (void* p : g.ipc_open) cudaIpcCloseMemHandle(p);

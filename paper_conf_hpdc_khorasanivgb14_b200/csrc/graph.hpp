@@ -51,7 +51,8 @@ struct KParams {
   const uint32_t* shard_cnt;   // Sl real entry counts
   const uint16_t* dest;        // P local DestIndex (filler = N)
   const uint32_t* ev;          // P EdgeValue or null
-  uint32_t* srcvalue;          // P+1 SrcValue of this partition's shard entries
+  uint32_t* srcvalue;          // P+1 SrcValue of this partition's shard entries (read by stage 2)
+  uint32_t* sv_write;          // single partition: where stage 4 writes (= srcvalue; the other buffer in BSP mode)
   uint32_t* const* sv_peer;    // G: SrcValue of every partition (sv_peer[own] = srcvalue); stage 4 of a
                                // source shard stores into the partition that owns each window's target
   const uint16_t* srcloc;      // GS: P SrcIndex - (source shard)*N
@@ -182,6 +183,8 @@ struct Graph {
   // per-run state
   uint32_t* d_srcvalue = nullptr;   // P+1
   bool srcvalue_ipc = false;        // allocated with cudaMalloc (exported to the other ranks)
+  bool bsp = false;                 // two-phase BSP mode: stage 4 writes the next pass's SrcValue copy
+  uint32_t* d_srcvalue2 = nullptr;  // BSP mode: the second SrcValue buffer
   void* d_vv = nullptr;             // nvl * 8 bytes
   void* d_init[8] = {};             // user initial values per algorithm (this partition's slice)
   float init_max_abs[8] = {};       // largest |initial value| given per algorithm

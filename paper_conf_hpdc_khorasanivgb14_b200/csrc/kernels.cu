@@ -804,7 +804,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
             d = desc[slot];
             // the partition owning this tile's windows (this one on a single GPU):
             // in the multi-GPU mode the stores below go over NVLink to its SrcValue
-            uint32_t* const svq = p.G > 1 ? p.sv_peer[d.tgt] : p.srcvalue;
+            uint32_t* const svq = p.G > 1 ? p.sv_peer[d.tgt] : p.sv_write;
             if (any && d.kind == kDescStage4R) {
               // Mapper from runs: target(k) = k + D[r], D = RunT - RunK, for the run r
               // containing CW position k.  Runs start where the run-start bitmap has
@@ -897,7 +897,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
         // batch of 32 windows per warp with one entry per lane (gs_walk)
         gs_walk(p, s, lane, cwarp, kConsumerWarps, [&](uint32_t e, uint32_t l) {
           uint32_t val;
-          if (wb_get<A>(sm, aux, l, val)) { st_u32(p.srcvalue + e, val); ++stores; }
+          if (wb_get<A>(sm, aux, l, val)) { st_u32(p.sv_write + e, val); ++stores; }
         });
       }
 #pragma unroll
@@ -1150,6 +1150,7 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.V = g.V; p.N = g.N; p.S = g.S; p.source = source;
   p.s0 = g.s0; p.Sl = g.Sl;
   p.shard_off = g.d_shard_off; p.shard_cnt = g.d_shard_cnt; p.dest = g.d_dest; p.ev = g.d_ev; p.srcvalue = g.d_srcvalue;
+  p.sv_write = g.d_srcvalue;
   p.sv_peer = g.d_sv_peer;
   p.srcloc = g.d_srcloc; p.win = g.d_win; p.cw_off = g.d_cw_off; p.cw_cnt = g.d_cw_cnt; p.active = g.d_active;
   p.cw_src = g.d_cw_src; p.mapper = g.d_mapper; p.vv = g.d_vv; p.outdeg = g.d_outdeg;

@@ -51,6 +51,7 @@ class BuildOpts(ctypes.Structure):
         ("device_topology_budget", ctypes.c_uint64),
         ("pass_barrier", ctypes.c_int),
         ("keep_layout", ctypes.c_int),
+        ("mode", ctypes.c_int),
     ]
 
 
@@ -242,7 +243,8 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
                 smem_bytes_per_vertex: int = 0, device: int = 0, stream: Optional[int] = None,
                 host_loop: bool = False, world_size: int = 1, rank: int = 0,
                 nccl_id: Optional[bytes] = None, skip_clean_shards: bool = False,
-                device_topology_budget: int = 0, pass_barrier: int = 0, keep_layout: bool = False) -> Graph:
+                device_topology_budget: int = 0, pass_barrier: int = 0, keep_layout: bool = False,
+                mode="async") -> Graph:
     """cusha_build_graph.  src/dst/edge_values: numpy (host, copied in) or CUDA tensors (device).
     world_size > 1: destination-range partition; nccl_id = None simulates all
     partitions on this device, else one process per GPU over NCCL.
@@ -252,6 +254,7 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
     2 = always overlapped passes (one launch per run); False / 0 = automatic (overlapped unless the
     graph has many small shards per CTA, include/cusha.h).
     keep_layout: keep the arrays only get_layout reads (input edge index per entry, CW window table).
+    mode: "async" (the paper's schedule) or "bsp" (two-phase: each pass reads the previous pass's SrcValues).
     CUDA tensors must be int32/uint32 (edge_values also float32), contiguous and on `device`; with
     stream=None they are read on torch's current stream."""
     on_dev = _is_device(src)
@@ -290,6 +293,7 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
     o.device_topology_budget = int(device_topology_budget)
     o.pass_barrier = int(pass_barrier)
     o.keep_layout = int(keep_layout)
+    o.mode = {"async": 0, "bsp": 1}[mode] if isinstance(mode, str) else int(mode)
     idbuf = None
     if nccl_id is not None:
         if len(nccl_id) != 128:
