@@ -89,7 +89,8 @@ def test_bsp_float_k_pass_states(repr):
         close(got, oracle.trajectory("nn", 4096, s2, d2, 512, ev=w, init=x0, max_passes=k)["values"])
     s3, d3, c, q0 = hs_inputs()
     for k in (1, 3):
-        _, got, _, _, _ = bsp_run("hs", 4096, s3, d3, 512, repr, ev=as_bits(c), init=q0, max_iters=k)
+        _, got, _, _, _ = bsp_run("hs", 4096, s3, d3, 512, repr, ev=as_bits(c), init=np.stack([q0, q0], 1),
+                                  max_iters=k)
         close(got[:, 0], oracle.trajectory("hs", 4096, s3, d3, 512, ev=c, init=q0, max_passes=k)["values"],
               extra=1e-5 * 100)
     s4, d4, G, v0, a0 = cs_inputs()
