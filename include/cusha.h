@@ -221,6 +221,9 @@ typedef struct {
   uint32_t partitions;             /* partitions of the graph (row e); 1 = unpartitioned         */
   uint32_t max_in_degree;          /* largest in-degree (fixed-point range check)                */
   uint64_t max_part_device_bytes;  /* the largest partition's device_bytes (= device_bytes at 1)  */
+  uint32_t ring_slots;             /* last run: TMA ring slots per CTA of the shard pass          */
+  uint32_t l2_read_ahead;          /* last run: 1 = stage-2 tiles were prefetched into L2 ahead of
+                                      the ring (a pass streams more than twice the L2)          */
 } cusha_stats;
 
 /* ---------------------------------------------------------------- build */

@@ -569,7 +569,9 @@ static int pass_config(const Graph& g, const PassKernel& pk, PassCfg* c) {
 static int pass_ahead(const Graph& g, int alg) {
   int l2 = 0;
   if (cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, g.device) != cudaSuccess || l2 <= 0) l2 = 126 << 20;
-  const uint64_t bytes = (uint64_t)g.P * (6 + (alg_needs_edge_values(alg) ? 4 : 0)) + (uint64_t)g.Q * 8;
+  // stage 2: SrcValue + DestIndex (+ EdgeValue); stage 4: GS SrcIndex, CW SrcIndexCW + Mapper form
+  const uint64_t bytes = (uint64_t)g.P * (6 + (alg_needs_edge_values(alg) ? 4 : 0) + (g.repr == CUSHA_REPR_GSHARDS ? 2 : 0)) +
+                         (uint64_t)g.Q * 8;
   return bytes > 2ull * (uint64_t)l2 ? 1 : 0;
 }
 
@@ -847,6 +849,8 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   s.stage2_bytes_per_iter = sum.stage2_bytes_per_iter;
   s.wb_bytes_all_active = sum.wb_bytes_all_active;
   s.mapper_form = (uint32_t)cfg.mapj;
+  s.ring_slots = cfg.nst;
+  s.l2_read_ahead = (uint32_t)pass_ahead(g, a);
   s.device_loop = host_loop ? 0 : (multi ? 2 : 1);
   h->last_alg = a;
   h->have_values = true;

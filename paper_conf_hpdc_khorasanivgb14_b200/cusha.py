@@ -89,6 +89,8 @@ class Stats(ctypes.Structure):
         ("partitions", ctypes.c_uint32),
         ("max_in_degree", ctypes.c_uint32),
         ("max_part_device_bytes", ctypes.c_uint64),
+        ("ring_slots", ctypes.c_uint32),
+        ("l2_read_ahead", ctypes.c_uint32),
     ]
 
 

@@ -284,3 +284,45 @@ def test_host_loop_mode_same_results(c1, repr):
     pr_check(got, x_star)
     got, st = gpu_run("bfs", V, s, d, repr=repr, N=128, host_loop=True, max_iters=3, expect_converged=False)
     assert st["iterations"] == 3 and st["converged"] == 0
+
+
+# -------------------------------------- layout of unsorted input with duplicates
+@pytest.mark.parametrize("repr", REPRS)
+def test_layout_shuffled_duplicates_self_loops(repr):
+    """The builder's order is the definition's (shard(dst), src, dst, INPUT
+    ORDER) (L129, R17) on an edge list that is shuffled and carries duplicate
+    edges and self-loops (kept as separate edges, R22): every array bit-exact
+    against oracle.build_shards, and the integer fixed points still exact."""
+    V = 3000
+    s, d = graphgen.rmat(V, 30000, seed=81)
+    rng = np.random.default_rng(81)
+    dup = rng.integers(0, len(s), 4000)
+    loops = rng.integers(0, V, 500).astype(np.uint32)
+    s = np.concatenate([s, s[dup], loops])
+    d = np.concatenate([d, d[dup], loops])
+    perm = rng.permutation(len(s))
+    s, d = s[perm].astype(np.uint32), d[perm].astype(np.uint32)
+    w = graphgen.edge_u32(s, d, seed=81, lo=1, hi=255)
+    for N in (97, 512):
+        ref = oracle.build_shards(V, s, d, N)
+        S = ref["S"]
+        with cusha.build_graph(V, s, d, edge_values=w, repr=repr, vertices_per_shard=N, keep_layout=True) as g:
+            off = cusha.get_layout(g, "shard_offsets").astype(np.int64)
+            cnt = cusha.get_layout(g, "shard_sizes").astype(np.int64)
+            eid = cusha.get_layout(g, "edge_id")
+            dest = cusha.get_layout(g, "dest_local").astype(np.int64)
+            real = np.concatenate([np.arange(off[j], off[j] + cnt[j]) for j in range(S)])
+            np.testing.assert_array_equal(eid[real], ref["gs_eid"])          # includes the tie-break order
+            np.testing.assert_array_equal(dest[real] + np.repeat(np.arange(S), cnt) * N, ref["gs_dst"])
+            if repr == "cw":
+                coff = cusha.get_layout(g, "cw_offsets").astype(np.int64)
+                ccnt = cusha.get_layout(g, "cw_sizes").astype(np.int64)
+                mapper = cusha.get_layout(g, "mapper").astype(np.int64)
+                to_unpadded = np.full(int(off[-1]) + 1, -1, np.int64)
+                to_unpadded[real] = np.arange(len(real))
+                creal = np.concatenate([np.arange(coff[i], coff[i] + ccnt[i]) for i in range(S)])
+                np.testing.assert_array_equal(to_unpadded[mapper[creal]], ref["mapper"].astype(np.int64))
+            for alg, want, ev in (("bfs", oracle.bfs(V, s, d, 0), None), ("sssp", oracle.sssp(V, s, d, w, 0), w),
+                                  ("cc", oracle.cc(V, s, d), None)):
+                assert cusha.run(alg, g) == cusha.OK
+                np.testing.assert_array_equal(cusha.get_values(g), want, err_msg=f"{alg} N={N}")
