@@ -6,7 +6,13 @@ textbook / Dijkstra definitions finish in seconds even at scale 26).  C2
 PageRank is compared with the oracle converged to 1e-9 (R10).  C5 PageRank
 (1.07 B edges; the oracle's sweeps would take minutes) is checked through a
 property that holds at any size: the fixed-point residual of every vertex is
-within the bound implied by the eps = 1e-5 stopping rule."""
+within the bound implied by the eps = 1e-5 stopping rule, and
+element by element against the oracle converged to 1e-9 (R10): on a committed
+sample (tests/golden/c5_pr_sample.npz, written by tools/golden_c5_pr.py, which
+calls only oracle/) and, where the full oracle vector is present
+(tests/golden_cache/, git-ignored, same script), on every vertex."""
+import os
+
 import numpy as np
 import pytest
 
@@ -83,3 +89,24 @@ def test_c5_pagerank_residual(c5):
     bad = np.abs(res) > bound
     assert not bad.any(), f"{bad.sum()} vertices violate the residual bound; worst {np.abs(res)[bad].max()}"
     assert (x >= 0.15 - 1e-6).all()
+
+
+GOLD = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", "c5_pr_sample.npz")
+FULL = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden_cache", "c5_pr_xstar.f64")
+
+
+def test_c5_pagerank_vs_oracle_1e9(c5):
+    """north_star: PR must match an oracle converged to 1e-9 (R10 bound) - at C5,
+    in bench.py's launch configuration (default |N|, CW, overlapped passes)."""
+    z = np.load(GOLD)
+    assert int(z["V"]) == c5.V and int(z["E"]) == c5.E and float(z["tol"]) == 1e-9
+    x, st = run("pr", c5)
+    assert st["device_loop"] == 2
+    idx = z["idx"].astype(np.int64)
+    maxerr, n_abs = pr_check(x[idx], z["xstar"])
+    print(f"C5 PR sample: {idx.size} vertices (incl. the 2,000 largest x*), max|err| {maxerr:.2e}, "
+          f"{n_abs} over 1e-4 abs; oracle {int(z['sweeps'])} sweeps")
+    if os.path.exists(FULL) and os.path.getsize(FULL) == 8 * c5.V:
+        xs = np.fromfile(FULL, np.float64)
+        maxerr, n_abs = pr_check(x, xs)
+        print(f"C5 PR all {c5.V} vertices: max|err| {maxerr:.2e}, {n_abs} over 1e-4 abs")

@@ -2,7 +2,7 @@
 # Evidence for profiles/<tag>/: ncu launch list of the default bench command,
 # ncu --set full of its shard_pass launch (one launch per run: overlapped
 # passes) and of one per-pass launch (host-loop mode), and bench lines.
-TAG=${1:-r1}
+TAG=${1:-r2}
 O=gpurun_out/$TAG; mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" > $O/build.log 2>&1
 # every launch of one bench step (default mode), device time and DRAM bytes
@@ -15,3 +15,4 @@ timeout 900 ncu --set full --cache-control none --clock-control none --import-so
 timeout 900 python bench.py --cache-dir /tmp/gg > $O/bench_C2.json 2> $O/bench_C2.err; echo "bench $?"
 for w in C1 C3 C3gs C4cc C4sswp; do timeout 600 python bench.py --workload $w --steps 5 --warmup 3 --cache-dir /tmp/gg --cpu-budget 5 > $O/bench_$w.json 2>$O/bench_$w.err; done; echo "others $?"
 timeout 300 python bench.py --workload C2 --steps 5 --warmup 3 --pass-barrier --no-e2e --no-cpu-baseline --cache-dir /tmp/gg > $O/bench_C2_passbarrier.json 2>/dev/null; echo "barrier $?"
+for w in C5pr C5bfs; do timeout 900 python bench.py --workload $w --steps 3 --warmup 3 --no-e2e --cache-dir /tmp/gg --cpu-budget 5 > $O/bench_$w.json 2>$O/bench_$w.err; done; echo "c5 $?"
