@@ -192,7 +192,8 @@ typedef struct {
   uint32_t iterations;             /* shard passes of the last run (incl. the converged one)   */
   uint32_t converged;              /* 1 if the last run's final pass committed nothing         */
   double build_ms;                 /* cusha_build_graph wall time on the stream (incl. H2D)    */
-  double h2d_ms;                   /* part of build_ms spent copying host inputs              */
+  double h2d_ms;                   /* build start to the last host-input copy landing (the copies
+                                      overlap the first layout pass, row f2)                   */
   double run_ms;                   /* last cusha_run: init + all shard passes (device events)  */
   double loop_ms;                  /* last cusha_run: the shard passes only (device events)    */
   uint64_t h2d_bytes;              /* bytes copied host->device by the build                   */

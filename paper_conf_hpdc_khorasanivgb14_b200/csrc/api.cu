@@ -301,24 +301,53 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   const uint32_t *d_src = src, *d_dst = dst, *d_val = edge_values;
   void* tmp = nullptr;
   uint64_t h2d = 0;
+  InputChunks chunks;
+  cudaStream_t cs = nullptr;  // copy stream of the host-input path (row f2)
+  struct CopyGuard {
+    InputChunks* c;
+    cudaStream_t* s;
+    ~CopyGuard() {
+      if (*s) { cudaStreamSynchronize(*s); cudaStreamDestroy(*s); }
+      for (int i = 0; i < c->n; ++i) cudaEventDestroy(c->ready[i]);
+      if (c->all) cudaEventDestroy(c->all);
+    }
+  } cg{&chunks, &cs};
   if (o.input_location == CUSHA_INPUT_HOST && E) {
+    // the host edge list crosses in chunks on a copy stream; the layout's first
+    // pass (keys, degrees) consumes each chunk as it lands (DESIGN.md f2)
     const uint64_t nvals = edge_values ? 3 : 2;
     if ((rc = cu(dev_alloc(&tmp, nvals * E * 4, h->stream), "cudaMallocAsync(inputs)"))) return bail(rc);
     uint32_t* t = static_cast<uint32_t*>(tmp);
-    if ((rc = cu(cudaMemcpyAsync(t, src, E * 4, cudaMemcpyHostToDevice, h->stream), "H2D src")) ||
-        (rc = cu(cudaMemcpyAsync(t + E, dst, E * 4, cudaMemcpyHostToDevice, h->stream), "H2D dst")) ||
-        (edge_values &&
-         (rc = cu(cudaMemcpyAsync(t + 2 * E, edge_values, E * 4, cudaMemcpyHostToDevice, h->stream), "H2D values")))) {
+    if ((rc = cu(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking), "cudaStreamCreate(copy)")) ||
+        (rc = cu(cudaEventRecord(eh, h->stream), "event"))) {  // the allocation precedes the copies
+      cudaFreeAsync(tmp, h->stream);
+      return bail(rc);
+    }
+    chunks.n = E >= (1ull << 22) ? 8 : 1;
+    for (int c = 0; c <= chunks.n; ++c) chunks.bounds[c] = E * (uint64_t)c / (uint64_t)chunks.n;
+    rc = cu(cudaStreamWaitEvent(cs, eh, 0), "wait");
+    for (int c = 0; c < chunks.n && !rc; ++c) {
+      const uint64_t lo = chunks.bounds[c], n = chunks.bounds[c + 1] - lo;
+      if ((rc = cu(cudaEventCreateWithFlags(&chunks.ready[c], cudaEventDisableTiming), "event")) ||
+          (rc = cu(cudaMemcpyAsync(t + lo, src + lo, n * 4, cudaMemcpyHostToDevice, cs), "H2D src")) ||
+          (rc = cu(cudaMemcpyAsync(t + E + lo, dst + lo, n * 4, cudaMemcpyHostToDevice, cs), "H2D dst")) ||
+          (rc = cu(cudaEventRecord(chunks.ready[c], cs), "event")))
+        break;
+    }
+    if (!rc && edge_values)
+      rc = cu(cudaMemcpyAsync(t + 2 * E, edge_values, E * 4, cudaMemcpyHostToDevice, cs), "H2D values");
+    if (!rc && !(rc = cu(cudaEventCreate(&chunks.all), "event"))) rc = cu(cudaEventRecord(chunks.all, cs), "event");
+    if (rc) {
+      cudaStreamSynchronize(cs);
       cudaFreeAsync(tmp, h->stream);
       return bail(rc);
     }
     d_src = t; d_dst = t + E; d_val = edge_values ? t + 2 * E : nullptr;
     h2d = nvals * E * 4;
   }
-  CKA(cudaEventRecord(eh, h->stream));
   std::string err;
-  rc = build_layout(g, d_src, d_dst, d_val, err);
-  if (tmp) cudaFreeAsync(tmp, h->stream);
+  rc = build_layout(g, d_src, d_dst, d_val, err, chunks.n ? &chunks : nullptr);
+  if (tmp) cudaFreeAsync(tmp, h->stream);  // stream order: the build waited for every copy
   if (rc) {
     set_error("build: " + err);
     return bail(rc);
@@ -399,7 +428,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   CKA(cudaEventSynchronize(e1));
   float ms = 0, ms_h2d = 0;
   cudaEventElapsedTime(&ms, e0, e1);
-  cudaEventElapsedTime(&ms_h2d, e0, eh);
+  if (chunks.all) cudaEventElapsedTime(&ms_h2d, e0, chunks.all);  // build start to the last copy landing
   cusha_stats& st = h->st;
   st.num_vertices = V;
   st.num_edges = E;

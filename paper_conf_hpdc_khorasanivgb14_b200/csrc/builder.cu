@@ -44,15 +44,23 @@ inline unsigned grid_for(uint64_t n, unsigned block = 256) {
 
 #define GRID_STRIDE(i, n) for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < (n); i += (uint64_t)gridDim.x * blockDim.x)
 
-__global__ void k_make_keys(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst, uint64_t E, uint32_t V,
-                            uint32_t N, int bn, int bsrc, uint64_t* keys, uint32_t* ids, uint32_t* bad) {
-  GRID_STRIDE(e, E) {
+// One pass over the input edges [lo, hi): the G-Shards sort key, the input
+// index (the sort's payload, R17), out-degrees (PR NbrsNum, L318) and
+// in-degrees (fixed-point range check).  Run per chunk as the host copy
+// streams in (DESIGN.md f2).
+__global__ void k_ingest(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst, uint64_t lo, uint64_t hi,
+                         uint32_t V, uint32_t N, int bn, int bsrc, uint64_t* keys, uint32_t* ids, uint32_t* bad,
+                         uint32_t* outdeg, uint32_t* indeg) {
+  GRID_STRIDE(i, hi - lo) {
+    const uint64_t e = lo + i;
     const uint32_t s = src[e], d = dst[e];
     if (s >= V || d >= V) {
       *bad = 1;
       keys[e] = 0;
     } else {
       keys[e] = ((uint64_t)(d / N) << (bsrc + bn)) | ((uint64_t)s << bn) | (uint64_t)(d % N);
+      atomicAdd(&outdeg[s], 1u);
+      atomicAdd(&indeg[d], 1u);
     }
     ids[e] = (uint32_t)e;
   }
@@ -138,14 +146,6 @@ __global__ void k_windows_tail(const uint64_t* __restrict__ keys, const uint32_t
   }
 }
 
-__global__ void k_outdeg(const uint32_t* __restrict__ src, uint64_t E, uint32_t* outdeg) {
-  GRID_STRIDE(e, E) atomicAdd(&outdeg[src[e]], 1u);
-}
-// largest in-degree: the shard entries of one destination are consecutive
-// within its shard only after sorting by dst, so count with atomics instead
-__global__ void k_indeg(const uint32_t* __restrict__ dst, uint64_t E, uint32_t* indeg) {
-  GRID_STRIDE(e, E) atomicAdd(&indeg[dst[e]], 1u);
-}
 __global__ void k_max_u32(const uint32_t* __restrict__ a, uint64_t n, uint32_t* out) {
   uint32_t m = 0;
   GRID_STRIDE(i, n) m = max(m, a[i]);
@@ -372,7 +372,8 @@ int build_runs(Graph& g, std::string& err) {
   return CUSHA_OK;
 }
 
-int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const uint32_t* d_val, std::string& err) {
+int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const uint32_t* d_val, std::string& err,
+                 const InputChunks* chunks) {
   cudaStream_t st = g.stream;
   const uint64_t E = g.E;
   const uint32_t V = g.V, N = g.N, S = g.S;
@@ -384,22 +385,39 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   PhaseTimer pt(st);
   t_alloc_stream = st;
 
-  DevBuf keys, keys2, ids, ids2, bad, start, padded, temp;
+  DevBuf keys, keys2, ids, ids2, bad, start, padded, temp, indeg, mx;
   CK(dalloc((uint64_t**)&keys.p, E));
   CK(dalloc((uint64_t**)&keys2.p, E));
   CK(dalloc((uint32_t**)&ids.p, E));
   CK(dalloc((uint32_t**)&ids2.p, E));
+  CK(dalloc(&g.d_outdeg, V));
+  CK(dalloc((uint32_t**)&indeg.p, V));
+  CK(dalloc((uint32_t**)&mx.p, 2));
   pt.mark("alloc keys/ids");
   CK(dalloc((uint32_t**)&bad.p, 1));
   CK(cudaMemsetAsync(bad.p, 0, 4, st));
-  if (E) k_make_keys<<<grid_for(E), 256, 0, st>>>(d_src, d_dst, E, V, N, bn, bsrc, (uint64_t*)keys.p, (uint32_t*)ids.p,
-                                                  (uint32_t*)bad.p);
+  CK(cudaMemsetAsync(g.d_outdeg, 0, (size_t)V * 4, st));
+  CK(cudaMemsetAsync(indeg.p, 0, (size_t)V * 4, st));
+  CK(cudaMemsetAsync(mx.p, 0, 8, st));
+  // keys + degrees per input chunk, each as soon as its host copy has landed
+  const int nchunks = chunks && chunks->n ? chunks->n : 1;
+  for (int c = 0; c < nchunks; ++c) {
+    const uint64_t lo = chunks && chunks->n ? chunks->bounds[c] : 0, hi = chunks && chunks->n ? chunks->bounds[c + 1] : E;
+    if (chunks && chunks->n) CK(cudaStreamWaitEvent(st, chunks->ready[c], 0));
+    if (hi > lo)
+      k_ingest<<<grid_for(hi - lo), 256, 0, st>>>(d_src, d_dst, lo, hi, V, N, bn, bsrc, (uint64_t*)keys.p,
+                                                  (uint32_t*)ids.p, (uint32_t*)bad.p, g.d_outdeg, (uint32_t*)indeg.p);
+  }
   CK(cudaGetLastError());
-  uint32_t h_bad = 0;
-  CK(cudaMemcpyAsync(&h_bad, bad.p, 4, cudaMemcpyDeviceToHost, st));
+  // range of the float algorithms' fixed-point sums (include/cusha.h "Fixed-point range")
+  k_max_u32<<<grid_for(V), 256, 0, st>>>((uint32_t*)indeg.p, V, (uint32_t*)mx.p);
+  uint32_t h[2] = {0, 0};
+  CK(cudaMemcpyAsync(h, mx.p, 4, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(h + 1, bad.p, 4, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
-  if (h_bad) { err = "edge endpoint >= num_vertices"; return CUSHA_EINVAL; }
-  pt.mark("keys + validate");
+  if (h[1]) { err = "edge endpoint >= num_vertices"; return CUSHA_EINVAL; }
+  g.max_indeg = h[0];
+  pt.mark("keys + degrees + validate");
 
   // ---- G-Shards order
   cub::DoubleBuffer<uint64_t> kb((uint64_t*)keys.p, (uint64_t*)keys2.p);
@@ -443,6 +461,12 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   if (g.keep_ids) CK(dalloc(&g.d_eid, P));  // layout inspection only (no kernel reads it)
   if (d_val) { CK(dalloc(&g.d_ev, P)); g.has_ev = true; }
   pt.mark("offsets + alloc shard arrays");
+  if (chunks && chunks->n) CK(cudaStreamWaitEvent(st, chunks->all, 0));  // the edge values' copy trails the src/dst chunks
+  uint32_t ev_bits = 0;
+  if (d_val && E) {
+    k_max_abs_f32<<<grid_for(E), 256, 0, st>>>(d_val, E, (uint32_t*)mx.p + 1);
+    CK(cudaMemcpyAsync(&ev_bits, (uint32_t*)mx.p + 1, 4, cudaMemcpyDeviceToHost, st));
+  }
   k_fill_shard_pads<<<grid_for((uint64_t)S * kPad), 256, 0, st>>>(g.d_shard_off, g.d_shard_cnt, S, N, g.d_dest,
                                                                    g.d_srcloc, g.d_eid, g.d_ev);
   if (E)
@@ -461,24 +485,6 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
 
   // ---- out-degrees (PR NbrsNum, L318) and |CW_i|
   pt.mark("window table");
-  CK(dalloc(&g.d_outdeg, V));
-  CK(cudaMemsetAsync(g.d_outdeg, 0, (size_t)V * 4, st));
-  if (E) k_outdeg<<<grid_for(E), 256, 0, st>>>(d_src, E, g.d_outdeg);
-  {  // range of the float algorithms' fixed-point sums (include/cusha.h "Fixed-point range")
-    DevBuf indeg, mx;
-    CK(dalloc((uint32_t**)&indeg.p, V));
-    CK(dalloc((uint32_t**)&mx.p, 2));
-    CK(cudaMemsetAsync(indeg.p, 0, (size_t)V * 4, st));
-    CK(cudaMemsetAsync(mx.p, 0, 8, st));
-    if (E) k_indeg<<<grid_for(E), 256, 0, st>>>(d_dst, E, (uint32_t*)indeg.p);
-    k_max_u32<<<grid_for(V), 256, 0, st>>>((uint32_t*)indeg.p, V, (uint32_t*)mx.p);
-    if (d_val && E) k_max_abs_f32<<<grid_for(E), 256, 0, st>>>(d_val, E, (uint32_t*)mx.p + 1);
-    uint32_t h[2] = {0, 0};
-    CK(cudaMemcpyAsync(h, mx.p, 8, cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    g.max_indeg = h[0];
-    std::memcpy(&g.max_abs_ev, &h[1], 4);
-  }
   CK(dalloc(&g.d_cw_cnt, S));
   k_cw_counts<<<S, 256, 0, st>>>(g.d_outdeg, V, N, g.d_cw_cnt);
   CK(cudaGetLastError());
@@ -529,6 +535,7 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   }
   pt.mark("Mapper runs");
   CK(cudaStreamSynchronize(st));
+  std::memcpy(&g.max_abs_ev, &ev_bits, 4);
   return CUSHA_OK;
 }
 

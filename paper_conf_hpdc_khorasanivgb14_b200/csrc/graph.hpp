@@ -227,7 +227,17 @@ bool alg_needs_edge_values(int alg);
 bool alg_needs_init(int alg);
 
 // builder.cu
-int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const uint32_t* d_val, std::string& err);
+// Host inputs copied in chunks on a copy stream (row f2): chunk c = edges
+// [bounds[c], bounds[c+1]) of src/dst is on the device once ready[c] fired;
+// `all` fires after every copy (edge values included).
+struct InputChunks {
+  int n = 0;
+  uint64_t bounds[17] = {};
+  cudaEvent_t ready[16] = {};
+  cudaEvent_t all = nullptr;
+};
+int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const uint32_t* d_val, std::string& err,
+                 const InputChunks* chunks = nullptr);
 int build_runs(Graph& g, std::string& err);       // Mapper runs (CW, CUSHA_RLE builds)
 int offload_topology(Graph& g, std::string& err); // row f3: move shards >= host_shard to pinned host memory
 void partition_bounds(uint32_t S, const uint64_t* work, uint32_t G, uint32_t* bounds);
