@@ -176,6 +176,10 @@ typedef struct {
    *   the oracle's mode T pass for pass (tests/test_gpu_bsp.py).  Single
    *   partition only; one launch per pass plus a copy of SrcValue.         */
   int mode;
+  /* One process per GPU: how long (ms) a rank waits for its peers' collective
+   * before it aborts the communicator and returns CUSHA_ENCCL (an NCCL
+   * asynchronous error does the same at once).  0 = 300000.                 */
+  uint32_t comm_timeout_ms;
 } cusha_build_opts;
 
 enum { CUSHA_MODE_ASYNC = 0, CUSHA_MODE_BSP = 1 };

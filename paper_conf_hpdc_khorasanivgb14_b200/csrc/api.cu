@@ -158,7 +158,8 @@ static int connect_ipc_peers(Graph& g) {
   CKA(dev_alloc(&drecv, sizeof(mine) * G, g.stream));
   CKA(cudaMemcpyAsync(dsend, mine, sizeof(mine), cudaMemcpyHostToDevice, g.stream));
   std::string err;
-  const int rc = nccl_allgather_bytes(g, dsend, drecv, sizeof(mine), err);
+  int rc = nccl_allgather_bytes(g, dsend, drecv, sizeof(mine), err);
+  if (!rc) rc = nccl_wait(g, g.comm_timeout_ms, err);
   if (rc) return fail(rc, "IPC handle exchange: " + err);
   std::vector<cudaIpcMemHandle_t> all(2 * G);
   CKA(cudaMemcpyAsync(all.data(), drecv, sizeof(mine) * G, cudaMemcpyDeviceToHost, g.stream));
@@ -414,6 +415,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
       CKA(cudaStreamSynchronize(h->stream));
     } else {
       Graph& p = *h->parts[0];
+      p.comm_timeout_ms = o.comm_timeout_ms ? o.comm_timeout_ms : 300000u;
       if ((rc = nccl_init(p, o.nccl_unique_id, err))) {
         set_error("NCCL: " + err);
         return bail(rc);
@@ -823,7 +825,11 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
         CKA(cudaGraphLaunch(h->exec[a], st));
       }
       CKA(cudaMemcpyAsync(g.h_ctl, g.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, st));
-      CKA(cudaStreamSynchronize(st));
+      if (h->mode == kModeNccl) {  // never hang on a failed peer
+        if ((rc = nccl_wait(g, g.comm_timeout_ms, err))) return fail(rc, err);
+      } else {
+        CKA(cudaStreamSynchronize(st));
+      }
       if (g.h_ctl->converged || g.h_ctl->iter >= max_iters) break;
     }
   }
@@ -896,7 +902,8 @@ static int copy_values(const cusha_graph* h, void* dst, bool to_host) {
     void* full = nullptr;
     CKA(dev_alloc(&full, (size_t)V * vb, h->stream));
     std::string err;
-    const int rc = nccl_gather_values(g, full, (uint32_t)vb, err);
+    int rc = nccl_gather_values(g, full, (uint32_t)vb, err);
+    if (!rc) rc = nccl_wait(g, g.comm_timeout_ms, err);
     if (rc) {
       cudaFreeAsync(full, h->stream);
       return fail(rc, "gather: " + err);

@@ -206,6 +206,7 @@ struct Graph {
   uint32_t** d_dirty_peer = nullptr;// G: dirty[] of every partition (skip_clean only)
   std::vector<void*> ipc_open;      // peer allocations mapped with cudaIpcOpenMemHandle
   void* nccl_comm = nullptr;        // ncclComm_t (real multi-GPU)
+  uint32_t comm_timeout_ms = 300000;
   // stats
   cusha_stats st{};
   int last_alg = -1;
@@ -259,6 +260,7 @@ int nccl_init(Graph& g, const void* id128, std::string& err);
 int nccl_allgather_bytes(Graph& g, const void* dsend, void* drecv, size_t bytes, std::string& err);
 int nccl_allreduce_max_u32(Graph& g, const uint32_t* dsend, uint32_t* drecv, std::string& err);
 int nccl_gather_values(Graph& g, void* dfull, uint32_t value_bytes, std::string& err);  // every rank's vv slice
+int nccl_wait(Graph& g, uint32_t timeout_ms, std::string& err);  // stream drained, or abort on error / timeout
 void nccl_destroy(Graph& g);
 
 }  // namespace cusha

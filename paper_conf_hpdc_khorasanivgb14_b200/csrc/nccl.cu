@@ -13,7 +13,9 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cstring>
+#include <thread>
 #include <string>
 
 #include "graph.hpp"
@@ -30,6 +32,8 @@ struct NcclApi {
   decltype(&ncclBroadcast) broadcast = nullptr;
   decltype(&ncclAllGather) allGather = nullptr;
   decltype(&ncclAllReduce) allReduce = nullptr;
+  decltype(&ncclCommGetAsyncError) asyncError = nullptr;
+  decltype(&ncclCommAbort) commAbort = nullptr;
   decltype(&ncclGroupStart) groupStart = nullptr;
   decltype(&ncclGroupEnd) groupEnd = nullptr;
   decltype(&ncclGetErrorString) errorString = nullptr;
@@ -50,11 +54,13 @@ const NcclApi& api() {
     x.broadcast = reinterpret_cast<decltype(x.broadcast)>(dlsym(h, "ncclBroadcast"));
     x.allGather = reinterpret_cast<decltype(x.allGather)>(dlsym(h, "ncclAllGather"));
     x.allReduce = reinterpret_cast<decltype(x.allReduce)>(dlsym(h, "ncclAllReduce"));
+    x.asyncError = reinterpret_cast<decltype(x.asyncError)>(dlsym(h, "ncclCommGetAsyncError"));
+    x.commAbort = reinterpret_cast<decltype(x.commAbort)>(dlsym(h, "ncclCommAbort"));
     x.groupStart = reinterpret_cast<decltype(x.groupStart)>(dlsym(h, "ncclGroupStart"));
     x.groupEnd = reinterpret_cast<decltype(x.groupEnd)>(dlsym(h, "ncclGroupEnd"));
     x.errorString = reinterpret_cast<decltype(x.errorString)>(dlsym(h, "ncclGetErrorString"));
     x.ok = x.getUniqueId && x.commInitRank && x.commDestroy && x.broadcast && x.groupStart && x.groupEnd &&
-           x.errorString && x.allGather && x.allReduce;
+           x.errorString && x.allGather && x.allReduce && x.asyncError && x.commAbort;
     if (!x.ok) x.why = "libnccl.so.2 lacks a required symbol";
     return x;
   }();
@@ -91,11 +97,13 @@ int nccl_init(Graph& g, const void* id128, std::string& err) {
 }
 
 int nccl_allgather_bytes(Graph& g, const void* dsend, void* drecv, size_t bytes, std::string& err) {
+  if (!g.nccl_comm) { err = "the NCCL communicator was aborted"; return CUSHA_ENCCL; }
   NC(api().allGather(dsend, drecv, bytes, ncclUint8, static_cast<ncclComm_t>(g.nccl_comm), g.stream));
   return CUSHA_OK;
 }
 
 int nccl_allreduce_max_u32(Graph& g, const uint32_t* dsend, uint32_t* drecv, std::string& err) {
+  if (!g.nccl_comm) { err = "the NCCL communicator was aborted"; return CUSHA_ENCCL; }
   NC(api().allReduce(dsend, drecv, 1, ncclUint32, ncclMax, static_cast<ncclComm_t>(g.nccl_comm), g.stream));
   return CUSHA_OK;
 }
@@ -103,6 +111,7 @@ int nccl_allreduce_max_u32(Graph& g, const uint32_t* dsend, uint32_t* drecv, std
 // Rank r broadcasts its VertexValues slice (its vertices [v0, v0 + nvl)) into
 // the same place of every rank's |V|-element buffer dfull.
 int nccl_gather_values(Graph& g, void* dfull, uint32_t vb, std::string& err) {
+  if (!g.nccl_comm) { err = "the NCCL communicator was aborted"; return CUSHA_ENCCL; }
   ncclComm_t comm = static_cast<ncclComm_t>(g.nccl_comm);
   char* full = static_cast<char*>(dfull);
   NC(api().groupStart());
@@ -114,6 +123,43 @@ int nccl_gather_values(Graph& g, void* dfull, uint32_t vb, std::string& err) {
   }
   NC(api().groupEnd());
   return CUSHA_OK;
+}
+
+// Wait for the work enqueued on g.stream so far without hanging on a failed
+// peer: poll the stream and NCCL's asynchronous error state; on an NCCL error
+// or after timeout_ms the communicator is aborted (every pending collective
+// returns) and CUSHA_ENCCL is returned.
+int nccl_wait(Graph& g, uint32_t timeout_ms, std::string& err) {
+  cudaEvent_t ev;
+  if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess) { err = "event"; return CUSHA_ECUDA; }
+  cudaEventRecord(ev, g.stream);
+  const auto t0 = std::chrono::steady_clock::now();
+  ncclComm_t comm = static_cast<ncclComm_t>(g.nccl_comm);
+  int rc = CUSHA_OK;
+  for (;;) {
+    const cudaError_t q = cudaEventQuery(ev);
+    if (q == cudaSuccess) break;
+    if (q != cudaErrorNotReady) { err = std::string("stream: ") + cudaGetErrorString(q); rc = CUSHA_ECUDA; break; }
+    ncclResult_t ar = ncclSuccess;
+    if (api().asyncError(comm, &ar) != ncclSuccess || (ar != ncclSuccess && ar != ncclInProgress)) {
+      err = std::string("NCCL asynchronous error: ") + api().errorString(ar);
+      rc = CUSHA_ENCCL;
+      break;
+    }
+    const double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    if (ms > timeout_ms) {
+      err = "NCCL timeout: a rank did not reach the collective within " + std::to_string(timeout_ms) + " ms";
+      rc = CUSHA_ENCCL;
+      break;
+    }
+    std::this_thread::sleep_for(std::chrono::microseconds(50));
+  }
+  cudaEventDestroy(ev);
+  if (rc == CUSHA_ENCCL) {
+    api().commAbort(comm);
+    g.nccl_comm = nullptr;
+  }
+  return rc;
 }
 
 void nccl_destroy(Graph& g) {

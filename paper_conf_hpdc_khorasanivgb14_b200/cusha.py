@@ -52,6 +52,7 @@ class BuildOpts(ctypes.Structure):
         ("pass_barrier", ctypes.c_int),
         ("keep_layout", ctypes.c_int),
         ("mode", ctypes.c_int),
+        ("comm_timeout_ms", ctypes.c_uint32),
     ]
 
 

@@ -92,7 +92,7 @@ def test_c5_pagerank_residual(c5):
 
 
 GOLD = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", "c5_pr_sample.npz")
-FULL = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden_cache", "c5_pr_xstar.f64")
+FULL = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden_cache", "c5_pr_xstar.f32")
 
 
 def test_c5_pagerank_vs_oracle_1e9(c5):
@@ -106,7 +106,7 @@ def test_c5_pagerank_vs_oracle_1e9(c5):
     maxerr, n_abs = pr_check(x[idx], z["xstar"])
     print(f"C5 PR sample: {idx.size} vertices (incl. the 2,000 largest x*), max|err| {maxerr:.2e}, "
           f"{n_abs} over 1e-4 abs; oracle {int(z['sweeps'])} sweeps")
-    if os.path.exists(FULL) and os.path.getsize(FULL) == 8 * c5.V:
-        xs = np.fromfile(FULL, np.float64)
+    if os.path.exists(FULL) and os.path.getsize(FULL) == 4 * c5.V:
+        xs = np.fromfile(FULL, np.float32).astype(np.float64)   # x* rounded to f32: 6e-8 relative
         maxerr, n_abs = pr_check(x, xs)
         print(f"C5 PR all {c5.V} vertices: max|err| {maxerr:.2e}, {n_abs} over 1e-4 abs")

@@ -239,3 +239,25 @@ def test_pr_residual_vs_dense_and_fixed_point():
     np.testing.assert_allclose(oracle.pagerank_residual(V, s, d, x), want, atol=1e-12)
     xs, _ = oracle.pagerank(V, s, d, tol=1e-13)
     assert np.abs(oracle.pagerank_residual(V, s, d, xs.astype(np.float32))).max() < 1e-5
+
+
+def test_c5_golden_sample_is_consistent():
+    """The committed C5 PageRank sample (tools/golden_c5_pr.py: oracle.pagerank to
+    1e-9 on graphgen C5) is internally consistent: the config's sizes, a sorted
+    sample that contains the 16 first vertices, every x* >= 1 - d (R6: x = (1-d)
+    + d * a non-negative sum), and the mass below |V| (R6: sum x* = |V| minus the
+    dangling leak).  With the git-ignored full vector present, the sample equals
+    its entries and the recorded SHA-256 matches."""
+    import hashlib
+    import os
+    z = np.load(os.path.join(os.path.dirname(__file__), "golden", "c5_pr_sample.npz"))
+    V = int(z["V"])
+    assert V == 1 << 26 and int(z["E"]) == 1 << 30 and float(z["tol"]) == 1e-9
+    idx = z["idx"].astype(np.int64)
+    assert (np.diff(idx) > 0).all() and idx[0] == 0 and (idx[:16] == np.arange(16)).all() and idx[-1] < V
+    assert (z["xstar"] >= 0.15 - 1e-12).all()
+    assert 0 < float(z["mass"]) < V
+    full = os.path.join(os.path.dirname(__file__), "golden_cache", "c5_pr_xstar.f32")
+    if os.path.exists(full):
+        xs = np.fromfile(full, np.float32)
+        np.testing.assert_array_equal(xs[idx], z["xstar"].astype(np.float32))

@@ -10,9 +10,11 @@ oracle.pagerank (fp64 Jacobi of Table 3, R6-R8) to max |dx| <= 1e-9
                                      vertices plus the 2,000 largest x*, their
                                      x* (fp64), the sweep count, the mass sum,
                                      and the SHA-256 of the full fp64 vector;
-  tests/golden_cache/c5_pr_xstar.f64 git-ignored: the full x* vector (537 MB)
-                                     for the element-by-element leg
-                                     (tests/test_gpu_c5_parity.py), when present.
+  tests/golden_cache/c5_pr_xstar.f32 git-ignored: the full x* vector rounded
+                                     to float32 (268 MB; relative rounding
+                                     6e-8, far inside the 1e-4 bound) for the
+                                     element-by-element leg of
+                                     tests/test_gpu_fullsize.py, when present.
 Nothing here reads the CUDA path."""
 import hashlib
 import os
@@ -43,7 +45,7 @@ def main():
                         sweeps=np.int64(sweeps), V=np.int64(wl.V), E=np.int64(wl.E), mass=np.float64(x.sum()),
                         sha256=np.array(digest), tol=np.float64(1e-9))
     os.makedirs(os.path.join(ROOT, "tests", "golden_cache"), exist_ok=True)
-    x.tofile(os.path.join(ROOT, "tests", "golden_cache", "c5_pr_xstar.f64"))
+    x.astype(np.float32).tofile(os.path.join(ROOT, "tests", "golden_cache", "c5_pr_xstar.f32"))
     print(f"wrote sample ({idx.size} vertices) and full vector; sha256 {digest}", flush=True)
 
 
