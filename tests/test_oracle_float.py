@@ -246,9 +246,8 @@ def test_c5_golden_sample_is_consistent():
     1e-9 on graphgen C5) is internally consistent: the config's sizes, a sorted
     sample that contains the 16 first vertices, every x* >= 1 - d (R6: x = (1-d)
     + d * a non-negative sum), and the mass below |V| (R6: sum x* = |V| minus the
-    dangling leak).  With the git-ignored full vector present, the sample equals
-    its entries and the recorded SHA-256 matches."""
-    import hashlib
+    dangling leak).  With the git-ignored full vector (float32) present, the
+    sample equals its entries."""
     import os
     z = np.load(os.path.join(os.path.dirname(__file__), "golden", "c5_pr_sample.npz"))
     V = int(z["V"])
