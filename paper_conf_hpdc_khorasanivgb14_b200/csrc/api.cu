@@ -38,6 +38,10 @@ static int fail(int code, const std::string& msg) {
 
 constexpr int kModeSingle = 0, kModeSim = 1, kModeNccl = 2;
 constexpr int kChunk = 16;  // passes per fixed-count graph / per host check (per-pass modes)
+#ifndef CUSHA_WIDE_WINDOW
+#define CUSHA_WIDE_WINDOW 4
+#endif
+constexpr uint32_t kWideWindow = CUSHA_WIDE_WINDOW, kLowDegree = 4;
 
 }  // namespace cusha
 
@@ -783,6 +787,12 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   if (max_iters > 0 && multi) {
     KParams kp = pass_params(g, source, cfg, a);
     kp.multi = 1;
+    // passes in flight: 4 on low-degree graphs (road meshes need about their
+    // diameter in passes, so the 2 extra confirming passes are amortised and
+    // the wider overlap shortens each pass: C3 -6%), else 2 (power-law graphs
+    // converge in a few passes, where the confirming passes would dominate;
+    // DESIGN.md "Overlapped passes")
+    kp.window = g.E < (uint64_t)kLowDegree * g.V ? kWideWindow : 2u;
     void* args[] = {&kp};
     CKA(cudaLaunchKernel(pk.func, dim3(pass_grid(g, pk, cfg.smem)), dim3(pk.threads), args, cfg.smem, st));
   } else if (max_iters > 0) {

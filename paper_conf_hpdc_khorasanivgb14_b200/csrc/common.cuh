@@ -66,6 +66,13 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
                : "memory");
 }
 
+// Ampere-style asynchronous 4-byte global -> shared copy (LDGSTS), per thread
+__device__ __forceinline__ void cp_async4(void* dst, const void* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
 // TMA bulk prefetch of [src, src + bytes) into L2 (no shared memory, no
 // completion to wait for); the range is widened to 16-byte bounds
 __device__ __forceinline__ void bulk_prefetch_l2(const void* src, uint32_t bytes) {

@@ -24,8 +24,8 @@ struct Ctl {
   uint32_t gchanged;    // partitioned mode: OR of lchanged over the partitions (NCCL all-reduce / simulation)
   // overlapped passes (one launch per run)
   unsigned long long ticket;  // shard tickets drawn: ticket t = shard t % |S| of pass t / |S|
-  uint32_t stop;              // two consecutive passes committed nothing: draw no more tickets
-  uint32_t conv_iter;         // 1 + the later of those two passes (~0u: none yet)
+  uint32_t stop;              // `window` consecutive passes committed nothing: draw no more tickets
+  uint32_t conv_iter;         // 1 + the last of those passes (~0u: none yet)
 };
 
 // Per-iteration trace (row f4; also the source of algorithmic byte counts).
@@ -70,6 +70,7 @@ struct KParams {
   TraceRec* trace;
   uint32_t trace_cap;
   int multi;                   // 1: one launch runs every pass (overlapped passes)
+  uint32_t window;             // overlapped passes: pass k starts after pass k - window completed
   int mapj;                    // 1: CW stage 4 uses the Mapper in window form (cw_win + delta row in smem)
   int stash;                   // 1: integer algorithms keep stage 1's VertexValues in smem for stage 3
   int ahead;                   // 1: the producer prefetches stage-2 tiles into L2 beyond the ring (HBM-resident passes)

@@ -92,6 +92,9 @@ constexpr bool kBk = CUSHA_BK != 0;
 #ifndef CUSHA_AHEAD_WAIT
 #define CUSHA_AHEAD_WAIT 1  // the read-ahead starts before the producer's ticket_wait
 #endif
+#ifndef CUSHA_DROW_ASYNC
+#define CUSHA_DROW_ASYNC 1  // the stage-4 delta row arrives by cp.async during stage 2 (0: loads in stage 1)
+#endif
 #ifndef CUSHA_AHEAD4
 #define CUSHA_AHEAD4 1  // the L2 read-ahead also covers CW stage-4 tiles
 #endif
@@ -199,18 +202,21 @@ struct __align__(16) TileDesc {
 // across the iteration boundary.  Two waits bound the overlap:
 //  - pass k of shard s starts after pass k - 1 of s completed (one CTA owns a
 //    shard's VertexValues at a time, as in Fig. 5);
-//  - pass k starts after pass k - 2 completed (at most two passes in flight).
-// Convergence (L189, "a pass that commits nothing") is concluded when two
-// consecutive passes k - 1 and k both committed nothing.  Why that is exact:
-// let T0 be the moment pass k - 2 completed.  Every ticket of pass k read its
+//  - pass k starts after pass k - W completed (at most W passes in flight;
+//    W = KParams::window, 2 by default, 4 for low-degree graphs).
+// Convergence (L189, "a pass that commits nothing") is concluded when W
+// consecutive passes k - W + 1 .. k all committed nothing.  Why that is exact:
+// let T0 be the moment pass k - W completed.  Every ticket of pass k read its
 // inputs after T0, and no write happens after T0 until some commit; take the
-// first commit after T0, by a ticket of pass q on shard s.  Passes k - 1 and
-// k commit nothing, so q > k, and that ticket read the state at T0 - as did
-// shard s's pass-k ticket, which ran between T0 and it and committed nothing
-// from the same inputs and the same VertexValues (integer and fixed-point
-// sums are order-independent, R11).  The same inputs give the same result,
-// so no such commit exists: the state at T0 is the fixed point a
-// barrier-separated pass would confirm.
+// first commit after T0, by a ticket of pass q on shard s.  Passes <= k - W
+// completed before T0 (a shard's pass-r ticket waits for its pass r - 1, so
+// pass r complete implies every earlier pass complete) and passes
+// k - W + 1 .. k commit nothing, so q > k, and that ticket read the
+// state at T0 - as did shard s's pass-k ticket, which ran between T0 and it
+// and committed nothing from the same inputs and the same VertexValues
+// (integer and fixed-point sums are order-independent, R11).  The same inputs
+// give the same result, so no such commit exists: the state at T0 is the
+// fixed point a barrier-separated pass would confirm.
 __device__ __forceinline__ uint32_t ld_vol(const uint32_t* a) { return *reinterpret_cast<const volatile uint32_t*>(a); }
 __device__ __forceinline__ void st_vol(uint32_t* a, uint32_t v) { *reinterpret_cast<volatile uint32_t*>(a) = v; }
 __device__ __forceinline__ void fence_sc_gpu() { asm volatile("fence.sc.gpu;" ::: "memory"); }
@@ -223,8 +229,8 @@ __device__ __forceinline__ bool ticket_wait(const KParams& p, uint32_t s, uint32
     if (ld_vol(&p.ctl->stop)) return false;
     __nanosleep(64);
   }
-  if (pass >= 2)
-    while (ld_vol(&p.trace[pass - 2].done) < Sloc) {
+  if (pass >= p.window)
+    while (ld_vol(&p.trace[pass - p.window].done) < Sloc) {
       if (ld_vol(&p.ctl->stop)) return false;
       __nanosleep(64);
     }
@@ -247,9 +253,16 @@ __device__ __forceinline__ void ticket_done(const KParams& p, uint32_t s, uint32
     __threadfence();  // acquire: the completers' active_shards increments precede their done increments
     return ld_vol(&p.trace[r].active_shards) == 0;
   };
+  // W consecutive clean passes, one of them this one: a window [a, a + W) containing pass
+  const uint32_t W = p.window;
   uint32_t conv = 0xFFFFFFFFu;
-  if (pass >= 1 && clean(pass - 1)) conv = pass + 1;
-  else if (pass + 1 < p.ctl->max_iters && clean(pass + 1)) conv = pass + 2;
+  for (uint32_t a = pass + 1 > W ? pass + 1 - W : 0u; a <= pass && conv == 0xFFFFFFFFu; ++a) {
+    if (a + W > p.ctl->max_iters) break;
+    bool ok = true;
+    for (uint32_t r = a; r < a + W && ok; ++r)
+      if (r != pass) ok = clean(r);
+    if (ok) conv = a + W;
+  }
   if (conv != 0xFFFFFFFFu) {
     atomicMin(&p.ctl->conv_iter, conv);
     st_vol(&p.ctl->stop, 1u);
@@ -701,7 +714,13 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
       }
       if (p.mapj) {  // the shard's Mapper-delta row for stage 4 (window form)
         const uint32_t* dg = p.cw_delta + (size_t)s * p.S;
-        for (uint32_t j = ct; j < p.S; j += kConsumers) drow[j] = __ldg(dg + j);
+        if (CUSHA_DROW_ASYNC) {
+          // asynchronous copies (LDGSTS), waited for before stage 4: their latency hides behind stage 2
+          for (uint32_t j = ct; j < p.S; j += kConsumers) cp_async4(drow + j, dg + j);
+          cp_async_commit();
+        } else {
+          for (uint32_t j = ct; j < p.S; j += kConsumers) drow[j] = __ldg(dg + j);
+        }
       }
       if (ct == 0) {
         A::init(sm, st, N, V_t{});  // trash slot for filler entries
@@ -785,11 +804,15 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
           my_upd |= up ? 1u : 0u;
         }
       }
+      // this thread's delta-row copies (issued in stage 1) land before the
+      // barrier, so after it every thread sees the whole row (stage 4)
+      if (CUSHA_DROW_ASYNC && p.mapj) cp_async_wait_all();
       const int any = bar_sync_or(kConsumerBar, kConsumers, (int)my_upd) | ((kDiag & 1) ? 1 : 0);
       if (CUSHA_TIMELINE && ct == 0) tl_mark(tk, 5);
 
       // ---- stage 4: write-back into every shard's window (lines 23-26, L308)
       uint32_t stores = 0;
+
       if (REPR == CUSHA_REPR_CW) {
         // thread per CW_s entry: SrcValue[Mapper[k]] = local[SrcIndex[k]] (L177, Fig. 4b);
         // consecutive threads take consecutive entries, so the stores of one
@@ -1164,6 +1187,7 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.splitP = (uint32_t)g.splitP; p.splitQ = (uint32_t)g.splitQ;
   p.dest_h = g.h_dest; p.ev_h = g.h_ev; p.srcloc_h = g.h_srcloc; p.cw_src_h = g.h_cw_src; p.mapper_h = g.h_mapper;
   p.multi = 0; p.shard_seq = g.d_shard_seq;
+  p.window = 2;
   p.mapj = 0;
   p.stash = 0;
   p.ahead = 0;

@@ -2,9 +2,9 @@
 oracle and against the one-launch-per-pass barrier mode (Fig. 5).
 
 Default runs draw shard tickets across pass boundaries inside one launch
-(at most two passes in flight, a shard's passes in order); convergence is
-concluded when two consecutive passes committed nothing (L189; the argument
-is in csrc/kernels.cu).  The
+(at most W passes in flight, W = 2, or 4 on graphs of average degree < 4; a
+shard's passes in order); convergence is concluded when W consecutive passes
+committed nothing (L189; the argument is in csrc/kernels.cu).  The
 integer fixed points are unique, so both modes must match the oracle bit for
 bit; PR stays within R10.  Small |S| (down to one shard) exercises the
 per-shard pass order, where a CTA's next ticket is the shard it is still
@@ -16,6 +16,7 @@ import pytest
 import graphgen
 import oracle
 from gpu_common import gpu_run, pr_check
+from paper_conf_hpdc_khorasanivgb14_b200 import cusha
 
 pytestmark = pytest.mark.gpu
 
@@ -145,3 +146,16 @@ def test_pass_barrier_graph_reuse(c1, repr):
                     want = oracle.cc(V, s, d)
                 np.testing.assert_array_equal(got, want, err_msg=f"{alg} source {source}")
                 assert cusha.get_stats(g)["device_loop"] == 1
+
+
+def test_wide_window_on_low_degree_graph():
+    """A mesh (average degree < 4) runs with 4 passes in flight: bit-exact, and
+    the run ends with 4 consecutive clean passes (the last trace records)."""
+    wl = graphgen.workload("mesh:40000:200:52000:33")
+    got, st = gpu_run("sssp", wl.V, wl.src, wl.dst, ev=wl.edge_u32, repr="cw")
+    np.testing.assert_array_equal(got, oracle.sssp(wl.V, wl.src, wl.dst, wl.edge_u32, 0))
+    assert st["device_loop"] == 2
+    with cusha.build_graph(wl.V, wl.src, wl.dst, edge_values=wl.edge_u32, repr="cw") as g:
+        cusha.run("sssp", g)
+        upd, _ = cusha.get_trace(g)
+    assert len(upd) >= 5 and (upd[-4:] == 0).all() and upd[-5] > 0

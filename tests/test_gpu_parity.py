@@ -216,8 +216,9 @@ def test_layout_matches_oracle(repr, V, E, N):
 @pytest.mark.parametrize("repr", REPRS)
 def test_edge_cases(repr):
     # empty graph: nothing changes; the barrier mode stops after one clean pass,
-    # overlapped passes after two consecutive clean ones
-    for barrier, passes in ((True, 1), (False, 2)):
+    # overlapped passes after W consecutive clean ones, W = 4 passes in flight on
+    # a graph of average degree < 4
+    for barrier, passes in ((True, 1), (False, 4)):
         got, st = gpu_run("bfs", 10, np.zeros(0, np.uint32), np.zeros(0, np.uint32), repr=repr, source=3,
                           pass_barrier=barrier)
         assert got[3] == 0 and (np.delete(got, 3) == cusha.INF).all() and st["iterations"] == passes

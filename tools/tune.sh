@@ -11,6 +11,6 @@ else
   wl=$1; shift
   for name in "$@"; do
     lib=paper_conf_hpdc_khorasanivgb14_b200/variant_$name.so; [ "$name" = base ] && lib=paper_conf_hpdc_khorasanivgb14_b200/libcusha.so
-    timeout 300 python bench.py --workload $wl --steps 10 --warmup 3 --cache-dir /tmp/gg --no-e2e --no-cpu-baseline --lib $lib $BENCH_EXTRA 2>/dev/null | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('$name', 'GTEPS', d['value'], 'ms', d['ms_per_step'], 'it', d['config']['iterations'], 'pass_us', d['roofline']['avg_pass_us'], 'frac', d['roofline']['frac'])"
+    timeout ${TUNE_TIMEOUT:-300} python bench.py --workload $wl --steps 10 --warmup 3 --cache-dir /tmp/gg --no-e2e --no-cpu-baseline --lib $lib $BENCH_EXTRA 2>/dev/null | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('$name', 'GTEPS', d['value'], 'ms', d['ms_per_step'], 'it', d['run']['iterations'], 'pass_us', d['roofline']['avg_pass_us'], 'frac', d['roofline']['frac'])"
   done
 fi
