@@ -92,6 +92,9 @@ constexpr bool kBk = CUSHA_BK != 0;
 #ifndef CUSHA_AHEAD_WAIT
 #define CUSHA_AHEAD_WAIT 1  // the read-ahead starts before the producer's ticket_wait
 #endif
+#ifndef CUSHA_EARLY_SEQ
+#define CUSHA_EARLY_SEQ 1  // a shard's next pass is released by the consumers at the end of its ticket, not by the bookkeeper
+#endif
 #ifndef CUSHA_DROW_ASYNC
 #define CUSHA_DROW_ASYNC 1  // the stage-4 delta row arrives by cp.async during stage 2 (0: loads in stage 1)
 #endif
@@ -209,8 +212,9 @@ struct __align__(16) TileDesc {
 // let T0 be the moment pass k - W completed.  Every ticket of pass k read its
 // inputs after T0, and no write happens after T0 until some commit; take the
 // first commit after T0, by a ticket of pass q on shard s.  Passes <= k - W
-// completed before T0 (a shard's pass-r ticket waits for its pass r - 1, so
-// pass r complete implies every earlier pass complete) and passes
+// finished writing before T0 (a shard's pass-r ticket starts after its pass
+// r - 1 finished writing, so pass r complete implies every earlier pass's
+// writes complete) and passes
 // k - W + 1 .. k commit nothing, so q > k, and that ticket read the
 // state at T0 - as did shard s's pass-k ticket, which ran between T0 and it
 // and committed nothing from the same inputs and the same VertexValues
@@ -242,9 +246,10 @@ __device__ __forceinline__ bool ticket_wait(const KParams& p, uint32_t s, uint32
 // ticket (s, pass) finished (its stores ordered before by the caller's
 // barrier; fences are cumulative).  The thread completing the last ticket of
 // a clean pass looks at both neighbouring passes.
-__device__ __forceinline__ void ticket_done(const KParams& p, uint32_t s, uint32_t pass, uint32_t Sloc) {
+__device__ __forceinline__ void ticket_done(const KParams& p, uint32_t s, uint32_t pass, uint32_t Sloc,
+                                            bool set_seq = true) {
   __threadfence();
-  st_vol(&p.shard_seq[s], pass + 1);
+  if (set_seq) st_vol(&p.shard_seq[s], pass + 1);
   if (atomicAdd(&p.trace[pass].done, 1u) != Sloc - 1) return;
   fence_sc_gpu();  // pairs with the other neighbour's completer: at least one of two sees both complete
   if (ld_vol(&p.trace[pass].active_shards) != 0) return;
@@ -625,8 +630,9 @@ __device__ __forceinline__ void ticket_bookkeeping(const KParams& p, uint32_t s,
       }
     }
   }
-  // overlapped passes: every consumer's stores precede this (barriers; fences are cumulative)
-  if (p.multi) ticket_done(p, s, it, Sloc);
+  // overlapped passes: every consumer's stores precede this (barriers; fences are cumulative);
+  // with CUSHA_EARLY_SEQ the consumers released the shard's next pass already
+  if (p.multi) ticket_done(p, s, it, Sloc, !(CUSHA_EARLY_SEQ && kBk));
 }
 
 template <class A, int REPR>
@@ -952,6 +958,14 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
       // ---- per-shard bookkeeping: convergence flag (line 26), predictor, trace
       if (ct == 0) {
         if (kBk) {
+          if (CUSHA_EARLY_SEQ && p.multi) {
+            // the shard's next pass may start now: every consumer's stores of this
+            // ticket precede this fence (barrier above; the fence is cumulative).
+            // The trace / done bookkeeping follows in the bookkeeper warp; the
+            // convergence argument needs only the writes complete (kernels.cu top)
+            __threadfence();
+            st_vol(&p.shard_seq[s], it + 1);
+          }
           // hand the ticket to the bookkeeper warp (every consumer's stores precede
           // this through the barrier above; the bookkeeper's fence is cumulative)
           const uint32_t b = ntk & 1u;
