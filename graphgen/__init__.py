@@ -150,8 +150,8 @@ def workload(name: str, cache_dir: Optional[str] = None) -> Workload:
     C4: HiggsTwitter-shaped symmetric R-MAT, V=456,631, 7,427,937 pairs
         (E=14,855,874), widths U[1,255] symmetric, seed 4 (CC, SSWP).
     C5: R-MAT scale 26, V=2^26, E=2^30, seed 5 (PR, BFS).
-    R27 / R28: R-MAT scale 27 / 28, edge factor 16, seeds 9 / 10 (row f3, graphs
-        near / beyond one GPU's HBM).
+    R27 / R28: R-MAT scale 27 / 28, edge factor 16 / 15, seeds 9 / 10 (row f3,
+        graphs near / beyond one GPU's HBM).
     """
     if cache_dir:
         path = os.path.join(cache_dir, f"graphgen_{name}.npz")
@@ -184,10 +184,11 @@ def workload(name: str, cache_dir: Optional[str] = None) -> Workload:
         V = 1 << 26
         src, dst = rmat(V, 1 << 30, seed=5)
     elif name in ("R27", "R28"):
-        # row f3 (L455): R-MAT scale 27 / 28, edge factor 16, seeds 9 / 10
+        # row f3 (L455): R-MAT scale 27 (edge factor 16) / 28 (edge factor 15:
+        # 4.03 G edges, below the ABI's 2^32 - 2^26 limit), seeds 9 / 10
         k = 27 if name == "R27" else 28
         V = 1 << k
-        src, dst = rmat(V, 16 << k, seed=k - 18)
+        src, dst = rmat(V, (16 if k == 27 else 15) << k, seed=k - 18)
     elif name.startswith("rmat:"):
         # rmat:V:E:seed  (parity-test sizes)
         _, V, E, seed = name.split(":")

@@ -15,7 +15,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 OUT = os.path.join(HERE, "libcusha.so")
 OBJDIR = os.path.join(HERE, "build")
-SOURCES = ["api.cu", "builder.cu", "kernels.cu", "nccl.cu"]
+SOURCES = ["api.cu", "builder.cu", "kernels.cu", "nccl.cu", "partition.cu"]
 
 
 def nccl_include() -> str:

@@ -248,8 +248,6 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
     return fail(CUSHA_EUNSUPPORTED, "the partitioned (multi-GPU) mode uses the CW representation");
   if (o.world_size > 1 && o.nccl_unique_id && (o.rank < 0 || o.rank >= o.world_size))
     return fail(CUSHA_EINVAL, "rank out of range");
-  if (o.world_size > 1 && o.device_topology_budget)
-    return fail(CUSHA_EUNSUPPORTED, "host-streamed topology is for a single partition (row f3)");
   uint32_t N = o.vertices_per_shard ? o.vertices_per_shard : cusha_shard_size(V, E, o.smem_bytes_per_vertex, 0, 0);
   if (N > 65534) return fail(CUSHA_EINVAL, "vertices_per_shard must be <= 65534");
   if (o.pass_barrier < 0 || o.pass_barrier > 2) return fail(CUSHA_EINVAL, "pass_barrier must be 0, 1 or 2");
@@ -317,7 +315,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
       if (c->all) cudaEventDestroy(c->all);
     }
   } cg{&chunks, &cs};
-  if (o.input_location == CUSHA_INPUT_HOST && E) {
+  if (h->mode == kModeSingle && o.input_location == CUSHA_INPUT_HOST && E) {
     // the host edge list crosses in chunks on a copy stream; the layout's first
     // pass (keys, degrees) consumes each chunk as it lands (DESIGN.md f2)
     const uint64_t nvals = edge_values ? 3 : 2;
@@ -351,11 +349,13 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
     h2d = nvals * E * 4;
   }
   std::string err;
-  rc = build_layout(g, d_src, d_dst, d_val, err, chunks.n ? &chunks : nullptr);
-  if (tmp) cudaFreeAsync(tmp, h->stream);  // stream order: the build waited for every copy
-  if (rc) {
-    set_error("build: " + err);
-    return bail(rc);
+  if (h->mode == kModeSingle) {
+    rc = build_layout(g, d_src, d_dst, d_val, err, chunks.n ? &chunks : nullptr);
+    if (tmp) cudaFreeAsync(tmp, h->stream);  // stream order: the build waited for every copy
+    if (rc) {
+      set_error("build: " + err);
+      return bail(rc);
+    }
   }
   if (h->mode == kModeSingle) {
     // CW reads no window table after the build (unless skipping clean shards or inspecting the layout)
@@ -371,15 +371,23 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
     }
     if ((rc = alloc_run_state(g, false))) return bail(rc);
   } else {
-    // destination-range partition (row e): split by work, then keep per
-    // partition only its shards and the CW of its source shards
-    std::vector<uint64_t> work;
-    if ((rc = partition_work(g, work, err))) {
+    // destination-range partition (row e): the shard-pair counts place the
+    // bounds (near-equal work); each partition then sorts only its own in- and
+    // out-edges, streamed from wherever the edge list lives (partition.cu)
+    PlanInput pin;
+    pin.V = V; pin.N = N; pin.E = E; pin.src = src; pin.dst = dst; pin.val = edge_values;
+    pin.host = o.input_location == CUSHA_INPUT_HOST; pin.stream = h->stream;
+    Plan plan;
+    struct PlanGuard {
+      Plan* p;
+      cudaStream_t s;
+      ~PlanGuard() { free_plan(*p, s); }
+    } pgd{&plan, h->stream};
+    if ((rc = plan_partitions(pin, G, plan, err))) {
       set_error("partition: " + err);
       return bail(rc);
     }
-    std::vector<uint32_t> bounds(G + 1);
-    partition_bounds(S, work.data(), G, bounds.data());
+    if (plan.bounds.size() - 1 != G) return bail(fail(CUSHA_EINVAL, "partition count"));
     std::vector<Graph*> parts;
     const uint32_t r0 = h->mode == kModeNccl ? (uint32_t)o.rank : 0u, r1 = h->mode == kModeNccl ? r0 + 1 : G;
     for (uint32_t r = r0; r < r1; ++r) {
@@ -387,8 +395,8 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
       if (!p) { for (Graph* x : parts) { free_device_arrays(*x); delete x; } return bail(fail(CUSHA_ENOMEM, "host")); }
       parts.push_back(p);
       p->device = o.device; p->stream = h->stream; p->skip_clean = g.skip_clean; p->host_loop = true;
-      p->pass_barrier = 1; p->world_size = o.world_size; p->rank = (int)r;
-      if ((rc = build_part(g, bounds, r, *p, h->mode == kModeNccl, err))) {
+      p->pass_barrier = 1; p->world_size = o.world_size; p->rank = (int)r; p->keep_ids = g.keep_ids;
+      if ((rc = build_part_direct(pin, plan, r, *p, err))) {
         for (Graph* x : parts) { free_device_arrays(*x); delete x; }
         set_error("partition: " + err);
         return bail(rc);
@@ -397,8 +405,17 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
         cudaFreeAsync(p->d_win, h->stream);
         p->d_win = nullptr;
       }
+      // row f3: the partition's per-entry topology beyond the budget goes to
+      // pinned host memory now, before the next partition's build needs HBM
+      p->topo_budget = g.topo_budget;
+      if ((rc = offload_topology(*p, err))) {
+        for (Graph* x : parts) { free_device_arrays(*x); delete x; }
+        set_error("host topology: " + err);
+        return bail(rc);
+      }
     }
-    // the global layout is released; the handle now holds the partitions
+    if (pin.host) h2d = (1 + 2ull * (r1 - r0)) * (edge_values ? 3 : 2) * 4 * E;  // the streamed passes
+    // the handle now holds the partitions
     free_device_arrays(g);
     delete glob;
     h->parts = parts;
@@ -459,7 +476,8 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
     st.max_part_device_bytes = std::max(st.max_part_device_bytes, b);
     st.entries_padded += p->P;
   }
-  st.host_bytes = g0(h).host_bytes;
+  st.host_bytes = 0;
+  for (Graph* p : h->parts) st.host_bytes += p->host_bytes;
   st.host_shard = g0(h).host_shard;
   *out = h;
   set_error("");

@@ -581,7 +581,7 @@ int move_tail(T*& dev, T*& host, uint64_t n, uint64_t split, cudaStream_t st, ui
 int offload_topology(Graph& g, std::string& err) {
   cudaStream_t st = g.stream;
   t_alloc_stream = st;
-  const uint32_t S = g.S;
+  const uint32_t S = g.Sl;  // the graph's (partition's) own shards
   g.splitP = g.P;
   g.splitQ = g.Q;
   g.host_shard = S;
@@ -626,155 +626,6 @@ void partition_bounds(uint32_t S, const uint64_t* work, uint32_t G, uint32_t* bo
     bounds[q] = s;
   }
   bounds[G] = S;
-}
-
-// ------------------------------------------------ destination-range partition (row e)
-// Work per shard for the split: stage-2 entries (its in-edges) + stage-4
-// entries (|CW_s|, the out-edges of its vertices).
-int partition_work(const Graph& glob, std::vector<uint64_t>& work, std::string& err) {
-  const uint32_t S = glob.S;
-  std::vector<uint32_t> cnt(S), ccnt(S, 0);
-  CK(cudaMemcpyAsync(cnt.data(), glob.d_shard_cnt, 4ull * S, cudaMemcpyDeviceToHost, glob.stream));
-  CK(cudaMemcpyAsync(ccnt.data(), glob.d_cw_cnt, 4ull * S, cudaMemcpyDeviceToHost, glob.stream));
-  CK(cudaStreamSynchronize(glob.stream));
-  work.resize(S);
-  for (uint32_t s = 0; s < S; ++s) work[s] = (uint64_t)cnt[s] + ccnt[s];
-  return CUSHA_OK;
-}
-
-namespace {
-__global__ void k_rebase(const uint32_t* __restrict__ in, uint64_t n, uint32_t sub, uint32_t* out) {
-  GRID_STRIDE(i, n) out[i] = in[i] - sub;
-}
-// partition owning global padded shard position m: pb[q] <= m < pb[q+1]
-__device__ __forceinline__ uint32_t part_of_pos(const uint32_t* pb, uint32_t G, uint32_t m) {
-  uint32_t lo = 0, hi = G;
-  while (hi - lo > 1) {
-    const uint32_t mid = (lo + hi) >> 1;
-    if (pb[mid] <= m) lo = mid;
-    else hi = mid;
-  }
-  return lo;
-}
-// Mapper of the partition's CW_i: the target position local to the partition
-// that owns it (filler entries: 0xFFFFFFFF; no kernel reads them)
-__global__ void k_mapper_local(const uint32_t* __restrict__ m, uint64_t n, const uint32_t* __restrict__ pb, uint32_t G,
-                               uint32_t trash, uint32_t* out) {
-  GRID_STRIDE(k, n) {
-    const uint32_t t = m[k];
-    out[k] = t == trash ? 0xFFFFFFFFu : t - pb[part_of_pos(pb, G, t)];
-  }
-}
-// window-form Mapper of the partition: Mapper_loc[k_loc] = delta_loc[il][j] + k_loc with
-// k_loc = k - c0 and targets local to owner(j):  delta_loc = delta + c0 - pb[owner(j)]  (mod 2^32)
-__global__ void k_delta_local(const uint32_t* __restrict__ delta, uint32_t Sl, uint32_t S, uint32_t c0,
-                              const uint32_t* __restrict__ pb, const uint8_t* __restrict__ owner, uint32_t* out) {
-  GRID_STRIDE(t, (uint64_t)Sl * S) {
-    const uint32_t j = (uint32_t)(t % S);
-    out[t] = delta[t] + c0 - pb[owner[j]];
-  }
-}
-// cwp[il][q] = first CW_i position (local) whose target lies in partition q:
-// CW_i lists W_i0, W_i1, ... in shard order (L175), so that is the start of
-// CW_i plus the sizes of W_ij for j < bounds[q]; cwp[il][G] = end of CW_i.
-__global__ void k_cwp_local(const uint32_t* __restrict__ win_rows, const uint32_t* __restrict__ cw_off_loc,
-                            const uint32_t* __restrict__ cw_cnt, const uint32_t* __restrict__ bounds, uint32_t Sl,
-                            uint32_t S, uint32_t G, uint32_t* cwp) {
-  GRID_STRIDE(t, (uint64_t)Sl * (G + 1)) {
-    const uint32_t il = (uint32_t)(t / (G + 1)), q = (uint32_t)(t % (G + 1));
-    uint32_t acc = 0;
-    if (q == G) {
-      acc = cw_cnt[il];
-    } else {
-      const uint32_t* r0 = win_rows + (size_t)il * S;
-      const uint32_t* r1 = r0 + S;
-      for (uint32_t j = 0; j < bounds[q]; ++j) acc += r1[j] - r0[j];
-    }
-    cwp[t] = cw_off_loc[il] + acc;
-  }
-}
-template <class T>
-int dcopy(T** dst, const T* src, uint64_t n, cudaStream_t st, std::string& err) {
-  CK(dalloc(dst, n));
-  if (n) CK(cudaMemcpyAsync(*dst, src, n * sizeof(T), cudaMemcpyDeviceToDevice, st));
-  return CUSHA_OK;
-}
-}  // namespace
-
-int build_part(const Graph& glob, const std::vector<uint32_t>& bounds, uint32_t r, Graph& g, bool srcvalue_ipc,
-               std::string& err) {
-  (void)srcvalue_ipc;
-  cudaStream_t st = g.stream;
-  t_alloc_stream = st;
-  const uint32_t S = glob.S, N = glob.N, V = glob.V, G = (uint32_t)bounds.size() - 1;
-  const uint32_t s0 = bounds[r], s1 = bounds[r + 1], Sl = s1 - s0;
-  std::vector<uint32_t> so(S + 1), co(S + 1), cnt(S);
-  CK(cudaMemcpyAsync(so.data(), glob.d_shard_off, 4ull * (S + 1), cudaMemcpyDeviceToHost, st));
-  CK(cudaMemcpyAsync(co.data(), glob.d_cw_off, 4ull * (S + 1), cudaMemcpyDeviceToHost, st));
-  CK(cudaMemcpyAsync(cnt.data(), glob.d_shard_cnt, 4ull * S, cudaMemcpyDeviceToHost, st));
-  CK(cudaStreamSynchronize(st));
-  g.V = V; g.N = N; g.S = S; g.E = glob.E; g.repr = CUSHA_REPR_CW; g.has_ev = glob.has_ev;
-  g.keep_ids = glob.keep_ids; g.max_indeg = glob.max_indeg; g.max_abs_ev = glob.max_abs_ev;
-  g.G = G; g.part = r; g.h_bounds = bounds;
-  g.s0 = s0; g.Sl = Sl; g.v0 = s0 * N; g.nvl = std::min<uint64_t>(V, (uint64_t)s1 * N) - g.v0;
-  const uint32_t pos0 = so[s0], c0 = co[s0];
-  g.P = so[s1] - pos0;
-  g.Q = co[s1] - c0;
-  g.E_loc = 0;
-  for (uint32_t s = s0; s < s1; ++s) g.E_loc += cnt[s];
-  // host tables: bounds, owner, position bounds of the partitions
-  std::vector<uint8_t> owner(S);
-  std::vector<uint32_t> pb(G + 1);
-  for (uint32_t q = 0; q < G; ++q) {
-    pb[q] = so[bounds[q]];
-    for (uint32_t s = bounds[q]; s < bounds[q + 1]; ++s) owner[s] = (uint8_t)q;
-  }
-  pb[G] = so[S];
-  DevBuf dpb;
-  CK(dalloc((uint32_t**)&dpb.p, G + 1));
-  CK(dalloc(&g.d_bounds, G + 1));
-  CK(dalloc(&g.d_owner, S));
-  CK(cudaMemcpyAsync(dpb.p, pb.data(), 4ull * (G + 1), cudaMemcpyHostToDevice, st));
-  CK(cudaMemcpyAsync(g.d_bounds, bounds.data(), 4ull * (G + 1), cudaMemcpyHostToDevice, st));
-  CK(cudaMemcpyAsync(g.d_owner, owner.data(), S, cudaMemcpyHostToDevice, st));
-  // the partition's shards: in-edges of its vertices (positions rebased to 0)
-  CK(dalloc(&g.d_shard_off, (uint64_t)Sl + 1));
-  k_rebase<<<grid_for((uint64_t)Sl + 1), 256, 0, st>>>(glob.d_shard_off + s0, (uint64_t)Sl + 1, pos0, g.d_shard_off);
-  int rc;
-  if ((rc = dcopy(&g.d_shard_cnt, glob.d_shard_cnt + s0, Sl, st, err)) ||
-      (rc = dcopy(&g.d_dest, glob.d_dest + pos0, g.P, st, err)))
-    return rc;
-  if (glob.d_ev && (rc = dcopy(&g.d_ev, glob.d_ev + pos0, g.P, st, err))) return rc;
-  if (glob.d_eid && (rc = dcopy(&g.d_eid, glob.d_eid + pos0, g.P, st, err))) return rc;
-  // window-table rows of its source shards (emptiness tests; positions stay global)
-  if ((rc = dcopy(&g.d_win, glob.d_win + (size_t)s0 * S, ((uint64_t)Sl + 1) * S, st, err))) return rc;
-  // the Concatenated Windows of its source shards, every target partition
-  CK(dalloc(&g.d_cw_off, (uint64_t)Sl + 1));
-  k_rebase<<<grid_for((uint64_t)Sl + 1), 256, 0, st>>>(glob.d_cw_off + s0, (uint64_t)Sl + 1, c0, g.d_cw_off);
-  if ((rc = dcopy(&g.d_cw_cnt, glob.d_cw_cnt + s0, Sl, st, err)) ||
-      (rc = dcopy(&g.d_cw_src, glob.d_cw_src + c0, g.Q, st, err)) ||
-      (rc = dcopy(&g.d_cw_win, glob.d_cw_win + c0, g.Q, st, err)))
-    return rc;
-  CK(dalloc(&g.d_mapper, g.Q));
-  if (g.Q)
-    k_mapper_local<<<grid_for(g.Q), 256, 0, st>>>(glob.d_mapper + c0, g.Q, (const uint32_t*)dpb.p, G, (uint32_t)glob.P,
-                                                  g.d_mapper);
-  CK(dalloc(&g.d_cw_delta, (uint64_t)Sl * S));
-  k_delta_local<<<grid_for((uint64_t)Sl * S), 256, 0, st>>>(glob.d_cw_delta + (size_t)s0 * S, Sl, S, c0,
-                                                             (const uint32_t*)dpb.p, g.d_owner, g.d_cw_delta);
-  CK(dalloc(&g.d_cwp, (uint64_t)Sl * (G + 1)));
-  k_cwp_local<<<grid_for((uint64_t)Sl * (G + 1)), 256, 0, st>>>(g.d_win, g.d_cw_off, g.d_cw_cnt, g.d_bounds, Sl, S, G,
-                                                                  g.d_cwp);
-  if ((rc = dcopy(&g.d_outdeg, glob.d_outdeg + g.v0, g.nvl, st, err))) return rc;
-  CK(dalloc(&g.d_active, Sl));
-  if (g.skip_clean) CK(dalloc(&g.d_dirty, Sl));
-  CK(dalloc(&g.d_shard_seq, Sl));
-  CK(cudaGetLastError());
-  CK(cudaStreamSynchronize(st));
-  g.splitP = g.P;
-  g.splitQ = g.Q;
-  g.host_shard = Sl;
-  return CUSHA_OK;
 }
 
 void free_device_arrays(Graph& g) {

@@ -243,12 +243,33 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
 int build_runs(Graph& g, std::string& err);       // Mapper runs (CW, CUSHA_RLE builds)
 int offload_topology(Graph& g, std::string& err); // row f3: move shards >= host_shard to pinned host memory
 void partition_bounds(uint32_t S, const uint64_t* work, uint32_t G, uint32_t* bounds);
-int partition_work(const Graph& glob, std::vector<uint64_t>& work, std::string& err);
-// the partition r of a global layout (bounds: G+1 shard bounds); srcvalue_ipc:
-// SrcValue by cudaMalloc (exportable) instead of the stream-ordered pool
-int build_part(const Graph& glob, const std::vector<uint32_t>& bounds, uint32_t r, Graph& part, bool srcvalue_ipc,
-               std::string& err);
 void free_device_arrays(Graph& g);  // every device / pinned array of g (not its stream or events)
+
+// partition.cu: the per-partition layout built straight from the edge list
+struct PlanInput {
+  uint32_t V = 0, N = 0;
+  uint64_t E = 0;
+  const uint32_t *src = nullptr, *dst = nullptr, *val = nullptr;  // host or device
+  bool host = false;
+  cudaStream_t stream = nullptr;
+};
+struct Plan {  // from the shard-pair counts C[i][j] = |W_ij|
+  uint32_t V = 0, N = 0, S = 0;
+  uint64_t E = 0;
+  uint32_t* d_C = nullptr;        // S*S
+  uint32_t* d_win = nullptr;      // (S+1)*S: start of W_ij in shard j, local to j's partition
+  uint32_t* d_R = nullptr;        // S*S: start of W_ij inside CW_i
+  uint32_t* d_outdeg = nullptr;   // V
+  std::vector<uint32_t> in, out;  // entries per shard (its in-edges) / per CW_i (its vertices' out-edges)
+  std::vector<uint32_t> bounds;   // G+1
+  std::vector<uint8_t> owner;     // S
+  std::vector<uint32_t> offl, coffl;  // padded offset of shard j / CW_i inside its partition
+  uint32_t max_indeg = 0;
+  float max_abs_ev = 0.f;
+};
+int plan_partitions(const PlanInput& in, uint32_t G, Plan& plan, std::string& err);
+void free_plan(Plan& plan, cudaStream_t st);
+int build_part_direct(const PlanInput& in, const Plan& plan, uint32_t r, Graph& part, std::string& err);
 cudaError_t dev_alloc(void** p, size_t bytes, cudaStream_t s);  // the library's private stream-ordered pool
 cudaError_t trim_pool(int dev);                                  // release its unused blocks
 

@@ -69,15 +69,22 @@ def test_host_topology_zero_budget_is_all_hbm(rm):
         assert st["host_bytes"] == 0 and st["host_shard"] == st["num_shards"]
 
 
-def test_host_topology_is_for_one_partition(rm):
-    """Host-streamed topology (row f3) and the destination-range partition
-    (row e) are alternatives for a graph larger than one GPU's HBM; combined
-    they are refused (include/cusha.h)."""
+def test_host_topology_partitioned(rm):
+    """Row f3 with the destination-range partition: every partition keeps its
+    per-entry topology in pinned host memory (budget 1 byte per partition) and
+    only SrcValue / VertexValues in HBM; the stage-4 stores still reach the
+    sibling partitions.  Results stay bit-exact."""
     V, s, d, w = rm
-    with pytest.raises(cusha.CushaError) as e:
-        cusha.build_graph(V, s, d, edge_values=w, repr="cw", vertices_per_shard=500, world_size=4,
-                          device_topology_budget=1)
-    assert e.value.code == cusha.EUNSUPPORTED
+    with cusha.build_graph(V, s, d, edge_values=w, repr="cw", vertices_per_shard=500, world_size=4,
+                           device_topology_budget=1) as g:
+        st = cusha.get_stats(g)
+        assert st["partitions"] == 4 and st["host_bytes"] > 0
+        for q in range(4):
+            assert cusha.get_part_stats(g, q)["device_bytes"] < 16 * V
+        assert cusha.run("sssp", g) == cusha.OK
+        np.testing.assert_array_equal(cusha.get_values(g), oracle.sssp(V, s, d, w, 0))
+        assert cusha.run("bfs", g) == cusha.OK
+        np.testing.assert_array_equal(cusha.get_values(g), oracle.bfs(V, s, d, 0))
 
 
 def test_host_topology_mesh_many_passes():
