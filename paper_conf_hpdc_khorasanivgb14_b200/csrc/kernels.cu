@@ -228,16 +228,29 @@ __device__ __forceinline__ void fence_sc_gpu() { asm volatile("fence.sc.gpu;" ::
 // the producer's waits before ticket (s, pass) may read anything; false: the
 // run stopped meanwhile (the ticket is abandoned - every waiting ticket polls
 // stop, so an abandoned ticket never leaves another one waiting for it)
-__device__ __forceinline__ bool ticket_wait(const KParams& p, uint32_t s, uint32_t pass, uint32_t Sloc) {
+// known: every pass below it is known (to this producer) to have completed
+__device__ __forceinline__ bool ticket_wait(const KParams& p, uint32_t s, uint32_t pass, uint32_t Sloc, uint32_t& known) {
+  // both conditions' first reads in flight together (the common case: both hold)
+  const bool need_w = pass >= p.window && pass - p.window >= known;
+  const uint32_t seq0 = ld_vol(&p.shard_seq[s]);
+  const uint32_t done0 = need_w ? ld_vol(&p.trace[pass - p.window].done) : Sloc;
+  if (seq0 >= pass && done0 >= Sloc) {
+    if (need_w) known = pass - p.window + 1;
+    __threadfence();                                      // acquire the completed passes' stores ...
+    asm volatile("fence.proxy.async.global;" ::: "memory");  // ... for the TMA (async-proxy) reads too
+    return true;
+  }
   while (ld_vol(&p.shard_seq[s]) < pass) {
     if (ld_vol(&p.ctl->stop)) return false;
     __nanosleep(64);
   }
-  if (pass >= p.window)
+  if (pass >= p.window && pass - p.window >= known) {
     while (ld_vol(&p.trace[pass - p.window].done) < Sloc) {
       if (ld_vol(&p.ctl->stop)) return false;
       __nanosleep(64);
     }
+    known = pass - p.window + 1;  // pass r complete implies every earlier pass complete
+  }
   __threadfence();                                      // acquire the completed passes' stores ...
   asm volatile("fence.proxy.async.global;" ::: "memory");  // ... for the TMA (async-proxy) reads too
   return true;
@@ -475,24 +488,34 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
   };
   // tiles prefetched into L2 beyond the ring, when the pass streams from HBM (KParams::ahead)
   const uint32_t ahead = p.ahead ? CUSHA_AHEAD : 0u;
+  const uint32_t max_iters = p.ctl->max_iters;  // constant during the launch
+  uint32_t known_done = 0;                      // passes below it have completed (ticket_wait)
   for (uint32_t round = 0;; ++round) {
     uint32_t s;  // local shard index
+    uint32_t sb = 0, se = 0;  // the shard's entry range (read before the waits in overlapped mode)
+    uint32_t ca = 0, cb = 0;  // one partition: CW_s = [ca, cb) (read with them)
+    uint8_t act = 0;          // stage-4 predictor (a hint: a stale read costs bandwidth, not correctness)
     if (p.multi) {
       // overlapped passes: the next ticket, whatever pass it belongs to
-      bool over = ld_vol(&p.ctl->stop) != 0;
+      const unsigned long long t = atomicAdd(&p.ctl->ticket, 1ull);
+      cur_pass = (uint32_t)(t / Sloc);
+      s = (uint32_t)(t - (unsigned long long)cur_pass * Sloc);
+      bool over = cur_pass >= max_iters || ld_vol(&p.ctl->stop) != 0;
+      if (CUSHA_TIMELINE && !over) tl_mark((uint32_t)t, 0);
       if (!over) {
-        const unsigned long long t = atomicAdd(&p.ctl->ticket, 1ull);
-        cur_pass = (uint32_t)(t / Sloc);
-        s = (uint32_t)(t - (unsigned long long)cur_pass * Sloc);
-        over = cur_pass >= p.ctl->max_iters || ld_vol(&p.ctl->stop) != 0;
-        if (CUSHA_TIMELINE && !over) tl_mark((uint32_t)t, 0);
-      }
-      if (!over) {
-        // the shard's first stage-2 tiles start towards L2 while the producer
-        // waits (a prefetch reads nothing into the CTA, so it needs no ordering)
+        // the shard's scalars and first stage-2 tiles start towards the SM / L2
+        // while the producer waits (a prefetch reads nothing into the CTA, so it
+        // needs no ordering; the offsets are read-only)
+        sb = p.shard_off[s];
+        se = p.shard_off[s + 1];
+        act = p.active[s];
+        if (REPR == CUSHA_REPR_CW && p.G == 1) {
+          ca = p.cw_off[s];
+          cb = ca + p.cw_cnt[s];
+        }
         if (CUSHA_AHEAD_WAIT && ahead)
-          for (uint32_t j = 0; j <= ahead; ++j) pf2(p.shard_off[s] + j * kTile, p.shard_off[s + 1]);
-        over = !ticket_wait(p, s, cur_pass, Sloc);
+          for (uint32_t j = 0; j <= ahead; ++j) pf2(sb + j * kTile, se);
+        over = !ticket_wait(p, s, cur_pass, Sloc, known_done);
       }
       if (over) {
         push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
@@ -521,8 +544,17 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
       __threadfence();                                      // acquire the writers' SrcValue stores ...
       asm volatile("fence.proxy.async.global;" ::: "memory");  // ... for the TMA (async-proxy) reads below
     }
-    const bool spec = CUSHA_SPEC && REPR == CUSHA_REPR_CW && (CUSHA_SPEC_ALWAYS || p.active[s]);
-    const uint32_t b = p.shard_off[s], e = p.shard_off[s + 1];
+    if (!p.multi) {
+      sb = p.shard_off[s];
+      se = p.shard_off[s + 1];
+      act = p.active[s];
+      if (REPR == CUSHA_REPR_CW && p.G == 1) {
+        ca = p.cw_off[s];
+        cb = ca + p.cw_cnt[s];
+      }
+    }
+    const bool spec = CUSHA_SPEC && REPR == CUSHA_REPR_CW && (CUSHA_SPEC_ALWAYS || act);
+    const uint32_t b = sb, e = se;
     if (CUSHA_PF == 1) {
       // the consumers' global reads of this shard (stage 1/3 VertexValues and
       // NbrsNum, the stage-4 delta row) become L2 hits: one TMA prefetch each
@@ -535,8 +567,8 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     uint32_t qa = 0, qz = 0, a0 = 0, b0 = 0;
     if (REPR == CUSHA_REPR_CW) {
       for (uint32_t q = 0; q < p.G; ++q) {
-        uint32_t x, y;
-        segment(s, q, &x, &y);
+        uint32_t x = ca, y = cb;
+        if (p.G > 1) segment(s, q, &x, &y);
         if (x < y) {
           if (qz == 0) { qa = q; a0 = x; }
           qz = q + 1;
