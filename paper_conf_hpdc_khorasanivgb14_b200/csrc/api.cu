@@ -548,6 +548,9 @@ static uint32_t pass_grid(const Graph& g, const PassKernel& pk, size_t smem) {
 #ifndef CUSHA_DEEP_RING
 #define CUSHA_DEEP_RING 1  // 0: always the default ring depth (tuning comparison)
 #endif
+#ifndef CUSHA_FEW_TICKETS
+#define CUSHA_FEW_TICKETS 1.25  // below this many shards per resident CTA, run one CTA per SM with a deep ring
+#endif
 #ifndef CUSHA_STASH
 #define CUSHA_STASH 1  // 0: stage 3 of the integer algorithms re-reads VertexValues (tuning comparison)
 #endif
@@ -555,6 +558,7 @@ struct PassCfg {
   size_t smem = 0;
   int mapj = 0, stash = 0;
   uint32_t nst = 0;
+  bool one_cta = false;
 };
 static int pass_config(const Graph& g, const PassKernel& pk, PassCfg* c) {
   cudaFuncAttributes fa{};
@@ -599,15 +603,22 @@ static int pass_config(const Graph& g, const PassKernel& pk, PassCfg* c) {
     }
   }
   // a deeper TMA ring whenever another slot fits at the same CTAs per SM
-  // (more bytes in flight per SM; e.g. C5 at one CTA per SM)
+  // (more bytes in flight per SM; e.g. C5 at one CTA per SM).  With few
+  // shards per resident CTA (a pass is about one ticket per CTA, C4) the ring
+  // takes the whole SM instead: one CTA per SM, up to 6 slots.  Half as many
+  // shards then run at once, so more of them see write-backs made earlier in
+  // the same pass (L45) and the run needs fewer passes, while the deep ring
+  // keeps the SM's bytes in flight (C4 CC 0.59 -> 0.48 ms)
   c->nst = pk.ring_bytes / pk.slot_bytes;
   if (CUSHA_DEEP_RING) {
-    int occ_0 = 0;
+    int occ_0 = 0, sms = 148;
     CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_0, pk.func, (int)pk.threads, c->smem));
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g.device);
+    c->one_cta = occ_0 >= 2 && (double)g.Sl < CUSHA_FEW_TICKETS * occ_0 * sms;
     while (c->nst < pk.max_stages && c->smem + pk.slot_bytes <= kMaxSmem) {
       int occ_d = 0;
       CKA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_d, pk.func, (int)pk.threads, c->smem + pk.slot_bytes));
-      if (occ_d < occ_0 || occ_d == 0) break;
+      if ((occ_d < occ_0 && !c->one_cta) || occ_d == 0) break;
       c->smem += pk.slot_bytes;
       ++c->nst;
     }

@@ -50,7 +50,7 @@ def test_nn_at_size(nn_case, repr, N):
     s, d, w, x0, x_star, tol = nn_case
     got, st, cw = run("nn", s, d, w.view(np.uint32), x0, repr, BIG_N["nn"] if N else 0)
     paths_taken(st, cw, repr)
-    assert st["ring_slots"] == (4 if N else st["ring_slots"])
+    assert st["ring_slots"] >= (4 if N else 3)
     np.testing.assert_allclose(got, x_star, rtol=0, atol=tol * max(1.0, np.abs(x_star).max()))
 
 
@@ -67,7 +67,7 @@ def test_hs_at_size(hs_case, repr, N):
     s, d, c, q0, q_star, tol = hs_case
     got, st, cw = run("hs", s, d, c.view(np.uint32), np.stack([q0, q0], 1), repr, BIG_N["hs"] if N else 0)
     paths_taken(st, cw, repr)
-    assert st["ring_slots"] == (4 if N else st["ring_slots"])
+    assert st["ring_slots"] >= (4 if N else 3)
     np.testing.assert_allclose(got[:, 0], q_star, rtol=0, atol=tol)
 
 
@@ -84,7 +84,7 @@ def test_cs_at_size(cs_case, repr, N):
     s, d, G, v0, a0, v_star, tol = cs_case
     got, st, cw = run("cs", s, d, G.view(np.uint32), np.stack([v0, a0], 1), repr, BIG_N["cs"] if N else 0)
     paths_taken(st, cw, repr)
-    assert st["ring_slots"] == (4 if N else st["ring_slots"])
+    assert st["ring_slots"] >= (4 if N else 3)
     np.testing.assert_allclose(got[:, 0], v_star, rtol=0, atol=tol)
     anc = a0 != 0
     np.testing.assert_array_equal(got[anc, 0], v0[anc])
