@@ -14,6 +14,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "algorithms.cuh"
 #include "graph.hpp"
 
@@ -37,6 +39,13 @@ static int fail(int code, const std::string& msg) {
   } while (0)
 
 constexpr int kModeSingle = 0, kModeSim = 1, kModeNccl = 2;
+
+// NVTX ranges around the ABI calls (SURVEY §5 tracing): header-only NVTX v3,
+// free unless a tool (nsys, ncu --nvtx) is attached
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
 constexpr int kChunk = 16;  // passes per fixed-count graph / per host check (per-pass modes)
 #ifndef CUSHA_WIDE_WINDOW
 #define CUSHA_WIDE_WINDOW 4
@@ -234,6 +243,7 @@ uint32_t cusha_shard_size(uint32_t V, uint64_t E, uint32_t vertex_bytes, uint32_
 int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_t* dst, const uint32_t* edge_values,
                       const cusha_build_opts* opts, cusha_graph** out) {
   if (!out) return fail(CUSHA_EINVAL, "out is NULL");
+  NvtxRange nvtx("cusha_build_graph");
   *out = nullptr;
   if (V == 0) return fail(CUSHA_EINVAL, "num_vertices must be > 0");
   if (V >= (1u << 31)) return fail(CUSHA_EINVAL, "num_vertices must be < 2^31");
@@ -753,6 +763,7 @@ extern "C" {
 int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max_iters) {
   if (!h) return fail(CUSHA_EINVAL, "graph is NULL");
   if ((int)alg < 0 || (int)alg >= kNumAlgs) return fail(CUSHA_EINVAL, "bad algorithm");
+  NvtxRange nvtx("cusha_run");
   Graph& g = g0(h);
   const int a = (int)alg;
   const uint32_t V = h->st.num_vertices;
@@ -964,6 +975,7 @@ int cusha_get_values(const cusha_graph* h, void* out, size_t out_bytes) {
   if (!h->have_values) return fail(CUSHA_ESTATE, "no run yet");
   const size_t want = (size_t)h->st.num_vertices * value_bytes(h->last_alg);
   if (out_bytes != want) return fail(CUSHA_EINVAL, "out_bytes must be |V| * value_bytes(last algorithm)");
+  NvtxRange nvtx("cusha_get_values");
   CKA(cudaSetDevice(h->device));
   return copy_values(h, out, true);
 }

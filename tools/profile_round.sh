@@ -2,7 +2,7 @@
 # Evidence for profiles/<tag>/: ncu launch list of the default bench command,
 # ncu --set full of its shard_pass launch (one launch per run: overlapped
 # passes) and of one per-pass launch (host-loop mode), and bench lines.
-TAG=${1:-r2}
+TAG=${1:-r2final}
 O=gpurun_out/$TAG; mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" > $O/build.log 2>&1
 # every launch of one bench step (default mode), device time and DRAM bytes
