@@ -64,6 +64,8 @@ struct cusha_graph {
   bool own_stream = false;
   int device = 0;
   cudaGraphExec_t exec[cusha::kNumAlgs] = {};  // per-pass mode: kChunk passes per graph (single partition)
+  cudaGraphExec_t chunk_exec[cusha::kNumAlgs] = {};  // partitioned / BSP: one captured chunk of rounds
+  bool chunk_uncapturable[cusha::kNumAlgs] = {};
   cusha::Ctl** d_ctls = nullptr;                // partitioned: device array of the partitions' Ctl (sim) / own (NCCL)
   cusha_stats st{};
   int last_alg = -1;
@@ -94,6 +96,8 @@ static void free_handle(cusha_graph* h) {
   if (!h) return;
   cudaSetDevice(h->device);
   for (auto& e : h->exec)
+    if (e) cudaGraphExecDestroy(e);
+  for (auto& e : h->chunk_exec)
     if (e) cudaGraphExecDestroy(e);
   for (Graph* g : h->parts) {
     free_device_arrays(*g);
@@ -787,6 +791,8 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     p->trace_dirty = 0;
     for (auto& e : h->exec)  // kernel params captured the old trace pointer
       if (e) { cudaGraphExecDestroy(e); e = nullptr; }
+    for (auto& e : h->chunk_exec)
+      if (e) { cudaGraphExecDestroy(e); e = nullptr; }
   }
   const PassKernel& pk = pass_kernel(a, g.repr);
   PassCfg cfg;
@@ -846,30 +852,61 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
       kps.push_back(pass_params(*p, source, cfg, a));
       grids.push_back(pass_grid(*p, pk, cfg.smem));
     }
-    uint32_t* cur = g.d_srcvalue;  // BSP: the copy this pass reads (init wrote d_srcvalue)
-    uint32_t* nxt = g.d_srcvalue2;
+    // one chunk = kChunk rounds of (every partition's pass [+ BSP copy], the
+    // convergence decision); 16 passes per host check.  BSP alternates the two
+    // SrcValue copies, an even number of times per chunk, so every chunk starts
+    // from d_srcvalue.
+    auto enqueue_chunk = [&](std::string& e2) -> int {
+      uint32_t* cur = g.d_srcvalue;  // BSP: the copy this pass reads (init wrote d_srcvalue)
+      uint32_t* nxt = g.d_srcvalue2;
+      for (int k = 0; k < kChunk; ++k) {
+        if (g.bsp) {
+          // two-phase BSP: stage 4 writes the copy the NEXT pass reads, which
+          // starts as this pass's input (entries no shard writes carry over)
+          CKA(cudaMemcpyAsync(nxt, cur, 4 * (g.P + 1), cudaMemcpyDeviceToDevice, st));
+          kps[0].srcvalue = cur;
+          kps[0].sv_write = nxt;
+          std::swap(cur, nxt);
+        }
+        for (size_t r = 0; r < h->parts.size(); ++r) {
+          void* args[] = {&kps[r]};
+          CKA(cudaLaunchKernel(pk.func, dim3(grids[r]), dim3(pk.threads), args, cfg.smem, st));
+        }
+        if (h->mode == kModeSim) {
+          CKA(launch_close_parts(h->d_ctls, (uint32_t)h->parts.size(), st));
+        } else if (h->mode == kModeNccl) {
+          const int r2 = nccl_allreduce_max_u32(g, &g.d_ctl->lchanged, &g.d_ctl->gchanged, e2);
+          if (r2) return fail(r2, "convergence all-reduce: " + e2);
+          CKA(launch_close_parts(h->d_ctls, 0, st));
+        }
+      }
+      return CUSHA_OK;
+    };
+    // partitioned / BSP chunks are captured once into a CUDA graph and replayed
+    // (one launch per 16 rounds instead of (partitions + 2) x 16 API calls);
+    // explicit host_loop (profilers) keeps the individual launches
+    const bool capture = host_loop && !g.host_loop && !h->chunk_uncapturable[a];
+    if (capture && !h->chunk_exec[a]) {
+      cudaGraph_t cg = nullptr;
+      bool ok = cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
+      std::string e2;
+      const int crc = ok ? enqueue_chunk(e2) : CUSHA_OK;
+      const cudaError_t ee = ok ? cudaStreamEndCapture(st, &cg) : cudaErrorUnknown;
+      ok = ok && crc == CUSHA_OK && ee == cudaSuccess && cg;
+      if (ok) ok = cudaGraphInstantiate(&h->chunk_exec[a], cg, 0) == cudaSuccess;
+      if (cg) cudaGraphDestroy(cg);
+      if (!ok) {  // run uncaptured (e.g. a library NCCL without stream-capture support)
+        cudaGetLastError();
+        h->chunk_exec[a] = nullptr;
+        h->chunk_uncapturable[a] = true;
+      }
+    }
     for (;;) {
       if (host_loop) {
-        for (int k = 0; k < kChunk; ++k) {
-          if (g.bsp) {
-            // two-phase BSP: stage 4 writes the copy the NEXT pass reads, which
-            // starts as this pass's input (entries no shard writes carry over)
-            CKA(cudaMemcpyAsync(nxt, cur, 4 * (g.P + 1), cudaMemcpyDeviceToDevice, st));
-            kps[0].srcvalue = cur;
-            kps[0].sv_write = nxt;
-            std::swap(cur, nxt);
-          }
-          for (size_t r = 0; r < h->parts.size(); ++r) {
-            void* args[] = {&kps[r]};
-            CKA(cudaLaunchKernel(pk.func, dim3(grids[r]), dim3(pk.threads), args, cfg.smem, st));
-          }
-          if (h->mode == kModeSim) {
-            CKA(launch_close_parts(h->d_ctls, (uint32_t)h->parts.size(), st));
-          } else if (h->mode == kModeNccl) {
-            if ((rc = nccl_allreduce_max_u32(g, &g.d_ctl->lchanged, &g.d_ctl->gchanged, err)))
-              return fail(rc, "convergence all-reduce: " + err);
-            CKA(launch_close_parts(h->d_ctls, 0, st));
-          }
+        if (h->chunk_exec[a]) {
+          CKA(cudaGraphLaunch(h->chunk_exec[a], st));
+        } else if ((rc = enqueue_chunk(err))) {
+          return rc;
         }
       } else {
         CKA(cudaGraphLaunch(h->exec[a], st));
