@@ -653,12 +653,36 @@ static int pass_ahead(const Graph& g, int alg) {
   return bytes > 2ull * (uint64_t)l2 ? 1 : 0;
 }
 
+// Ticket order.  A pass that stays in L2 (no read-ahead) is bound by its
+// slowest shards' latency, so it takes the largest shards first; a pass that
+// streams from HBM keeps shard order (neighbouring shards share SrcValue lines
+// in L2: largest-first was slower on C2, DESIGN.md tuning log v4).
+#ifndef CUSHA_BIG_FIRST
+#define CUSHA_BIG_FIRST 1
+#endif
+static int shard_order(Graph& g) {
+  if (g.d_order || !g.Sl) return CUSHA_OK;
+  std::vector<uint32_t> cnt(g.Sl), ccnt(g.Sl), ord(g.Sl);
+  CKA(cudaMemcpyAsync(cnt.data(), g.d_shard_cnt, 4ull * g.Sl, cudaMemcpyDeviceToHost, g.stream));
+  CKA(cudaMemcpyAsync(ccnt.data(), g.d_cw_cnt, 4ull * g.Sl, cudaMemcpyDeviceToHost, g.stream));
+  CKA(cudaStreamSynchronize(g.stream));
+  for (uint32_t s = 0; s < g.Sl; ++s) ord[s] = s;
+  std::stable_sort(ord.begin(), ord.end(), [&](uint32_t a, uint32_t b) {
+    return (uint64_t)cnt[a] + ccnt[a] > (uint64_t)cnt[b] + ccnt[b];
+  });
+  CKA(dev_alloc((void**)&g.d_order, 4ull * g.Sl, g.stream));
+  CKA(cudaMemcpyAsync(g.d_order, ord.data(), 4ull * g.Sl, cudaMemcpyHostToDevice, g.stream));
+  CKA(cudaStreamSynchronize(g.stream));
+  return CUSHA_OK;
+}
+
 static KParams pass_params(const Graph& g, uint32_t source, const PassCfg& c, int alg) {
   KParams kp = make_params(g, source);
   kp.mapj = c.mapj;
   kp.stash = c.stash;
   kp.nst = c.nst;
   kp.ahead = pass_ahead(g, alg);
+  if (CUSHA_BIG_FIRST && !kp.ahead) kp.order = g.d_order;
   return kp;
 }
 
@@ -797,6 +821,9 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   const PassKernel& pk = pass_kernel(a, g.repr);
   PassCfg cfg;
   if ((rc = pass_config(g, pk, &cfg))) return rc;
+  if (CUSHA_BIG_FIRST)
+    for (Graph* p : h->parts)
+      if (!pass_ahead(*p, a) && (rc = shard_order(*p))) return rc;
   const bool parted = h->mode != kModeSingle;
   const bool host_loop = g.host_loop || parted || g.bsp;
   // one launch for the whole run (overlapped passes) unless asked otherwise;

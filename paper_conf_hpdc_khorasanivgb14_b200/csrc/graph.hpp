@@ -76,6 +76,7 @@ struct KParams {
   int ahead;                   // 1: the producer prefetches stage-2 tiles into L2 beyond the ring (HBM-resident passes)
   uint32_t nst;                // ring slots of this run (kStages, or more when shared memory has room)
   uint32_t* shard_seq;         // Sl: passes of shard s completed (overlapped passes)
+  const uint32_t* order;       // Sl: shard processed by the q-th ticket of a pass (nullptr: shard order)
   // destination-range partition (row e); G = 1: single partition
   uint32_t G;                  // partitions
   const uint32_t* bounds;      // G+1 shard bounds of the partitions
@@ -153,6 +154,7 @@ struct Graph {
   uint8_t* d_active = nullptr;      // Sl: stage-4 prefetch predictor
   uint32_t* d_dirty = nullptr;      // Sl: clean-shard skipping flags
   uint32_t* d_shard_seq = nullptr;  // Sl: overlapped passes, per-shard pass order
+  uint32_t* d_order = nullptr;      // Sl: largest shards first (L2-resident passes; built on first use)
   int pass_barrier = 0;             // 0: automatic, 1: one launch per pass, 2: overlapped
   bool skip_clean = false;
   // host-streamed topology (row f3): shards >= host_shard keep their entry

@@ -500,6 +500,7 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
       const unsigned long long t = atomicAdd(&p.ctl->ticket, 1ull);
       cur_pass = (uint32_t)(t / Sloc);
       s = (uint32_t)(t - (unsigned long long)cur_pass * Sloc);
+      if (p.order && cur_pass < max_iters) s = p.order[s];
       bool over = cur_pass >= max_iters || ld_vol(&p.ctl->stop) != 0;
       if (CUSHA_TIMELINE && !over) tl_mark((uint32_t)t, 0);
       if (!over) {
@@ -525,6 +526,7 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     } else {
       // persistent grid: shards from the global queue; otherwise CTA b runs shard b only
       s = kPersistent ? atomicAdd(&p.ctl->next_shard, 1u) : (round == 0 ? blockIdx.x : Sloc);
+      if (p.order && s < Sloc) s = p.order[s];
       if (s >= Sloc) {
         push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
         return;
@@ -1233,6 +1235,7 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.splitP = (uint32_t)g.splitP; p.splitQ = (uint32_t)g.splitQ;
   p.dest_h = g.h_dest; p.ev_h = g.h_ev; p.srcloc_h = g.h_srcloc; p.cw_src_h = g.h_cw_src; p.mapper_h = g.h_mapper;
   p.multi = 0; p.shard_seq = g.d_shard_seq;
+  p.order = nullptr;
   p.window = 2;
   p.mapj = 0;
   p.stash = 0;
