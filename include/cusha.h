@@ -51,7 +51,7 @@ extern "C" {
 #define CUSHA_API
 #endif
 
-#define CUSHA_ABI_VERSION 4
+#define CUSHA_ABI_VERSION 5
 
 /* Return codes. */
 enum {
@@ -180,7 +180,21 @@ typedef struct {
    * before it aborts the communicator and returns CUSHA_ENCCL (an NCCL
    * asynchronous error does the same at once).  0 = 300000.                 */
   uint32_t comm_timeout_ms;
+  /* One process per GPU: how the ranks find each other's arrays.
+   * CUSHA_TRANSPORT_NCCL (0): with nccl_unique_id, cusha_build_graph
+   *   all-gathers the ranks' CUDA IPC handles over NCCL.
+   * CUSHA_TRANSPORT_IPC (1): no NCCL at all; after cusha_build_graph every
+   *   rank passes cusha_ipc_export's blob to the others (e.g. an all-gather
+   *   over torch.distributed) and calls cusha_ipc_connect with all of them.
+   * In both, everything after the bootstrap is peer memory: stage-4 stores
+   * into the owning rank's SrcValue, a per-pass barrier and convergence vote
+   * through the ranks' barrier blocks, and cusha_get_values reading every
+   * rank's slice.  Ranks may share one device (then the stores stay in HBM).  */
+  int transport;
 } cusha_build_opts;
+
+enum { CUSHA_TRANSPORT_NCCL = 0, CUSHA_TRANSPORT_IPC = 1 };
+#define CUSHA_IPC_BLOB_BYTES 256  /* cusha_ipc_export: four 64-byte cudaIpcMemHandle_t */
 
 enum { CUSHA_MODE_ASYNC = 0, CUSHA_MODE_BSP = 1 };
 
@@ -380,6 +394,18 @@ CUSHA_API const char* cusha_last_error(void);
 
 /* CUSHA_ABI_VERSION of the loaded library. */
 CUSHA_API int cusha_abi_version(void);
+
+/* One process per GPU (world_size > 1 with a rank): this rank's CUDA IPC
+ * handles (CUSHA_IPC_BLOB_BYTES, host buffer).  Errors: CUSHA_ESTATE (not a
+ * one-process-per-GPU graph), CUSHA_EINVAL, CUSHA_ECUDA.                    */
+CUSHA_API int cusha_ipc_export(cusha_graph* g, void* out, size_t bytes);
+
+/* Transport IPC: map every other rank's arrays; `all` holds world_size blobs
+ * from cusha_ipc_export in rank order (bytes = world_size *
+ * CUSHA_IPC_BLOB_BYTES).  Required once before the first cusha_run.
+ * cusha_run and cusha_get_values are collective: every rank calls them in the
+ * same order.  Errors: CUSHA_ESTATE, CUSHA_EINVAL, CUSHA_ECUDA.             */
+CUSHA_API int cusha_ipc_connect(cusha_graph* g, const void* all, size_t bytes);
 
 /* Multi-GPU helper: write a fresh 128-byte ncclUniqueId to out128 (rank 0
  * calls this and broadcasts it, e.g. over torch.distributed).  NCCL

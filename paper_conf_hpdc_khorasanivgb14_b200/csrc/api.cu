@@ -38,7 +38,10 @@ static int fail(int code, const std::string& msg) {
     }                                                                                              \
   } while (0)
 
-constexpr int kModeSingle = 0, kModeSim = 1, kModeNccl = 2;
+// one partition; G partitions in this process; one process per GPU
+// bootstrapped over NCCL; one process per GPU bootstrapped by the caller
+constexpr int kModeSingle = 0, kModeSim = 1, kModeNccl = 2, kModeIpc = 3;
+constexpr size_t kIpcBlob = 4 * sizeof(cudaIpcMemHandle_t);  // SrcValue, dirty, barrier block, VertexValues
 
 // NVTX ranges around the ABI calls (SURVEY §5 tracing): header-only NVTX v3,
 // free unless a tool (nsys, ncu --nvtx) is attached
@@ -125,22 +128,25 @@ static const Graph& g0(const cusha_graph* h) { return *h->parts[0]; }
 // other ranks can map them (CUDA IPC) and store into them over NVLink.
 static int alloc_run_state(Graph& g, bool ipc) {
   g.srcvalue_ipc = ipc;
-  if (ipc) {
+  if (ipc) {  // the arrays the other ranks map: SrcValue, dirty[], the barrier block, VertexValues
     CKA(cudaMalloc(&g.d_srcvalue, 4 * (g.P + 1)));
     if (g.skip_clean) {
       if (g.d_dirty) cudaFreeAsync(g.d_dirty, g.stream);
       g.d_dirty = nullptr;
       CKA(cudaMalloc(&g.d_dirty, 4ull * std::max<uint32_t>(g.Sl, 1)));
     }
+    CKA(cudaMalloc(&g.d_sync, sizeof(PeerSync)));
+    CKA(cudaMemsetAsync(g.d_sync, 0, sizeof(PeerSync), g.stream));
+    CKA(cudaMalloc(&g.d_vv, 8ull * std::max<uint32_t>(g.nvl, 1)));
   } else {
     CKA(dev_alloc((void**)&g.d_srcvalue, 4 * (g.P + 1), g.stream));
+    CKA(dev_alloc(&g.d_vv, 8ull * std::max<uint32_t>(g.nvl, 1), g.stream));
   }
   CKA(cudaMemsetAsync(g.d_srcvalue, 0, 4 * (g.P + 1), g.stream));
   if (g.bsp) {
     CKA(dev_alloc((void**)&g.d_srcvalue2, 4 * (g.P + 1), g.stream));
     CKA(cudaMemsetAsync(g.d_srcvalue2, 0, 4 * (g.P + 1), g.stream));
   }
-  CKA(dev_alloc(&g.d_vv, 8ull * std::max<uint32_t>(g.nvl, 1), g.stream));
   CKA(dev_alloc((void**)&g.d_ctl, sizeof(Ctl), g.stream));
   CKA(cudaMemsetAsync(g.d_ctl, 0, sizeof(Ctl), g.stream));
   g.h_ctl = new (std::nothrow) Ctl();
@@ -161,46 +167,77 @@ static int set_peer_tables(Graph& g, const std::vector<uint32_t*>& sv, const std
   return CUSHA_OK;
 }
 
-// One process per GPU: exchange the CUDA IPC handles of every rank's SrcValue
-// and dirty[] over NCCL (all-gather of 64-byte handles) and map the peers'.
-static int connect_ipc_peers(Graph& g) {
+// One process per GPU: this rank's CUDA IPC handles (SrcValue, dirty[], the
+// barrier block, VertexValues), and the mapping of every other rank's.
+static int ipc_export_blob(Graph& g, void* out) {
+  cudaIpcMemHandle_t h[4];
+  std::memset(h, 0, sizeof(h));
+  CKA(cudaIpcGetMemHandle(&h[0], g.d_srcvalue));
+  if (g.skip_clean) CKA(cudaIpcGetMemHandle(&h[1], g.d_dirty));
+  CKA(cudaIpcGetMemHandle(&h[2], g.d_sync));
+  CKA(cudaIpcGetMemHandle(&h[3], g.d_vv));
+  std::memcpy(out, h, sizeof(h));
+  return CUSHA_OK;
+}
+
+static int ipc_connect_blob(Graph& g, const void* all) {
   const uint32_t G = g.G;
-  cudaIpcMemHandle_t mine[2];
-  std::memset(mine, 0, sizeof(mine));
-  CKA(cudaIpcGetMemHandle(&mine[0], g.d_srcvalue));
-  if (g.skip_clean) CKA(cudaIpcGetMemHandle(&mine[1], g.d_dirty));
-  void* dsend = nullptr;
-  void* drecv = nullptr;
-  CKA(dev_alloc(&dsend, sizeof(mine), g.stream));
-  CKA(dev_alloc(&drecv, sizeof(mine) * G, g.stream));
-  CKA(cudaMemcpyAsync(dsend, mine, sizeof(mine), cudaMemcpyHostToDevice, g.stream));
-  std::string err;
-  int rc = nccl_allgather_bytes(g, dsend, drecv, sizeof(mine), err);
-  if (!rc) rc = nccl_wait(g, g.comm_timeout_ms, err);
-  if (rc) return fail(rc, "IPC handle exchange: " + err);
-  std::vector<cudaIpcMemHandle_t> all(2 * G);
-  CKA(cudaMemcpyAsync(all.data(), drecv, sizeof(mine) * G, cudaMemcpyDeviceToHost, g.stream));
-  CKA(cudaStreamSynchronize(g.stream));
-  cudaFreeAsync(dsend, g.stream);
-  cudaFreeAsync(drecv, g.stream);
+  std::vector<cudaIpcMemHandle_t> h(4 * G);
+  std::memcpy(h.data(), all, kIpcBlob * G);
   std::vector<uint32_t*> sv(G), dirty(G, nullptr);
+  std::vector<PeerSync*> sync(G);
+  g.vv_peer.assign(G, nullptr);
+  auto open = [&](const cudaIpcMemHandle_t& hd, void** p) -> int {
+    CKA(cudaIpcOpenMemHandle(p, hd, cudaIpcMemLazyEnablePeerAccess));
+    g.ipc_open.push_back(*p);
+    return CUSHA_OK;
+  };
+  int rc;
   for (uint32_t q = 0; q < G; ++q) {
     if (q == g.part) {
-      sv[q] = g.d_srcvalue;
-      dirty[q] = g.d_dirty;
+      sv[q] = g.d_srcvalue; dirty[q] = g.d_dirty; sync[q] = g.d_sync; g.vv_peer[q] = g.d_vv;
       continue;
     }
     void* p = nullptr;
-    CKA(cudaIpcOpenMemHandle(&p, all[2 * q], cudaIpcMemLazyEnablePeerAccess));
-    g.ipc_open.push_back(p);
+    if ((rc = open(h[4 * q], &p))) return rc;
     sv[q] = static_cast<uint32_t*>(p);
     if (g.skip_clean) {
-      CKA(cudaIpcOpenMemHandle(&p, all[2 * q + 1], cudaIpcMemLazyEnablePeerAccess));
-      g.ipc_open.push_back(p);
+      if ((rc = open(h[4 * q + 1], &p))) return rc;
       dirty[q] = static_cast<uint32_t*>(p);
     }
+    if ((rc = open(h[4 * q + 2], &p))) return rc;
+    sync[q] = static_cast<PeerSync*>(p);
+    if ((rc = open(h[4 * q + 3], &p))) return rc;
+    g.vv_peer[q] = p;
   }
-  return set_peer_tables(g, sv, dirty);
+  if ((rc = set_peer_tables(g, sv, dirty))) return rc;
+  CKA(dev_alloc((void**)&g.d_sync_peer, sizeof(PeerSync*) * G, g.stream));
+  CKA(cudaMemcpyAsync(g.d_sync_peer, sync.data(), sizeof(PeerSync*) * G, cudaMemcpyHostToDevice, g.stream));
+  CKA(cudaStreamSynchronize(g.stream));
+  g.connected = true;
+  return CUSHA_OK;
+}
+
+// NCCL bootstrap: all-gather every rank's handles, then map them
+static int connect_ipc_peers(Graph& g) {
+  const uint32_t G = g.G;
+  std::vector<uint8_t> mine(kIpcBlob), all(kIpcBlob * G);
+  int rc = ipc_export_blob(g, mine.data());
+  if (rc) return rc;
+  void* dsend = nullptr;
+  void* drecv = nullptr;
+  CKA(dev_alloc(&dsend, kIpcBlob, g.stream));
+  CKA(dev_alloc(&drecv, kIpcBlob * G, g.stream));
+  CKA(cudaMemcpyAsync(dsend, mine.data(), kIpcBlob, cudaMemcpyHostToDevice, g.stream));
+  std::string err;
+  rc = nccl_allgather_bytes(g, dsend, drecv, kIpcBlob, err);
+  if (!rc) rc = nccl_wait(g, g.comm_timeout_ms, err);
+  if (rc) return fail(rc, "IPC handle exchange: " + err);
+  CKA(cudaMemcpyAsync(all.data(), drecv, kIpcBlob * G, cudaMemcpyDeviceToHost, g.stream));
+  CKA(cudaStreamSynchronize(g.stream));
+  cudaFreeAsync(dsend, g.stream);
+  cudaFreeAsync(drecv, g.stream);
+  return ipc_connect_blob(g, all.data());
 }
 
 }  // namespace cusha
@@ -260,8 +297,10 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   if (o.world_size > 64) return fail(CUSHA_EINVAL, "world_size must be <= 64");
   if (o.world_size > 1 && o.repr != CUSHA_REPR_CW)
     return fail(CUSHA_EUNSUPPORTED, "the partitioned (multi-GPU) mode uses the CW representation");
-  if (o.world_size > 1 && o.nccl_unique_id && (o.rank < 0 || o.rank >= o.world_size))
-    return fail(CUSHA_EINVAL, "rank out of range");
+  if (o.transport != CUSHA_TRANSPORT_NCCL && o.transport != CUSHA_TRANSPORT_IPC)
+    return fail(CUSHA_EINVAL, "transport must be NCCL or IPC");
+  const bool multiproc = o.world_size > 1 && (o.nccl_unique_id || o.transport == CUSHA_TRANSPORT_IPC);
+  if (multiproc && (o.rank < 0 || o.rank >= o.world_size)) return fail(CUSHA_EINVAL, "rank out of range");
   uint32_t N = o.vertices_per_shard ? o.vertices_per_shard : cusha_shard_size(V, E, o.smem_bytes_per_vertex, 0, 0);
   if (N > 65534) return fail(CUSHA_EINVAL, "vertices_per_shard must be <= 65534");
   if (o.pass_barrier < 0 || o.pass_barrier > 2) return fail(CUSHA_EINVAL, "pass_barrier must be 0, 1 or 2");
@@ -270,9 +309,11 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
     return fail(CUSHA_EUNSUPPORTED, "the two-phase BSP mode runs one partition");
   if (N > V) N = V;
   const uint32_t S = (V + N - 1) / N;
-  const int mode = o.world_size == 1 ? kModeSingle : (o.nccl_unique_id ? kModeNccl : kModeSim);
+  const int mode = o.world_size == 1 ? kModeSingle
+                   : o.transport == CUSHA_TRANSPORT_IPC ? kModeIpc
+                   : (o.nccl_unique_id ? kModeNccl : kModeSim);
   const uint32_t G = std::min<uint32_t>((uint32_t)o.world_size, S);  // never more partitions than shards
-  if (mode == kModeNccl && G != (uint32_t)o.world_size) return fail(CUSHA_EINVAL, "world_size exceeds the number of shards");
+  if (multiproc && G != (uint32_t)o.world_size) return fail(CUSHA_EINVAL, "world_size exceeds the number of shards");
 
   cusha_graph* h = new (std::nothrow) cusha_graph();
   if (!h) return fail(CUSHA_ENOMEM, "host allocation");
@@ -304,7 +345,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   g.keep_ids = o.keep_layout != 0;
   g.bsp = o.mode == CUSHA_MODE_BSP;
   g.world_size = o.world_size;
-  g.rank = mode == kModeNccl ? o.rank : 0;
+  g.rank = multiproc ? o.rank : 0;
   cudaEvent_t e0 = nullptr, eh = nullptr, e1 = nullptr;
   if ((rc = cu(cudaEventCreate(&e0), "cudaEventCreate")) || (rc = cu(cudaEventCreate(&eh), "cudaEventCreate")) ||
       (rc = cu(cudaEventCreate(&e1), "cudaEventCreate")))
@@ -403,7 +444,8 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
     }
     if (plan.bounds.size() - 1 != G) return bail(fail(CUSHA_EINVAL, "partition count"));
     std::vector<Graph*> parts;
-    const uint32_t r0 = h->mode == kModeNccl ? (uint32_t)o.rank : 0u, r1 = h->mode == kModeNccl ? r0 + 1 : G;
+    const bool ranked = h->mode == kModeNccl || h->mode == kModeIpc;  // this process holds its rank's partition
+    const uint32_t r0 = ranked ? (uint32_t)o.rank : 0u, r1 = ranked ? r0 + 1 : G;
     for (uint32_t r = r0; r < r1; ++r) {
       Graph* p = new (std::nothrow) Graph();
       if (!p) { for (Graph* x : parts) { free_device_arrays(*x); delete x; } return bail(fail(CUSHA_ENOMEM, "host")); }
@@ -434,7 +476,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
     delete glob;
     h->parts = parts;
     for (Graph* p : h->parts)
-      if ((rc = alloc_run_state(*p, h->mode == kModeNccl))) return bail(rc);
+      if ((rc = alloc_run_state(*p, ranked))) return bail(rc);
     if (h->mode == kModeSim) {
       std::vector<uint32_t*> sv(G), dirty(G);
       std::vector<Ctl*> ctls(G);
@@ -449,16 +491,18 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
       CKA(cudaMemcpyAsync(h->d_ctls, ctls.data(), sizeof(Ctl*) * G, cudaMemcpyHostToDevice, h->stream));
       CKA(cudaStreamSynchronize(h->stream));
     } else {
+      // one process per GPU: the ranks map each other's arrays (CUDA IPC) -
+      // over an NCCL all-gather of the handles here, or (transport IPC) by the
+      // caller through cusha_ipc_export / cusha_ipc_connect
       Graph& p = *h->parts[0];
       p.comm_timeout_ms = o.comm_timeout_ms ? o.comm_timeout_ms : 300000u;
-      if ((rc = nccl_init(p, o.nccl_unique_id, err))) {
-        set_error("NCCL: " + err);
-        return bail(rc);
+      if (h->mode == kModeNccl) {
+        if ((rc = nccl_init(p, o.nccl_unique_id, err))) {
+          set_error("NCCL: " + err);
+          return bail(rc);
+        }
+        if ((rc = connect_ipc_peers(p))) return bail(rc);
       }
-      if ((rc = connect_ipc_peers(p))) return bail(rc);
-      CKA(dev_alloc((void**)&h->d_ctls, sizeof(Ctl*), h->stream));
-      CKA(cudaMemcpyAsync(h->d_ctls, &p.d_ctl, sizeof(Ctl*), cudaMemcpyHostToDevice, h->stream));
-      CKA(cudaStreamSynchronize(h->stream));
     }
   }
   CKA(cudaEventRecord(e1, h->stream));
@@ -477,7 +521,7 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
   st.h2d_ms = ms_h2d;
   st.h2d_bytes = h2d;
   st.world_size = o.world_size;
-  st.rank = h->mode == kModeNccl ? o.rank : 0;
+  st.rank = multiproc ? o.rank : 0;
   st.partitions = h->mode == kModeSingle ? 1 : G;
   st.max_in_degree = g0(h).max_indeg;
   st.device_bytes = 0;
@@ -798,6 +842,8 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   if ((a == kBFS || a == kSSSP || a == kSSWP) && source >= V) return fail(CUSHA_EINVAL, "source >= num_vertices");
   if (alg_needs_edge_values(a) && !g.has_ev) return fail(CUSHA_EINVAL, "algorithm needs edge_values");
   if (alg_needs_init(a) && !g.d_init[a]) return fail(CUSHA_EINVAL, "NN/HS/CS need cusha_set_vertex_values first");
+  const bool ranked = h->mode == kModeNccl || h->mode == kModeIpc;
+  if (ranked && !g.connected) return fail(CUSHA_ESTATE, "the ranks are not connected yet (cusha_ipc_connect)");
   int rc = check_fixed_range(g, a);
   if (rc) return rc;
   CKA(cudaSetDevice(h->device));
@@ -854,8 +900,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   for (Graph* p : h->parts) CKA(launch_reset_ctl(p->d_ctl, max_iters, st));
   for (Graph* p : h->parts) CKA(launch_init(*p, a, source, st));
   // every partition's SrcValue is initialised (R20) before any pass reads it
-  if (h->mode == kModeNccl && (rc = nccl_allreduce_max_u32(g, &g.d_ctl->lchanged, &g.d_ctl->gchanged, err)))
-    return fail(rc, "init barrier: " + err);
+  if (ranked) CKA(launch_peer_barrier(g, 0, g.comm_timeout_ms, st));
   CKA(cudaEventRecord(evm, st));
   if (max_iters > 0 && multi) {
     KParams kp = pass_params(g, source, cfg, a);
@@ -901,11 +946,10 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
         }
         if (h->mode == kModeSim) {
           CKA(launch_close_parts(h->d_ctls, (uint32_t)h->parts.size(), st));
-        } else if (h->mode == kModeNccl) {
-          const int r2 = nccl_allreduce_max_u32(g, &g.d_ctl->lchanged, &g.d_ctl->gchanged, e2);
-          if (r2) return fail(r2, "convergence all-reduce: " + e2);
-          CKA(launch_close_parts(h->d_ctls, 0, st));
+        } else if (ranked) {  // the barrier between ranks decides global convergence
+          CKA(launch_peer_barrier(g, 1, g.comm_timeout_ms, st));
         }
+        (void)e2;
       }
       return CUSHA_OK;
     };
@@ -939,10 +983,11 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
         CKA(cudaGraphLaunch(h->exec[a], st));
       }
       CKA(cudaMemcpyAsync(g.h_ctl, g.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, st));
-      if (h->mode == kModeNccl) {  // never hang on a failed peer
-        if ((rc = nccl_wait(g, g.comm_timeout_ms, err))) return fail(rc, err);
-      } else {
-        CKA(cudaStreamSynchronize(st));
+      CKA(cudaStreamSynchronize(st));  // (the barrier between ranks is bounded by comm_timeout_ms)
+      if (ranked) {
+        uint32_t perr = 0;
+        CKA(cudaMemcpy(&perr, &g.d_sync->err, 4, cudaMemcpyDeviceToHost));
+        if (perr) return fail(CUSHA_ENCCL, "a rank did not reach the pass barrier within comm_timeout_ms");
       }
       if (g.h_ctl->converged || g.h_ctl->iter >= max_iters) break;
     }
@@ -1008,28 +1053,32 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
 
 // copy every partition's VertexValues slice to dst (host or device)
 static int copy_values(const cusha_graph* h, void* dst, bool to_host) {
-  const uint32_t V = h->st.num_vertices;
   const size_t vb = value_bytes(h->last_alg);
   const cudaMemcpyKind kind = to_host ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
-  if (h->mode == kModeNccl) {
+  if (h->mode == kModeNccl || h->mode == kModeIpc) {
+    // every rank reads every rank's slice from its memory (CUDA IPC): a
+    // barrier before (all ranks finished their runs) and after (no rank frees
+    // or overwrites its slice while another still reads it); collective
     Graph& g = *h->parts[0];
-    void* full = nullptr;
-    CKA(dev_alloc(&full, (size_t)V * vb, h->stream));
-    std::string err;
-    int rc = nccl_gather_values(g, full, (uint32_t)vb, err);
-    if (!rc) rc = nccl_wait(g, g.comm_timeout_ms, err);
-    if (rc) {
-      cudaFreeAsync(full, h->stream);
-      return fail(rc, "gather: " + err);
+    CKA(launch_peer_barrier(g, 0, g.comm_timeout_ms, h->stream));
+    for (uint32_t q = 0; q < g.G; ++q) {
+      const uint64_t v0 = std::min<uint64_t>((uint64_t)g.h_bounds[q] * g.N, g.V);
+      const uint64_t v1 = std::min<uint64_t>((uint64_t)g.h_bounds[q + 1] * g.N, g.V);
+      if (v1 > v0)
+        CKA(cudaMemcpyAsync(static_cast<char*>(dst) + v0 * vb, g.vv_peer[q], (v1 - v0) * vb,
+                            to_host ? cudaMemcpyDeviceToHost : cudaMemcpyDefault, h->stream));
     }
-    CKA(cudaMemcpyAsync(dst, full, (size_t)V * vb, kind, h->stream));
-    cudaFreeAsync(full, h->stream);
-  } else {
-    for (const Graph* g : h->parts)
-      if (g->nvl)
-        CKA(cudaMemcpyAsync(static_cast<char*>(dst) + (size_t)g->v0 * vb, g->d_vv, (size_t)g->nvl * vb, kind,
-                            h->stream));
+    CKA(launch_peer_barrier(g, 0, g.comm_timeout_ms, h->stream));
+    CKA(cudaStreamSynchronize(h->stream));
+    uint32_t perr = 0;
+    CKA(cudaMemcpy(&perr, &g.d_sync->err, 4, cudaMemcpyDeviceToHost));
+    if (perr) return fail(CUSHA_ENCCL, "a rank did not reach the barrier within comm_timeout_ms");
+    return CUSHA_OK;
   }
+  for (const Graph* g : h->parts)
+    if (g->nvl)
+      CKA(cudaMemcpyAsync(static_cast<char*>(dst) + (size_t)g->v0 * vb, g->d_vv, (size_t)g->nvl * vb, kind,
+                          h->stream));
   CKA(cudaStreamSynchronize(h->stream));
   return CUSHA_OK;
 }
@@ -1067,7 +1116,7 @@ int cusha_get_part_stats(const cusha_graph* h, uint32_t part, cusha_stats* s) {
   s->device_bytes = device_bytes(g);
   s->max_part_device_bytes = s->device_bytes;
   s->entries_padded = g.P;
-  s->rank = h->mode == kModeNccl ? h->st.rank : (int)part;
+  s->rank = (h->mode == kModeNccl || h->mode == kModeIpc) ? h->st.rank : (int)part;
   if (h->have_values) {
     s->algorithmic_bytes = g.st.algorithmic_bytes;
     s->paper_bytes = g.st.paper_bytes;
@@ -1154,6 +1203,24 @@ int cusha_get_part_layout(const cusha_graph* h, uint32_t p, cusha_layout_part pa
   if (!h) return fail(CUSHA_EINVAL, "graph is NULL");
   if (p >= h->parts.size()) return fail(CUSHA_EINVAL, "partition not held by this handle");
   return layout_of(*h->parts[p], part, out, out_bytes, count);
+}
+
+int cusha_ipc_export(cusha_graph* h, void* out, size_t bytes) {
+  if (!h || !out) return fail(CUSHA_EINVAL, "null argument");
+  if (h->mode != kModeIpc && h->mode != kModeNccl) return fail(CUSHA_ESTATE, "not a one-process-per-GPU graph");
+  if (bytes != kIpcBlob) return fail(CUSHA_EINVAL, "bytes must be CUSHA_IPC_BLOB_BYTES");
+  CKA(cudaSetDevice(h->device));
+  return ipc_export_blob(*h->parts[0], out);
+}
+
+int cusha_ipc_connect(cusha_graph* h, const void* all, size_t bytes) {
+  if (!h || !all) return fail(CUSHA_EINVAL, "null argument");
+  if (h->mode != kModeIpc) return fail(CUSHA_ESTATE, "not a caller-bootstrapped (transport IPC) graph");
+  Graph& g = *h->parts[0];
+  if (g.connected) return fail(CUSHA_ESTATE, "already connected");
+  if (bytes != kIpcBlob * g.G) return fail(CUSHA_EINVAL, "bytes must be world_size * CUSHA_IPC_BLOB_BYTES");
+  CKA(cudaSetDevice(h->device));
+  return ipc_connect_blob(g, all);
 }
 
 int cusha_nccl_unique_id(void* out128) {

@@ -630,7 +630,7 @@ void partition_bounds(uint32_t S, const uint64_t* work, uint32_t G, uint32_t* bo
 
 void free_device_arrays(Graph& g) {
   void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcloc, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
-                  g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_vv, g.d_ctl, g.d_trace,
+                  g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_ctl, g.d_trace, g.d_sync_peer,
                   g.d_active, g.d_bounds, g.d_owner, g.d_cwp, g.d_run_k, g.d_run_t, g.d_sv_peer, g.d_dirty_peer,
                   g.d_run_unit, g.d_run_bits, g.d_run_d, g.d_shard_seq, g.d_cw_win, g.d_cw_delta, g.d_order};
   for (void* p : ptrs)
@@ -644,6 +644,15 @@ void free_device_arrays(Graph& g) {
     else cudaFreeAsync(g.d_srcvalue, g.stream);
   }
   if (g.d_srcvalue2) cudaFreeAsync(g.d_srcvalue2, g.stream);
+  if (g.d_vv) {
+    if (g.srcvalue_ipc) cudaFree(g.d_vv);
+    else cudaFreeAsync(g.d_vv, g.stream);
+  }
+  if (g.d_sync) cudaFree(g.d_sync);
+  g.d_sync = nullptr;
+  g.d_sync_peer = nullptr;
+  g.vv_peer.clear();
+  g.connected = false;
   g.d_srcvalue2 = nullptr;
   for (void*& p : g.d_init)
     if (p) { cudaFreeAsync(p, g.stream); p = nullptr; }

@@ -28,6 +28,15 @@ struct Ctl {
   uint32_t conv_iter;         // 1 + the last of those passes (~0u: none yet)
 };
 
+// One process per GPU (row e): every rank's barrier block, in its own memory,
+// mapped by the others (CUDA IPC).  Round r of the barrier uses slot r & 1.
+struct PeerSync {
+  uint32_t arrive[2];       // ranks that reached this round
+  uint32_t round;           // barrier rounds this rank completed
+  uint32_t err;             // 1: a peer did not arrive within the timeout
+  uint32_t changed[2][64];  // rank q's "committed an update" word of this round
+};
+
 // Per-iteration trace (row f4; also the source of algorithmic byte counts).
 struct TraceRec {
   uint32_t updated;          // vertices committed in stage 3
@@ -207,6 +216,10 @@ struct Graph {
   uint32_t* d_cwp = nullptr;        // Sl*(G+1)
   uint32_t** d_sv_peer = nullptr;   // G: SrcValue of every partition (device pointers valid on this device)
   uint32_t** d_dirty_peer = nullptr;// G: dirty[] of every partition (skip_clean only)
+  PeerSync* d_sync = nullptr;       // one process per GPU: this rank's barrier block (cudaMalloc, exported)
+  PeerSync** d_sync_peer = nullptr; // G: every rank's barrier block
+  std::vector<void*> vv_peer;       // G: every rank's VertexValues (for cusha_get_values)
+  bool connected = false;           // peers mapped (multi-process modes)
   std::vector<void*> ipc_open;      // peer allocations mapped with cudaIpcOpenMemHandle
   void* nccl_comm = nullptr;        // ncclComm_t (real multi-GPU)
   uint32_t comm_timeout_ms = 300000;
@@ -222,6 +235,9 @@ const PassKernel& pass_kernel(int alg, int repr);
 cudaError_t launch_init(const Graph& g, int alg, uint32_t source, cudaStream_t s);
 cudaError_t launch_reset_ctl(Ctl* ctl, uint32_t max_iters, cudaStream_t s);
 cudaError_t launch_close_parts(Ctl* const* ctls, uint32_t G, cudaStream_t s);  // partitioned: global convergence
+// one process per GPU: barrier over the ranks' PeerSync blocks; decide = also
+// OR the ranks' lchanged words into the convergence flag
+cudaError_t launch_peer_barrier(const Graph& g, int decide, uint32_t timeout_ms, cudaStream_t s);
 KParams make_params(const Graph& g, uint32_t source);
 size_t value_bytes(int alg);
 int timeline_copy(void* out, size_t bytes);  // CUSHA_TIMELINE builds: per-ticket stamps (else -1)
@@ -282,8 +298,6 @@ void set_error(const std::string& msg);
 int nccl_unique_id(void* out128, std::string& err);
 int nccl_init(Graph& g, const void* id128, std::string& err);
 int nccl_allgather_bytes(Graph& g, const void* dsend, void* drecv, size_t bytes, std::string& err);
-int nccl_allreduce_max_u32(Graph& g, const uint32_t* dsend, uint32_t* drecv, std::string& err);
-int nccl_gather_values(Graph& g, void* dfull, uint32_t value_bytes, std::string& err);  // every rank's vv slice
 int nccl_wait(Graph& g, uint32_t timeout_ms, std::string& err);  // stream drained, or abort on error / timeout
 void nccl_destroy(Graph& g);
 

@@ -1274,6 +1274,49 @@ cudaError_t launch_init(const Graph& g, int alg, uint32_t source, cudaStream_t s
   return cudaErrorInvalidValue;
 }
 
+// ------------------------------------ barrier between ranks (row e, one process per GPU)
+// After a pass: every rank stores its "committed an update" word into every
+// rank's block, then counts itself in; it waits until all G ranks arrived, and
+// the run has converged when no rank committed (L189).  The same G words
+// reach every rank, so all take the same decision.  A rank re-uses a slot two
+// rounds later only after every rank passed the round in between, which needs
+// this rank's arrival there - issued after the reset below.  Bounded: after
+// timeout_ms the rank flags err and stops its run instead of spinning forever.
+__global__ void peer_barrier(PeerSync* const* peers, uint32_t G, uint32_t rank, Ctl* ctl, uint32_t timeout_ms,
+                             int decide) {
+  if (threadIdx.x != 0) return;
+  __threadfence_system();  // this rank's pass (its stage-4 stores to the peers) before the arrival
+  PeerSync* me = peers[rank];
+  const uint32_t r = ld_vol(&me->round), par = r & 1u;
+  const uint32_t v = decide ? ld_vol(&ctl->lchanged) : 0u;
+  for (uint32_t q = 0; q < G; ++q) st_vol(&peers[q]->changed[par][rank], v);
+  __threadfence_system();
+  for (uint32_t q = 0; q < G; ++q) atomicAdd_system(&peers[q]->arrive[par], 1u);
+  uint64_t t0, t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  while (ld_vol(&me->arrive[par]) < G) {
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t - t0 > (uint64_t)timeout_ms * 1000000ull) {
+      me->err = 1u;
+      ctl->converged = 1u;  // stop this rank's run; the host reports the timeout
+      break;
+    }
+    __nanosleep(256);
+  }
+  __threadfence_system();
+  uint32_t any = 0;
+  for (uint32_t q = 0; q < G; ++q) any |= ld_vol(&me->changed[par][q]);
+  if (decide && !ctl->converged && ctl->iter >= 1 && !any) ctl->converged = 1u;
+  st_vol(&me->arrive[par], 0u);
+  st_vol(&me->round, r + 1);
+  __threadfence_system();
+}
+
+cudaError_t launch_peer_barrier(const Graph& g, int decide, uint32_t timeout_ms, cudaStream_t s) {
+  peer_barrier<<<1, 32, 0, s>>>(g.d_sync_peer, g.G, g.part, g.d_ctl, timeout_ms, decide);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_close_parts(Ctl* const* ctls, uint32_t G, cudaStream_t s) {
   // ctls: device array; G > 0: all partitions of this process (simulation); G == 0: one rank after its all-reduce
   close_parts<<<1, 32, 0, s>>>(ctls, G ? G : 1u, G ? 1 : 0);

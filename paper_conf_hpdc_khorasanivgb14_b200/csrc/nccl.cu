@@ -2,13 +2,13 @@
 //
 // libnccl.so.2 is opened at run time (dlopen), so single-GPU use has no NCCL
 // dependency; torch ships the library and has normally loaded it already.
-// The write-back values themselves never go through NCCL: stage 4 stores them
-// straight into the owning rank's SrcValue over NVLink (CUDA IPC mappings,
-// api.cu).  NCCL carries (1) at build time the 64-byte IPC handles of every
-// rank's SrcValue / dirty arrays (all-gather), (2) once per pass the
-// partition's "committed an update" word (all-reduce MAX), which is both the
-// global convergence test of L189 and the barrier between passes, and (3) at
-// cusha_get_values every rank's VertexValues slice (grouped broadcasts).
+// NCCL only bootstraps the ranks: at build time it all-gathers the CUDA IPC
+// handles of every rank's SrcValue, dirty[], barrier block and VertexValues.
+// Everything after that is peer memory over NVLink / NVSwitch (api.cu,
+// kernels.cu): stage 4 stores the write-back values straight into the owning
+// rank's SrcValue, the per-pass barrier and convergence vote are stores and
+// system-scope atomics into the ranks' barrier blocks, and cusha_get_values
+// reads every rank's VertexValues slice directly.
 #include <dlfcn.h>
 #include <nccl.h>
 
@@ -99,29 +99,6 @@ int nccl_init(Graph& g, const void* id128, std::string& err) {
 int nccl_allgather_bytes(Graph& g, const void* dsend, void* drecv, size_t bytes, std::string& err) {
   if (!g.nccl_comm) { err = "the NCCL communicator was aborted"; return CUSHA_ENCCL; }
   NC(api().allGather(dsend, drecv, bytes, ncclUint8, static_cast<ncclComm_t>(g.nccl_comm), g.stream));
-  return CUSHA_OK;
-}
-
-int nccl_allreduce_max_u32(Graph& g, const uint32_t* dsend, uint32_t* drecv, std::string& err) {
-  if (!g.nccl_comm) { err = "the NCCL communicator was aborted"; return CUSHA_ENCCL; }
-  NC(api().allReduce(dsend, drecv, 1, ncclUint32, ncclMax, static_cast<ncclComm_t>(g.nccl_comm), g.stream));
-  return CUSHA_OK;
-}
-
-// Rank r broadcasts its VertexValues slice (its vertices [v0, v0 + nvl)) into
-// the same place of every rank's |V|-element buffer dfull.
-int nccl_gather_values(Graph& g, void* dfull, uint32_t vb, std::string& err) {
-  if (!g.nccl_comm) { err = "the NCCL communicator was aborted"; return CUSHA_ENCCL; }
-  ncclComm_t comm = static_cast<ncclComm_t>(g.nccl_comm);
-  char* full = static_cast<char*>(dfull);
-  NC(api().groupStart());
-  for (uint32_t r = 0; r < g.G; ++r) {
-    const uint64_t v0 = std::min<uint64_t>((uint64_t)g.h_bounds[r] * g.N, g.V);
-    const uint64_t v1 = std::min<uint64_t>((uint64_t)g.h_bounds[r + 1] * g.N, g.V);
-    const void* send = r == g.part ? g.d_vv : full + v0 * vb;
-    NC(api().broadcast(send, full + v0 * vb, (v1 - v0) * vb, ncclUint8, (int)r, comm, g.stream));
-  }
-  NC(api().groupEnd());
   return CUSHA_OK;
 }
 

@@ -53,6 +53,7 @@ class BuildOpts(ctypes.Structure):
         ("keep_layout", ctypes.c_int),
         ("mode", ctypes.c_int),
         ("comm_timeout_ms", ctypes.c_uint32),
+        ("transport", ctypes.c_int),
     ]
 
 
@@ -120,6 +121,8 @@ def lib():
             "cusha_get_part_layout": (i32, [P, u32, i32, P, sz, ctypes.POINTER(u64)]),
             "cusha_get_part_stats": (i32, [P, u32, ctypes.POINTER(Stats)]),
             "cusha_trim_memory": (i32, [i32]),
+            "cusha_ipc_export": (i32, [P, P, sz]),
+            "cusha_ipc_connect": (i32, [P, P, sz]),
             "cusha_shard_size": (u32, [u32, u64, u32, u32, u32]),
             "cusha_value_bytes": (sz, [i32]),
             "cusha_last_error": (ctypes.c_char_p, []),
@@ -247,7 +250,7 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
                 host_loop: bool = False, world_size: int = 1, rank: int = 0,
                 nccl_id: Optional[bytes] = None, skip_clean_shards: bool = False,
                 device_topology_budget: int = 0, pass_barrier: int = 0, keep_layout: bool = False,
-                mode="async") -> Graph:
+                mode="async", transport: str = "nccl", comm_timeout_ms: int = 0) -> Graph:
     """cusha_build_graph.  src/dst/edge_values: numpy (host, copied in) or CUDA tensors (device).
     world_size > 1: destination-range partition; nccl_id = None simulates all
     partitions on this device, else one process per GPU over NCCL.
@@ -297,6 +300,8 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
     o.pass_barrier = int(pass_barrier)
     o.keep_layout = int(keep_layout)
     o.mode = {"async": 0, "bsp": 1}[mode] if isinstance(mode, str) else int(mode)
+    o.transport = {"nccl": 0, "ipc": 1}[transport] if isinstance(transport, str) else int(transport)
+    o.comm_timeout_ms = int(comm_timeout_ms)
     idbuf = None
     if nccl_id is not None:
         if len(nccl_id) != 128:
@@ -308,6 +313,23 @@ def build_graph(num_vertices: int, src, dst, edge_values=None, repr="gs", vertic
     _check(lib().cusha_build_graph(num_vertices, len(src), _ptr(src), _ptr(dst), _ptr(edge_values),
                                    ctypes.byref(o), ctypes.byref(h)), "cusha_build_graph")
     return Graph(h.value, num_vertices, len(src))
+
+
+IPC_BLOB_BYTES = 256
+
+
+def ipc_export(g: Graph) -> bytes:
+    """cusha_ipc_export: this rank's CUDA IPC handles (one process per GPU)."""
+    buf = ctypes.create_string_buffer(IPC_BLOB_BYTES)
+    _check(lib().cusha_ipc_export(g.handle, buf, IPC_BLOB_BYTES), "cusha_ipc_export")
+    return buf.raw
+
+
+def ipc_connect(g: Graph, blobs) -> None:
+    """cusha_ipc_connect: every rank's ipc_export blob, in rank order."""
+    allb = b"".join(bytes(b) for b in blobs)
+    buf = ctypes.create_string_buffer(allb, len(allb))
+    _check(lib().cusha_ipc_connect(g.handle, buf, len(allb)), "cusha_ipc_connect")
 
 
 def set_vertex_values(g: Graph, alg, values: np.ndarray):

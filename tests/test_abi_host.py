@@ -32,7 +32,7 @@ def test_library_exports_every_declared_symbol():
     out = subprocess.run(["nm", "-D", "--defined-only", cusha.LIB_PATH], capture_output=True, text=True).stdout
     exported = set(re.findall(r"\b(cusha_\w+)\b", out))
     assert names <= exported
-    assert cusha.abi_version() == 4
+    assert cusha.abi_version() == 5
 
 
 def test_struct_layout_matches_header(tmp_path):
