@@ -108,22 +108,21 @@ typedef struct {
    * and the integer algorithms store only changed vertices, so the exchange is
    * exactly the changed values, overlapped with the other shards' work.
    * After each pass the partitions' "committed an update" words are OR-ed:
-   * the global convergence test of L189.  CW representation only; no
-   * host-streamed topology.
-   *   nccl_unique_id != NULL: one process per GPU; every rank passes the full
-   *     edge list, its rank and the same 128-byte ncclUniqueId
-   *     (cusha_nccl_unique_id on rank 0, broadcast by the caller).  The ranks
-   *     map each other's SrcValue arrays with CUDA IPC (handles exchanged by
-   *     an NCCL all-gather during this call), so stage-4 stores travel over
-   *     NVLink / NVSwitch; the per-pass OR is an NCCL all-reduce.  Every rank
-   *     must make the same sequence of calls (build, run, get_values).
-   *   nccl_unique_id == NULL: all G partitions run in this process on one
+   * the global convergence test of L189.  CW representation only.
+   *   One process per GPU (nccl_unique_id != NULL, or transport IPC): every
+   *     rank passes the full edge list and its rank; it builds only its own
+   *     partition.  The ranks map each other's SrcValue, dirty[], barrier
+   *     block and VertexValues with CUDA IPC (see `transport`), so stage-4
+   *     stores travel over NVLink / NVSwitch and the per-pass OR and barrier
+   *     are stores and system-scope atomics in peer memory.  Every rank must
+   *     make the same sequence of calls (build, run, get_values).
+   *   nccl_unique_id == NULL (transport NCCL): all G partitions run in this process on one
    *     device (each partition with its own arrays, the same kernels and the
    *     same stores into the sibling partitions' SrcValue; the OR is a kernel
    *     over the partitions' words).  Used to test the partitioned algorithm
    *     on one GPU.                                                            */
   int world_size;                  /* 1 = single partition (0 is treated as 1)                  */
-  int rank;                        /* this process's rank, 0..world_size-1 (NCCL mode)          */
+  int rank;                        /* this process's rank, 0..world_size-1 (one process per GPU) */
   const void* nccl_unique_id;      /* 128-byte ncclUniqueId, or NULL (see above)                */
   /* Clean-shard skipping (opt-in; not in the paper, which processes every
    * shard in every iteration, Fig. 5 line 3 / L189).  1: a shard none of whose
@@ -176,9 +175,9 @@ typedef struct {
    *   the oracle's mode T pass for pass (tests/test_gpu_bsp.py).  Single
    *   partition only; one launch per pass plus a copy of SrcValue.         */
   int mode;
-  /* One process per GPU: how long (ms) a rank waits for its peers' collective
-   * before it aborts the communicator and returns CUSHA_ENCCL (an NCCL
-   * asynchronous error does the same at once).  0 = 300000.                 */
+  /* One process per GPU: how long (ms) a rank waits for its peers (the NCCL
+   * bootstrap, a pass barrier) before it gives up and returns CUSHA_ENCCL
+   * (an NCCL asynchronous error aborts the bootstrap at once).  0 = 300000.  */
   uint32_t comm_timeout_ms;
   /* One process per GPU: how the ranks find each other's arrays.
    * CUSHA_TRANSPORT_NCCL (0): with nccl_unique_id, cusha_build_graph
