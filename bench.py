@@ -264,23 +264,24 @@ def bench_cusha(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    dev = local
+    # --share-gpu (tests only): every rank on cuda:0 over a gloo group, to run
+    # this multi-rank path on a one-GPU box; its numbers are not a scaling result
+    dev = 0 if args.share_gpu else local
+    torch.cuda.set_device(dev)
     dist = None
     nccl_id = None
     if world > 1:
         # one process per GPU; libcusha's stage 4 stores into the other ranks'
-        # SrcValue over NVLink (CUDA IPC) and NCCL all-reduces the per-pass
-        # convergence word (destination-range partition);
-        # torch.distributed only carries rank 0's ncclUniqueId, the barriers and
-        # the max-over-ranks time
+        # SrcValue over NVLink and the pass barrier / convergence vote run in
+        # peer memory (CUDA IPC; destination-range partition).
+        # torch.distributed carries the ranks' IPC handles (transport IPC), the
+        # barriers and the max-over-ranks time
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{dev}"))
-        idt = torch.zeros(128, dtype=torch.uint8, device=f"cuda:{dev}")
-        if rank == 0:
-            idt.copy_(torch.frombuffer(bytearray(cusha.nccl_unique_id()), dtype=torch.uint8))
-        dist.broadcast(idt, 0)
-        nccl_id = bytes(idt.cpu().numpy().tobytes())
+        if args.share_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device(f"cuda:{dev}"))
+    cdev = "cpu" if args.share_gpu else f"cuda:{dev}"  # device of the small collectives
     alg, repr_, source, desc = WORKLOADS[args.workload]
     if args.N == 0 and args.workload == "C1":
         args.N = 128  # the L310 rule gives 3 shards at this size
@@ -291,7 +292,7 @@ def bench_cusha(args):
     wl = load_graph(args.workload, args.cache_dir)
     stream = torch.cuda.current_stream()
     if world > 1:
-        part = dict(world_size=world, rank=rank, nccl_id=nccl_id)
+        part = dict(world_size=world, rank=rank, transport="ipc")
     else:
         part = dict(world_size=max(1, args.sim_parts))  # > 1: one-process partition simulation (tests/tools)
 
@@ -303,14 +304,14 @@ def bench_cusha(args):
     def max_over_ranks(x):
         if dist is None:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device=f"cuda:{dev}")
+        t = torch.tensor([x], dtype=torch.float64, device=cdev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
     def sum_over_ranks(x):
         if dist is None:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device=f"cuda:{dev}")
+        t = torch.tensor([x], dtype=torch.float64, device=cdev)
         dist.all_reduce(t, op=dist.ReduceOp.SUM)
         return float(t.item())
 
@@ -320,9 +321,16 @@ def bench_cusha(args):
     if alg in ("sssp", "sswp"):
         ev = torch.from_numpy(wl.edge_u32.view(np.int32)).to(f"cuda:{dev}")
     torch.cuda.synchronize()
-    g = cusha.build_graph(wl.V, src_d, dst_d, edge_values=ev, repr=repr_, vertices_per_shard=args.N, device=dev,
-                          stream=stream.cuda_stream, host_loop=args.host_loop,
-                          skip_clean_shards=args.skip_clean, pass_barrier=args.pass_barrier, **part)
+    def connect(gh):
+        if world > 1:  # the caller's bootstrap of the IPC transport
+            blobs = [None] * world
+            dist.all_gather_object(blobs, cusha.ipc_export(gh))
+            cusha.ipc_connect(gh, blobs)
+        return gh
+
+    g = connect(cusha.build_graph(wl.V, src_d, dst_d, edge_values=ev, repr=repr_, vertices_per_shard=args.N,
+                                  device=dev, stream=stream.cuda_stream, host_loop=args.host_loop,
+                                  skip_clean_shards=args.skip_clean, pass_barrier=args.pass_barrier, **part))
     st0 = cusha.get_stats(g)
     log(f"[bench] rank {rank}/{world} built {repr_} |N|={st0['vertices_per_shard']} |S|={st0['num_shards']} "
         f"partitions={st0['partitions']} in {st0['build_ms']:.1f} ms; device bytes {st0['device_bytes'] / 1e9:.3f} GB "
@@ -375,10 +383,11 @@ def bench_cusha(args):
 
         def e2e_step():
             # the user's call sequence: build from host buffers (H2D inside), run, read the result (D2H)
-            gh = cusha.build_graph(wl.V, pin_s.numpy().view(np.uint32), pin_d.numpy().view(np.uint32),
-                                   edge_values=None if pin_w is None else pin_w.numpy().view(np.uint32),
-                                   repr=repr_, vertices_per_shard=args.N, device=dev, stream=stream.cuda_stream,
-                                   skip_clean_shards=args.skip_clean, pass_barrier=args.pass_barrier, **part)
+            gh = connect(cusha.build_graph(wl.V, pin_s.numpy().view(np.uint32), pin_d.numpy().view(np.uint32),
+                                           edge_values=None if pin_w is None else pin_w.numpy().view(np.uint32),
+                                           repr=repr_, vertices_per_shard=args.N, device=dev,
+                                           stream=stream.cuda_stream, skip_clean_shards=args.skip_clean,
+                                           pass_barrier=args.pass_barrier, **part))
             cusha.run(alg, gh, source=source)
             n = cusha.get_stats(gh)["edges_processed"]
             rc = cusha.lib().cusha_get_values(gh.handle, cusha._ptr(out), wl.V * vb)
@@ -421,7 +430,7 @@ def bench_cusha(args):
                 "passes": "one launch per pass, device-wide barrier between passes" if not overlapped
                 else "overlapped passes in one launch (DESIGN.md \"Overlapped passes\")",
                 "parallelism": (f"destination-range partition x{world}: stage-4 stores over NVLink (CUDA IPC), "
-                                "NCCL all-reduce of the convergence word") if world > 1 else
+                                "pass barrier and convergence vote in peer memory") if world > 1 else
                                (f"1 GPU, {local_parts} simulated partitions" if local_parts > 1 else "1 GPU"),
                 "partitions": st0["partitions"], "device_bytes_per_gpu": st0["max_part_device_bytes"]},
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
@@ -499,6 +508,8 @@ def main():
                     help="one launch per pass with a device-wide barrier between passes (Fig. 5) instead of "
                          "the default overlapped passes")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--share-gpu", action="store_true",
+                    help="tests only: all ranks on cuda:0 over gloo (exercises the multi-rank path on one GPU)")
     ap.add_argument("--sim-parts", type=int, default=1,
                     help="one process: simulate this many destination-range partitions on one GPU (tools/tests)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -508,7 +519,7 @@ def main():
     if world and world != args.gpus:
         log(f"[bench] WORLD_SIZE={world} but --gpus {args.gpus}")
         return 2
-    if args.gpus > 1 and not world and args.impl == "cusha":
+    if args.gpus > 1 and not world and args.impl == "cusha" and not args.share_gpu:
         return relaunch_under_torchrun(args)
     if world > 1:
         os.environ.setdefault("NCCL_DEBUG", "INFO")

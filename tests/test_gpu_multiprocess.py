@@ -143,3 +143,26 @@ def test_c4_cc_sswp_ranks_as_processes(world):
             rc, vals = res[r][alg]
             assert rc == 0
             np.testing.assert_array_equal(vals, ref, err_msg=f"rank {r} {alg}")
+
+
+def test_bench_two_ranks_on_one_gpu(tmp_path):
+    """bench.py's multi-rank path (torchrun launch, IPC bootstrap over
+    torch.distributed, max-over-ranks timing, one JSON line from rank 0) with
+    both ranks sharing cuda:0 (--share-gpu; the numbers are not a scaling
+    result, the code path is the driver's N>1 one)."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+                          "--master-addr", "127.0.0.1", "--master-port", str(_free_port()),
+                          os.path.join(root, "bench.py"), "--gpus", "2", "--share-gpu", "--workload", "C4cc",
+                          "--steps", "2", "--warmup", "3", "--e2e-steps", "1", "--no-cpu-baseline",
+                          "--cache-dir", str(tmp_path)],
+                         capture_output=True, text=True, timeout=500, cwd=root)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["run"]["partitions"] == 2
+    assert d["e2e"]["value"] > 0
