@@ -15,7 +15,8 @@ s, d = graphgen.rmat(V, 200000, seed=71)
 w = graphgen.edge_u32(s, d, seed=71, lo=1, hi=255)
 ALL = {"default": {}, "pass_barrier": {"pass_barrier": True}, "host_loop": {"host_loop": True},
        "partition3": {"world_size": 3}, "skip": {"skip_clean_shards": True},
-       "host_topology": {"device_topology_budget": 600000}}
+       "host_topology": {"device_topology_budget": 600000}, "bsp": {"mode": "bsp"},
+       "partition3_host": {"world_size": 3, "device_topology_budget": 1}}
 names = sys.argv[1:] or ["default"]
 if names == ["all"]:
     names = list(ALL)
@@ -24,7 +25,7 @@ NPS = int(os.environ.get("SAN_N", "500"))  # vertices per shard
 for mname in names:
     kw = ALL[mname]
     for repr_ in reprs:
-        if mname == "partition3" and repr_ == "gs":
+        if mname.startswith("partition3") and repr_ == "gs":
             continue  # the partitioned mode uses CW (include/cusha.h)
         for alg in ("bfs", "sssp", "pr", "cc"):
             with cusha.build_graph(V, s, d, edge_values=w if alg == "sssp" else None, repr=repr_,
