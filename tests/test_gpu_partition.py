@@ -147,3 +147,37 @@ def test_partition_device_bytes_shrink_with_G():
             sizes[G] = cusha.get_stats(g)["max_part_device_bytes"]
     for G in (2, 4, 8):
         assert sizes[G] < 1.6 * sizes[1] / G, sizes
+
+
+def test_partition_edge_cases():
+    """The partitioned build straight from the edge list on degenerate inputs:
+    no edges, a partial last shard, more partitions than shards, duplicate
+    edges and self-loops (R22), and an empty partition-to-be (one huge shard)."""
+    # no edges at all
+    z = np.zeros(0, np.uint32)
+    _, got, st, b = run_part("bfs", 1000, z, z, 4, N=100, source=7)
+    assert got[7] == 0 and (np.delete(got, 7) == 0xFFFFFFFF).all() and len(b) == 5
+    # partial last shard (V not a multiple of N), duplicates and self-loops
+    V = 1003
+    s, d = graphgen.rmat(1024, 9000, seed=95)
+    keep = (s < V) & (d < V)
+    s, d = s[keep], d[keep]
+    rng = np.random.default_rng(95)
+    dup = rng.integers(0, len(s), 500)
+    loops = rng.integers(0, V, 50).astype(np.uint32)
+    s = np.concatenate([s, s[dup], loops]).astype(np.uint32)
+    d = np.concatenate([d, d[dup], loops]).astype(np.uint32)
+    w = graphgen.edge_u32(s, d, seed=95, lo=1, hi=255)
+    for G in (2, 5):
+        _, got, _, _ = run_part("sssp", V, s, d, G, ev=w, N=97)
+        np.testing.assert_array_equal(got, oracle.sssp(V, s, d, w, 0))
+        _, got, _, _ = run_part("cc", V, s, d, G, N=97)
+        np.testing.assert_array_equal(got, oracle.cc(V, s, d))
+    # one shard holds almost all the work: the greedy split leaves a partition thin
+    V = 4000
+    hub_s = np.arange(1, 3000, dtype=np.uint32)
+    s2 = np.concatenate([hub_s, np.array([3500, 3600], np.uint32)])
+    d2 = np.concatenate([np.zeros(len(hub_s), np.uint32), np.array([3600, 3700], np.uint32)])
+    for G in (2, 4):
+        _, got, st, b = run_part("bfs", V, s2, d2, G, N=500, source=3500)
+        np.testing.assert_array_equal(got, oracle.bfs(V, s2, d2, 3500))
