@@ -382,7 +382,10 @@ int cusha_build_graph(uint32_t V, uint64_t E, const uint32_t* src, const uint32_
       return bail(rc);
     }
     chunks.n = E >= (1ull << 22) ? 8 : 1;
-    for (int c = 0; c <= chunks.n; ++c) chunks.bounds[c] = E * (uint64_t)c / (uint64_t)chunks.n;
+    if (const char* v = std::getenv("CUSHA_H2D_CHUNKS"))  // tuning probe only
+      if (E >= (1ull << 22)) chunks.n = std::max(1, std::min(16, std::atoi(v)));
+    for (int c = 0; c <= chunks.n; ++c)  // inner bounds on 256-edge boundaries (aligned chunk sorts)
+      chunks.bounds[c] = c == chunks.n ? E : (E * (uint64_t)c / (uint64_t)chunks.n) & ~255ull;
     rc = cu(cudaStreamWaitEvent(cs, eh, 0), "wait");
     for (int c = 0; c < chunks.n && !rc; ++c) {
       const uint64_t lo = chunks.bounds[c], n = chunks.bounds[c + 1] - lo;

@@ -15,6 +15,7 @@
 // shard j (L155), so Mapper and SrcIndexCW are read off the window table.
 #include <cub/cub.cuh>
 
+#include <algorithm>
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
@@ -60,10 +61,90 @@ __global__ void k_ingest(const uint32_t* __restrict__ src, const uint32_t* __res
     } else {
       keys[e] = ((uint64_t)(d / N) << (bsrc + bn)) | ((uint64_t)s << bn) | (uint64_t)(d % N);
       atomicAdd(&outdeg[s], 1u);
-      atomicAdd(&indeg[d], 1u);
+      if (indeg) atomicAdd(&indeg[d], 1u);
     }
     ids[e] = (uint32_t)e;
   }
+}
+
+// ---- chunked G-Shards sort (row f2).  With a host edge list
+// each input chunk is radix-sorted as soon as its copy lands and folded into
+// the sorted prefix of the earlier chunks by a stable merge: on equal keys the
+// prefix goes first, and every input index in it is smaller, so the result is
+// the one stable sort of the whole list (R17).  Only the last chunk's sort and
+// one merge pass remain after the copy.
+constexpr int kMergeItems = 8, kMergeThreads = 256, kMergeTile = kMergeItems * kMergeThreads;
+
+// merge path: how many of the first d outputs come from a (ties: a first)
+template <class I>
+__device__ __forceinline__ I merge_split(const uint64_t* a, I na, const uint64_t* b, I nb, I d) {
+  I lo = d > nb ? d - nb : 0, hi = d < na ? d : na;
+  while (lo < hi) {
+    const I mid = (lo + hi) >> 1;
+    if (a[mid] <= b[d - mid - 1]) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
+}
+__global__ void k_merge_splits(const uint64_t* __restrict__ a, uint64_t na, const uint64_t* __restrict__ b, uint64_t nb,
+                               uint64_t tiles, uint64_t* split) {
+  GRID_STRIDE(t, tiles + 1) split[t] = merge_split<uint64_t>(a, na, b, nb, min(t * (uint64_t)kMergeTile, na + nb));
+}
+// one tile of kMergeTile outputs per block: both input ranges staged in shared
+// memory, kMergeItems outputs per thread, written back coalesced
+__global__ void __launch_bounds__(kMergeThreads) k_merge(const uint64_t* __restrict__ ak, const uint32_t* __restrict__ ai,
+                                                         uint64_t na, const uint64_t* __restrict__ bk,
+                                                         const uint32_t* __restrict__ bi, uint64_t nb,
+                                                         const uint64_t* __restrict__ split, uint64_t* ok, uint32_t* oi) {
+  __shared__ uint64_t sk[kMergeTile];
+  __shared__ uint32_t si[kMergeTile];
+  const uint64_t d0 = blockIdx.x * (uint64_t)kMergeTile, d1 = min(d0 + kMergeTile, na + nb);
+  const uint64_t a0 = split[blockIdx.x], a1 = split[blockIdx.x + 1], b0 = d0 - a0;
+  const uint32_t la = (uint32_t)(a1 - a0), n = (uint32_t)(d1 - d0), lb = n - la;
+  for (uint32_t x = threadIdx.x; x < n; x += kMergeThreads) {
+    if (x < la) { sk[x] = ak[a0 + x]; si[x] = ai[a0 + x]; }
+    else { sk[x] = bk[b0 + x - la]; si[x] = bi[b0 + x - la]; }
+  }
+  __syncthreads();
+  const uint32_t d = min((uint32_t)threadIdx.x * kMergeItems, n);
+  uint32_t i = merge_split<uint32_t>(sk, la, sk + la, lb, d), j = d - i;
+  uint64_t rk[kMergeItems];
+  uint32_t ri[kMergeItems];
+#pragma unroll
+  for (int k = 0; k < kMergeItems; ++k) {
+    if (d + k < n) {
+      const bool from_a = j >= lb || (i < la && sk[i] <= sk[la + j]);
+      const uint32_t x = from_a ? i++ : la + j++;
+      rk[k] = sk[x];
+      ri[k] = si[x];
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int k = 0; k < kMergeItems; ++k)
+    if (d + k < n) { sk[d + k] = rk[k]; si[d + k] = ri[k]; }
+  __syncthreads();
+  for (uint32_t x = threadIdx.x; x < n; x += kMergeThreads) {
+    ok[d0 + x] = sk[x];
+    oi[d0 + x] = si[x];
+  }
+}
+
+// largest in-degree (fixed-point range check) from the shards: in-edges of a
+// vertex all sit in its shard, so one block per shard counts its DestIndex
+// values in shared memory (N counters) — no global atomics during ingest
+__global__ void k_indeg_max(const uint16_t* __restrict__ dest, const uint32_t* __restrict__ off,
+                            const uint32_t* __restrict__ cnt, uint32_t N, uint32_t* out) {
+  extern __shared__ uint32_t hist[];
+  for (uint32_t v = threadIdx.x; v < N; v += blockDim.x) hist[v] = 0;
+  __syncthreads();
+  const uint32_t b = off[blockIdx.x], e = b + cnt[blockIdx.x];
+  for (uint32_t p = b + threadIdx.x; p < e; p += blockDim.x) atomicAdd(&hist[dest[p]], 1u);
+  __syncthreads();
+  uint32_t m = 0;
+  for (uint32_t v = threadIdx.x; v < N; v += blockDim.x) m = max(m, hist[v]);
+  for (int o = 16; o; o >>= 1) m = max(m, __shfl_xor_sync(0xFFFFFFFFu, m, o));
+  if ((threadIdx.x & 31) == 0 && m) atomicMax(out, m);
 }
 
 // start[t] = first sorted index whose (key >> shift) >= t, for t = 0..S
@@ -386,51 +467,101 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   t_alloc_stream = st;
 
   DevBuf keys, keys2, ids, ids2, bad, start, padded, temp, indeg, mx;
+  // per-chunk sorts + merges (host input in several chunks) when the third
+  // pair of key/index buffers fits comfortably; otherwise one sort at the end
+  // (same result, DESIGN.md f2)
+  const int nch = chunks && chunks->n ? chunks->n : 1;
+  bool chunk_sort = nch > 1 && E && !std::getenv("CUSHA_NO_CHUNK_SORT");
+  if (chunk_sort) {
+    size_t fr = 0, tot = 0;
+    chunk_sort = cudaMemGetInfo(&fr, &tot) == cudaSuccess && fr > 48 * E + (2ull << 30);
+  }
+  DevBuf keys3, ids3, splits;
   CK(dalloc((uint64_t**)&keys.p, E));
   CK(dalloc((uint64_t**)&keys2.p, E));
   CK(dalloc((uint32_t**)&ids.p, E));
   CK(dalloc((uint32_t**)&ids2.p, E));
+  uint64_t max_chunk = 0;
+  if (chunk_sort) {
+    for (int c = 0; c < nch; ++c) max_chunk = std::max(max_chunk, chunks->bounds[c + 1] - chunks->bounds[c]);
+    CK(dalloc((uint64_t**)&keys3.p, E));
+    CK(dalloc((uint32_t**)&ids3.p, E));
+    CK(dalloc((uint64_t**)&splits.p, E / kMergeTile + 2));
+    size_t tb = 0;
+    cub::DoubleBuffer<uint64_t> kq(nullptr, nullptr);
+    cub::DoubleBuffer<uint32_t> vq(nullptr, nullptr);
+    CK(cub::DeviceRadixSort::SortPairs(nullptr, tb, kq, vq, (int64_t)max_chunk, 0, total, st));
+    CK(dev_alloc(&temp.p, tb ? tb : 1, st));
+  }
   CK(dalloc(&g.d_outdeg, V));
-  CK(dalloc((uint32_t**)&indeg.p, V));
+  // in-degrees: counted per shard after the scatter when N counters fit in
+  // shared memory, else by global atomics during ingest
+  const bool hist_indeg = 4ull * N <= 96 * 1024;
+  if (!hist_indeg) CK(dalloc((uint32_t**)&indeg.p, V));
   CK(dalloc((uint32_t**)&mx.p, 2));
   pt.mark("alloc keys/ids");
   CK(dalloc((uint32_t**)&bad.p, 1));
   CK(cudaMemsetAsync(bad.p, 0, 4, st));
   CK(cudaMemsetAsync(g.d_outdeg, 0, (size_t)V * 4, st));
-  CK(cudaMemsetAsync(indeg.p, 0, (size_t)V * 4, st));
+  if (!hist_indeg) CK(cudaMemsetAsync(indeg.p, 0, (size_t)V * 4, st));
   CK(cudaMemsetAsync(mx.p, 0, 8, st));
   // keys + degrees per input chunk, each as soon as its host copy has landed
-  const int nchunks = chunks && chunks->n ? chunks->n : 1;
-  for (int c = 0; c < nchunks; ++c) {
+  // chunked sort: raw chunk c lands in (keys, ids)[lo, hi); it is sorted with
+  // (keys2, ids2)[lo, hi) as the alternate buffer — free, since the sorted
+  // prefix occupies [0, lo) of whichever of (keys2, ids2) / (keys3, ids3) holds
+  // it — and merged with the prefix into the other one.
+  uint64_t* pk = (uint64_t*)keys2.p;
+  uint32_t* pi = (uint32_t*)ids2.p;
+  uint64_t* qk = (uint64_t*)keys3.p;
+  uint32_t* qi = (uint32_t*)ids3.p;
+  for (int c = 0; c < nch; ++c) {
     const uint64_t lo = chunks && chunks->n ? chunks->bounds[c] : 0, hi = chunks && chunks->n ? chunks->bounds[c + 1] : E;
     if (chunks && chunks->n) CK(cudaStreamWaitEvent(st, chunks->ready[c], 0));
     if (hi > lo)
       k_ingest<<<grid_for(hi - lo), 256, 0, st>>>(d_src, d_dst, lo, hi, V, N, bn, bsrc, (uint64_t*)keys.p,
                                                   (uint32_t*)ids.p, (uint32_t*)bad.p, g.d_outdeg, (uint32_t*)indeg.p);
+    if (chunk_sort) {
+      const uint64_t n = hi - lo;
+      cub::DoubleBuffer<uint64_t> kq((uint64_t*)keys.p + lo, pk + lo);
+      cub::DoubleBuffer<uint32_t> vq((uint32_t*)ids.p + lo, pi + lo);
+      size_t tb = 0;
+      CK(cub::DeviceRadixSort::SortPairs(nullptr, tb, kq, vq, (int64_t)max_chunk, 0, total, st));
+      if (n) CK(cub::DeviceRadixSort::SortPairs(temp.p, tb, kq, vq, (int64_t)n, 0, total, st));
+      const uint64_t tiles = (hi + kMergeTile - 1) / kMergeTile;
+      k_merge_splits<<<grid_for(tiles + 1), 256, 0, st>>>(pk, lo, kq.Current(), n, tiles, (uint64_t*)splits.p);
+      if (tiles)
+        k_merge<<<(unsigned)tiles, kMergeThreads, 0, st>>>(pk, pi, lo, kq.Current(), vq.Current(), n,
+                                                            (uint64_t*)splits.p, qk, qi);
+      std::swap(pk, qk);
+      std::swap(pi, qi);
+    }
   }
   CK(cudaGetLastError());
   // range of the float algorithms' fixed-point sums (include/cusha.h "Fixed-point range")
-  k_max_u32<<<grid_for(V), 256, 0, st>>>((uint32_t*)indeg.p, V, (uint32_t*)mx.p);
-  uint32_t h[2] = {0, 0};
-  CK(cudaMemcpyAsync(h, mx.p, 4, cudaMemcpyDeviceToHost, st));
+  if (!hist_indeg) k_max_u32<<<grid_for(V), 256, 0, st>>>((uint32_t*)indeg.p, V, (uint32_t*)mx.p);
+  // h and ev_bits receive async copies: the guard drains the stream before they go
+  uint32_t h[2] = {0, 0}, ev_bits = 0;
+  struct DrainOnExit {
+    cudaStream_t s;
+    ~DrainOnExit() { cudaStreamSynchronize(s); }
+  } drain{st};
   CK(cudaMemcpyAsync(h + 1, bad.p, 4, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   if (h[1]) { err = "edge endpoint >= num_vertices"; return CUSHA_EINVAL; }
-  g.max_indeg = h[0];
   pt.mark("keys + degrees + validate");
 
   // ---- G-Shards order
   cub::DoubleBuffer<uint64_t> kb((uint64_t*)keys.p, (uint64_t*)keys2.p);
   cub::DoubleBuffer<uint32_t> vb((uint32_t*)ids.p, (uint32_t*)ids2.p);
   size_t tbytes = 0;
-  if (E) {
+  if (E && !chunk_sort) {
     CK(cub::DeviceRadixSort::SortPairs(nullptr, tbytes, kb, vb, (int64_t)E, 0, total, st));
     CK(dev_alloc(&temp.p, tbytes, st));
     CK(cub::DeviceRadixSort::SortPairs(temp.p, tbytes, kb, vb, (int64_t)E, 0, total, st));
   }
   pt.mark("G-Shards sort");
-  const uint64_t* K = kb.Current();
-  const uint32_t* I = vb.Current();
+  const uint64_t* K = chunk_sort ? pk : kb.Current();
+  const uint32_t* I = chunk_sort ? pi : vb.Current();
 
   CK(dalloc((uint32_t**)&start.p, (uint64_t)S + 1));
   CK(dalloc((uint64_t**)&padded.p, (uint64_t)S + 1));
@@ -462,7 +593,6 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   if (d_val) { CK(dalloc(&g.d_ev, P)); g.has_ev = true; }
   pt.mark("offsets + alloc shard arrays");
   if (chunks && chunks->n) CK(cudaStreamWaitEvent(st, chunks->all, 0));  // the edge values' copy trails the src/dst chunks
-  uint32_t ev_bits = 0;
   if (d_val && E) {
     k_max_abs_f32<<<grid_for(E), 256, 0, st>>>(d_val, E, (uint32_t*)mx.p + 1);
     CK(cudaMemcpyAsync(&ev_bits, (uint32_t*)mx.p + 1, 4, cudaMemcpyDeviceToHost, st));
@@ -472,6 +602,29 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
   if (E)
     k_scatter_gs<<<grid_for(E), 256, 0, st>>>(K, I, E, (uint32_t*)start.p, g.d_shard_off, bn, bsrc, d_val, N, g.d_dest,
                                               g.d_srcloc, g.d_eid, g.d_ev);
+  // the in-degree count only reads DestIndex: a side stream runs it beside the
+  // window table and CW (joined before the build returns)
+  struct Side {
+    cudaStream_t s = nullptr;
+    cudaEvent_t fork = nullptr, join = nullptr;
+    ~Side() {
+      if (s) { cudaStreamSynchronize(s); cudaStreamDestroy(s); }
+      if (fork) cudaEventDestroy(fork);
+      if (join) cudaEventDestroy(join);
+    }
+  } side;
+  CK(cudaStreamCreateWithFlags(&side.s, cudaStreamNonBlocking));
+  CK(cudaEventCreateWithFlags(&side.fork, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&side.join, cudaEventDisableTiming));
+  CK(cudaEventRecord(side.fork, st));
+  CK(cudaStreamWaitEvent(side.s, side.fork, 0));
+  if (hist_indeg && E) {
+    if (4ull * N > 48 * 1024)
+      CK(cudaFuncSetAttribute(k_indeg_max, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(4 * N)));
+    k_indeg_max<<<S, 256, 4 * N, side.s>>>(g.d_dest, g.d_shard_off, g.d_shard_cnt, N, (uint32_t*)mx.p);
+  }
+  CK(cudaMemcpyAsync(h, mx.p, 4, cudaMemcpyDeviceToHost, side.s));
+  CK(cudaEventRecord(side.join, side.s));
   CK(cudaGetLastError());
 
   // ---- window table W_ij (both representations keep it; GS stage 4 reads it)
@@ -534,8 +687,10 @@ int build_layout(Graph& g, const uint32_t* d_src, const uint32_t* d_dst, const u
     }
   }
   pt.mark("Mapper runs");
+  CK(cudaStreamWaitEvent(st, side.join, 0));
   CK(cudaStreamSynchronize(st));
   std::memcpy(&g.max_abs_ev, &ev_bits, 4);
+  g.max_indeg = h[0];
   return CUSHA_OK;
 }
 

@@ -178,6 +178,7 @@ def test_layout_matches_oracle(repr, V, E, N):
             cw_win = cusha.get_layout(g, "cw_window").astype(np.int64)
             cw_delta = cusha.get_layout(g, "cw_delta").astype(np.int64).reshape(S, S)
     assert st["num_shards"] == S and st["vertices_per_shard"] == N
+    assert st["max_in_degree"] == (np.bincount(d, minlength=V).max() if E else 0)
     np.testing.assert_array_equal(cnt, np.diff(ref["shard_off"].astype(np.int64)))
     assert (off % 8 == 0).all()
     # unpadded view: real entries of each shard in order
@@ -327,3 +328,57 @@ def test_layout_shuffled_duplicates_self_loops(repr):
                                   ("cc", oracle.cc(V, s, d), None)):
                 assert cusha.run(alg, g) == cusha.OK
                 np.testing.assert_array_equal(cusha.get_values(g), want, err_msg=f"{alg} N={N}")
+
+
+# ------------------------------ chunked sort of a host edge list (row f2)
+@pytest.mark.parametrize("repr", REPRS)
+def test_layout_chunked_host_sort(repr, monkeypatch):
+    """A host edge list of >= 2^22 edges crosses in 8 chunks, each radix-sorted
+    as it lands and merged into the sorted prefix (builder.cu k_merge).  On a
+    shuffled list with many duplicate edges spread over every chunk (ties
+    across chunk boundaries, R17) the layout is bit-exact against
+    oracle.build_shards and identical to the single-sort build."""
+    V = 1500
+    s, d = graphgen.rmat(V, 300000, seed=83)
+    rng = np.random.default_rng(83)
+    pick = rng.integers(0, len(s), (1 << 22) + 12345 - len(s))
+    s = np.concatenate([s, s[pick]])
+    d = np.concatenate([d, d[pick]])
+    perm = rng.permutation(len(s))
+    s, d = s[perm].astype(np.uint32), d[perm].astype(np.uint32)
+    N = 200
+    ref = oracle.build_shards(V, s, d, N)
+    S = ref["S"]
+    parts = ("edge_id", "dest_local") + (("mapper", "cw_src_local") if repr == "cw" else ("src_index",))
+    got = {}
+    for chunked in (True, False):
+        if chunked:
+            monkeypatch.delenv("CUSHA_NO_CHUNK_SORT", raising=False)
+        else:
+            monkeypatch.setenv("CUSHA_NO_CHUNK_SORT", "1")
+        with cusha.build_graph(V, s, d, repr=repr, vertices_per_shard=N, keep_layout=True) as g:
+            got[chunked] = {p: cusha.get_layout(g, p) for p in parts + ("shard_offsets", "shard_sizes")}
+            if chunked:
+                max_indeg = cusha.get_stats(g)["max_in_degree"]
+                assert cusha.run("bfs", g) == cusha.OK
+                np.testing.assert_array_equal(cusha.get_values(g), oracle.bfs(V, s, d, 0))
+    for p in got[True]:
+        np.testing.assert_array_equal(got[True][p], got[False][p], err_msg=p)
+    off = got[True]["shard_offsets"].astype(np.int64)
+    cnt = got[True]["shard_sizes"].astype(np.int64)
+    real = np.concatenate([np.arange(off[j], off[j] + cnt[j]) for j in range(S)])
+    np.testing.assert_array_equal(got[True]["edge_id"][real], ref["gs_eid"])
+    assert max_indeg == np.bincount(d, minlength=V).max()
+    np.testing.assert_array_equal(got[True]["dest_local"][real].astype(np.int64) + np.repeat(np.arange(S), cnt) * N,
+                                  ref["gs_dst"])
+
+
+def test_max_in_degree_both_counting_paths():
+    """The largest in-degree (fixed-point range check) is counted per shard in
+    shared memory for N <= 24576 and by global atomics during ingest above."""
+    V = 70000
+    s, d = graphgen.rmat(V, 400000, seed=84)
+    want = np.bincount(d, minlength=V).max()
+    for N in (1000, 30000):
+        with cusha.build_graph(V, s, d, repr="cw", vertices_per_shard=N) as g:
+            assert cusha.get_stats(g)["max_in_degree"] == want

@@ -1,7 +1,9 @@
 """Time cusha_build_graph phases (CUSHA_DEBUG_BUILD=1) for a workload, host and device inputs."""
 import os, sys, time
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-os.environ["CUSHA_DEBUG_BUILD"] = "1"
+if "--quiet" not in sys.argv:
+    os.environ["CUSHA_DEBUG_BUILD"] = "1"
+sys.argv = [a for a in sys.argv if a != "--quiet"]
 import numpy as np, torch
 import graphgen
 from paper_conf_hpdc_khorasanivgb14_b200 import cusha
@@ -9,7 +11,7 @@ wl = graphgen.workload(sys.argv[1] if len(sys.argv) > 1 else "C2", cache_dir="/t
 repr_ = sys.argv[2] if len(sys.argv) > 2 else "cw"
 ps = torch.from_numpy(wl.src.view(np.int32)).pin_memory()
 pd = torch.from_numpy(wl.dst.view(np.int32)).pin_memory()
-for k in range(3):
+for k in range(int(os.environ.get("BT_REPS", "3"))):
     torch.cuda.synchronize()
     t = time.perf_counter()
     g = cusha.build_graph(wl.V, ps.numpy().view(np.uint32), pd.numpy().view(np.uint32), repr=repr_)
