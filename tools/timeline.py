@@ -39,6 +39,9 @@ with cusha.build_graph(wl.V, src, dst, edge_values=ev, repr=repr_, vertices_per_
     assert n > 0, cusha.lib().cusha_last_error()
 iters = st["iterations"]
 T = buf.reshape(-1, 10)[: min(n, (iters + 1) * S)].astype(np.int64)
+if out_path:  # raw stamps (row = ticket pass * S + shard) for per-shard analysis
+    np.savez_compressed(out_path.rsplit(".", 1)[0] + "_raw.npz", T=T, S=S, iters=iters,
+                        shard_cnt=cusha.get_layout(g, "shard_sizes"), cw_cnt=cusha.get_layout(g, "cw_sizes"))
 # steady state: skip the first 2 and the last 2 passes
 lo, hi = 2 * S, max(2 * S, (iters - 2) * S)
 T = T[lo:hi]
