@@ -54,6 +54,16 @@ constexpr int kChunk = 16;  // passes per fixed-count graph / per host check (pe
 #define CUSHA_WIDE_WINDOW 4
 #endif
 constexpr uint32_t kWideWindow = CUSHA_WIDE_WINDOW, kLowDegree = 4;
+constexpr uint32_t kHostTrace = 256;  // trace records read back with the Ctl block (more: a second copy)
+
+// launch configuration of the shard pass for one (graph, algorithm): computed
+// once per graph and algorithm (pass_config), reused by every later run
+struct PassCfg {
+  size_t smem = 0;
+  int mapj = 0, stash = 0;
+  uint32_t nst = 0;
+  bool one_cta = false;
+};
 
 }  // namespace cusha
 
@@ -73,6 +83,8 @@ struct cusha_graph {
   cusha_stats st{};
   int last_alg = -1;
   bool have_values = false;
+  cusha::PassCfg cfg[cusha::kNumAlgs];  // pass_config per algorithm (valid where cfg_ok)
+  bool cfg_ok[cusha::kNumAlgs] = {};
 };
 
 namespace cusha {
@@ -105,7 +117,9 @@ static void free_handle(cusha_graph* h) {
   for (Graph* g : h->parts) {
     free_device_arrays(*g);
     nccl_destroy(*g);
-    delete g->h_ctl;
+    if (g->h_ctl) cudaFreeHost(g->h_ctl);
+    for (cudaEvent_t e : {g->ev0, g->evm, g->ev1})
+      if (e) cudaEventDestroy(e);
     delete g;
   }
   h->parts.clear();
@@ -149,8 +163,14 @@ static int alloc_run_state(Graph& g, bool ipc) {
   }
   CKA(dev_alloc((void**)&g.d_ctl, sizeof(Ctl), g.stream));
   CKA(cudaMemsetAsync(g.d_ctl, 0, sizeof(Ctl), g.stream));
-  g.h_ctl = new (std::nothrow) Ctl();
-  if (!g.h_ctl) return fail(CUSHA_ENOMEM, "host allocation");
+  // pinned, so the end-of-run read-back is one asynchronous copy
+  void* hb = nullptr;
+  CKA(cudaMallocHost(&hb, sizeof(Ctl) + sizeof(TraceRec) * kHostTrace));
+  g.h_ctl = new (hb) Ctl();
+  g.h_trace = reinterpret_cast<TraceRec*>(static_cast<uint8_t*>(hb) + sizeof(Ctl));
+  CKA(cudaEventCreate(&g.ev0));
+  CKA(cudaEventCreate(&g.evm));
+  CKA(cudaEventCreate(&g.ev1));
   return CUSHA_OK;
 }
 
@@ -615,12 +635,6 @@ static uint32_t pass_grid(const Graph& g, const PassKernel& pk, size_t smem) {
 #ifndef CUSHA_STASH
 #define CUSHA_STASH 1  // 0: stage 3 of the integer algorithms re-reads VertexValues (tuning comparison)
 #endif
-struct PassCfg {
-  size_t smem = 0;
-  int mapj = 0, stash = 0;
-  uint32_t nst = 0;
-  bool one_cta = false;
-};
 static int pass_config(const Graph& g, const PassKernel& pk, PassCfg* c) {
   cudaFuncAttributes fa{};
   CKA(cudaFuncGetAttributes(&fa, pk.func));
@@ -720,6 +734,26 @@ static int shard_order(Graph& g) {
   CKA(dev_alloc((void**)&g.d_order, 4ull * g.Sl, g.stream));
   CKA(cudaMemcpyAsync(g.d_order, ord.data(), 4ull * g.Sl, cudaMemcpyHostToDevice, g.stream));
   CKA(cudaStreamSynchronize(g.stream));
+  return CUSHA_OK;
+}
+
+// Chunk table of the one-partition CW SrcValue initialisation
+// (init_srcvalue_cw_flat): (shard, first CW position) per kInitChunk entries
+// of every CW_i.  Built once per graph, on the first run.
+static int init_chunks(Graph& g) {
+  if (g.d_init_chunks || g.repr != CUSHA_REPR_CW || g.G != 1 || !g.Sl) return CUSHA_OK;
+  std::vector<uint32_t> off(g.Sl), cnt(g.Sl);
+  CKA(cudaMemcpyAsync(off.data(), g.d_cw_off, 4ull * g.Sl, cudaMemcpyDeviceToHost, g.stream));
+  CKA(cudaMemcpyAsync(cnt.data(), g.d_cw_cnt, 4ull * g.Sl, cudaMemcpyDeviceToHost, g.stream));
+  CKA(cudaStreamSynchronize(g.stream));
+  std::vector<uint2> ch;
+  for (uint32_t s = 0; s < g.Sl; ++s)
+    for (uint64_t k = 0; k < cnt[s]; k += kInitChunk) ch.push_back(make_uint2(s, off[s] + (uint32_t)k));
+  CKA(dev_alloc((void**)&g.d_init_chunks, sizeof(uint2) * std::max<size_t>(ch.size(), 1), g.stream));
+  if (!ch.empty())
+    CKA(cudaMemcpyAsync(g.d_init_chunks, ch.data(), sizeof(uint2) * ch.size(), cudaMemcpyHostToDevice, g.stream));
+  CKA(cudaStreamSynchronize(g.stream));
+  g.init_nchunks = (uint32_t)ch.size();
   return CUSHA_OK;
 }
 
@@ -868,11 +902,16 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
       if (e) { cudaGraphExecDestroy(e); e = nullptr; }
   }
   const PassKernel& pk = pass_kernel(a, g.repr);
-  PassCfg cfg;
-  if ((rc = pass_config(g, pk, &cfg))) return rc;
+  if (!h->cfg_ok[a]) {
+    if ((rc = pass_config(g, pk, &h->cfg[a]))) return rc;
+    h->cfg_ok[a] = true;
+  }
+  const PassCfg& cfg = h->cfg[a];
   if (CUSHA_BIG_FIRST)
     for (Graph* p : h->parts)
       if (!pass_ahead(*p, a) && (rc = shard_order(*p))) return rc;
+  for (Graph* p : h->parts)
+    if ((rc = init_chunks(*p))) return rc;
   const bool parted = h->mode != kModeSingle;
   const bool host_loop = g.host_loop || parted || g.bsp;
   // one launch for the whole run (overlapped passes) unless asked otherwise;
@@ -890,14 +929,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     if (p->trace_dirty) CKA(cudaMemsetAsync(p->d_trace, 0, sizeof(TraceRec) * (size_t)p->trace_dirty, st));
     p->trace_dirty = p->trace_cap;  // until this run's extent is known
   }
-  cudaEvent_t ev0, evm, ev1;
-  CKA(cudaEventCreate(&ev0));
-  CKA(cudaEventCreate(&evm));
-  CKA(cudaEventCreate(&ev1));
-  struct EvGuard {
-    cudaEvent_t a, b, c;
-    ~EvGuard() { cudaEventDestroy(a); cudaEventDestroy(b); cudaEventDestroy(c); }
-  } evg{ev0, evm, ev1};
+  cudaEvent_t ev0 = g.ev0, evm = g.evm, ev1 = g.ev1;
   std::string err;
   CKA(cudaEventRecord(ev0, st));
   for (Graph* p : h->parts) CKA(launch_reset_ctl(p->d_ctl, max_iters, st));
@@ -996,6 +1028,13 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     }
   }
   CKA(cudaEventRecord(ev1, st));
+  // one round trip for every partition's Ctl block and the head of its trace
+  // (the rest, for runs longer than kHostTrace passes, in read_trace)
+  for (Graph* p : h->parts) {
+    CKA(cudaMemcpyAsync(p->h_ctl, p->d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, st));
+    const uint32_t nt = std::min(kHostTrace, p->trace_cap);
+    if (nt) CKA(cudaMemcpyAsync(p->h_trace, p->d_trace, sizeof(TraceRec) * nt, cudaMemcpyDeviceToHost, st));
+  }
   CKA(cudaStreamSynchronize(st));
   float ms = 0, lms = 0;
   cudaEventElapsedTime(&ms, ev0, ev1);
@@ -1005,8 +1044,6 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
   Ctl c0{};
   for (size_t r = 0; r < h->parts.size(); ++r) {
     Graph& p = *h->parts[r];
-    CKA(cudaMemcpyAsync(p.h_ctl, p.d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, st));
-    CKA(cudaStreamSynchronize(st));
     Ctl c = *p.h_ctl;
     {  // passes whose trace records this run touched: its iterations, or every drawn ticket's pass
       const uint64_t drawn = multi && p.Sl ? c.ticket / p.Sl + 1 : 0;
@@ -1017,7 +1054,9 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
       c.iter = c.converged ? c.conv_iter : max_iters;
     }
     std::vector<TraceRec> tr;
-    if ((rc = read_trace(p, std::min(c.iter, p.trace_cap), tr))) return rc;
+    const uint32_t ntr = std::min(c.iter, p.trace_cap);
+    if (ntr <= kHostTrace) tr.assign(p.h_trace, p.h_trace + std::max<uint32_t>(ntr, 1));
+    else if ((rc = read_trace(p, ntr, tr))) return rc;
     account_run(p, a, c, multi, cfg.mapj != 0, p.st, tr);
     p.st.run_ms = ms;
     p.st.loop_ms = lms;

@@ -787,7 +787,8 @@ void free_device_arrays(Graph& g) {
   void* ptrs[] = {g.d_shard_off, g.d_shard_cnt, g.d_dest, g.d_srcloc, g.d_eid, g.d_ev, g.d_win, g.d_cw_off,
                   g.d_cw_cnt, g.d_cw_src, g.d_mapper, g.d_outdeg, g.d_ctl, g.d_trace, g.d_sync_peer,
                   g.d_active, g.d_bounds, g.d_owner, g.d_cwp, g.d_run_k, g.d_run_t, g.d_sv_peer, g.d_dirty_peer,
-                  g.d_run_unit, g.d_run_bits, g.d_run_d, g.d_shard_seq, g.d_cw_win, g.d_cw_delta, g.d_order};
+                  g.d_run_unit, g.d_run_bits, g.d_run_d, g.d_shard_seq, g.d_cw_win, g.d_cw_delta, g.d_order,
+                  g.d_init_chunks};
   for (void* p : ptrs)
     if (p) cudaFreeAsync(p, g.stream);
   if (g.d_dirty) {
@@ -820,6 +821,8 @@ void free_device_arrays(Graph& g) {
   g.d_dest = g.d_srcloc = g.d_cw_src = g.d_cw_win = nullptr;
   g.d_eid = g.d_ev = g.d_bounds = g.d_cwp = g.d_run_k = g.d_run_t = g.d_run_unit = g.d_run_bits = g.d_run_d = nullptr;
   g.d_shard_seq = g.d_cw_delta = g.d_dirty = g.d_srcvalue = g.d_order = nullptr;
+  g.d_init_chunks = nullptr;
+  g.init_nchunks = 0;
   g.d_vv = nullptr; g.d_ctl = nullptr; g.d_trace = nullptr; g.d_active = nullptr; g.d_owner = nullptr;
   g.d_sv_peer = nullptr; g.d_dirty_peer = nullptr;
   g.h_dest = nullptr; g.h_ev = nullptr; g.h_srcloc = nullptr; g.h_eid = nullptr; g.h_cw_src = nullptr;

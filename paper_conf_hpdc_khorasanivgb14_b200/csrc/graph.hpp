@@ -164,6 +164,8 @@ struct Graph {
   uint32_t* d_dirty = nullptr;      // Sl: clean-shard skipping flags
   uint32_t* d_shard_seq = nullptr;  // Sl: overlapped passes, per-shard pass order
   uint32_t* d_order = nullptr;      // Sl: largest shards first (L2-resident passes; built on first use)
+  uint2* d_init_chunks = nullptr;   // CW init: (shard, first CW position) per chunk of kInitChunk entries (first run)
+  uint32_t init_nchunks = 0;
   int pass_barrier = 0;             // 0: automatic, 1: one launch per pass, 2: overlapped
   bool skip_clean = false;
   // host-streamed topology (row f3): shards >= host_shard keep their entry
@@ -204,8 +206,11 @@ struct Graph {
   TraceRec* d_trace = nullptr;
   uint32_t trace_cap = 0;
   uint32_t trace_dirty = 0;         // leading trace records a previous run may have written
-  Ctl* h_ctl = nullptr;             // host mirror
-  cudaEvent_t ev0 = nullptr, ev1 = nullptr, evm = nullptr;
+  // pinned host mirror: the Ctl block, then the first kHostTrace trace records,
+  // read back in one copy at the end of a run
+  Ctl* h_ctl = nullptr;
+  TraceRec* h_trace = nullptr;
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr, evm = nullptr;  // run timing (created once per graph)
   // destination-range partition (row e)
   int world_size = 1, rank = 0;
   uint32_t G = 1;                   // partitions (1: unpartitioned)
@@ -232,6 +237,8 @@ struct Graph {
 
 // kernels.cu
 const PassKernel& pass_kernel(int alg, int repr);
+// CW entries per block of the SrcValue initialisation (one partition, G = 1)
+constexpr uint32_t kInitChunk = 2048;
 cudaError_t launch_init(const Graph& g, int alg, uint32_t source, cudaStream_t s);
 cudaError_t launch_reset_ctl(Ctl* ctl, uint32_t max_iters, cudaStream_t s);
 cudaError_t launch_close_parts(Ctl* const* ctls, uint32_t G, cudaStream_t s);  // partitioned: global convergence

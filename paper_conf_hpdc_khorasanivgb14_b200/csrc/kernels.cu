@@ -23,6 +23,8 @@
 // previous pass (a misprediction only costs bandwidth: an unpredicted active
 // shard reads its index arrays directly, a predicted inactive one drops them).
 #include <cstdio>
+#include <map>
+#include <mutex>
 
 #include "algorithms.cuh"
 #include "graph.hpp"
@@ -352,8 +354,9 @@ __device__ __forceinline__ bool wb_get(const uint32_t* sm, const uint32_t* aux, 
   if (A::kMonotone) {
     // integer algorithms: local == committed value whenever not updated, so
     // copies of unchanged vertices already hold it (R19) — store only changed
+    if (!((aux[l >> 5] >> (l & 31)) & 1u)) return false;
     val = sm[l];
-    return (aux[l >> 5] >> (l & 31)) & 1u;
+    return true;
   } else {
     val = aux[l];  // local_vertices as left by update_condition (Fig. 5 line 25)
     return true;
@@ -917,9 +920,24 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
 #pragma unroll
                 for (uint32_t u = 0; u < kS4U; ++u) {
                   const uint32_t i = i0 + u * kConsumers;
-                  const uint32_t j = i < d.hi ? (uint32_t)J[i] : 0xFFFFu;
-                  ok[u] = j != 0xFFFFu && wb_get<A>(sm, aux, L[i], val[u]);
-                  tg[u] = (ok[u] ? drow[j] : 0u) + d.base + i;
+                  if constexpr (A::kMonotone) {
+                    // the changed bit first: an unchanged source costs two shared
+                    // loads (SrcIndexCW, its bit), not five (padding entries carry
+                    // SrcIndexCW 0, a valid index, and window 0xFFFF)
+                    const uint32_t l = i < d.hi ? (uint32_t)L[i] : 0u;
+                    ok[u] = i < d.hi && ((aux[l >> 5] >> (l & 31)) & 1u);
+                    tg[u] = 0u;
+                    if (ok[u]) {
+                      const uint32_t j = J[i];
+                      ok[u] = j != 0xFFFFu;
+                      val[u] = sm[l];
+                      tg[u] = (ok[u] ? drow[j] : 0u) + d.base + i;
+                    }
+                  } else {
+                    const uint32_t j = i < d.hi ? (uint32_t)J[i] : 0xFFFFu;
+                    ok[u] = j != 0xFFFFu && wb_get<A>(sm, aux, L[i], val[u]);
+                    tg[u] = (ok[u] ? drow[j] : 0u) + d.base + i;
+                  }
                 }
 #pragma unroll
                 for (uint32_t u = 0; u < kS4U; ++u)
@@ -934,8 +952,15 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
 #pragma unroll
                 for (uint32_t u = 0; u < kS4U; ++u) {
                   const uint32_t i = i0 + u * kConsumers;
-                  tg[u] = i < d.hi ? M[i] : 0u;
-                  ok[u] = i < d.hi && wb_get<A>(sm, aux, L[i], val[u]);
+                  if constexpr (A::kMonotone) {  // the changed bit first (as above)
+                    const uint32_t l = i < d.hi ? (uint32_t)L[i] : 0u;
+                    ok[u] = i < d.hi && ((aux[l >> 5] >> (l & 31)) & 1u);
+                    tg[u] = ok[u] ? M[i] : 0u;
+                    if (ok[u]) val[u] = sm[l];
+                  } else {
+                    tg[u] = i < d.hi ? M[i] : 0u;
+                    ok[u] = i < d.hi && wb_get<A>(sm, aux, L[i], val[u]);
+                  }
                 }
 #pragma unroll
                 for (uint32_t u = 0; u < kS4U; ++u)
@@ -1152,6 +1177,45 @@ __global__ void __launch_bounds__(512) init_srcvalue_cw(const KParams p) {
   }
 }
 
+// One partition (G = 1): SrcValue[Mapper[k]] = wb_value(VertexValues[SrcIndexCW[k]])
+// over every CW entry k (R20), one block per chunk of kInitChunk entries of one
+// CW_i (chunks[b] = (i, first position)), 8 entries per thread with every
+// load issued before the stores: the entries are independent, so the stream
+// runs at bandwidth instead of one dependent chain per thread and shard.
+template <class A>
+__global__ void __launch_bounds__(256) init_srcvalue_cw_flat(const KParams p, const uint2* chunks) {
+  using V_t = typename A::Value;
+  constexpr uint32_t kU = kInitChunk / 256;
+  const uint2 c = chunks[blockIdx.x];
+  const uint32_t i = c.x, e = min(c.y + kInitChunk, p.cw_off[i] + p.cw_cnt[i]);
+  const V_t* vv = reinterpret_cast<const V_t*>(p.vv) + (size_t)i * p.N;
+  const uint32_t* od = p.outdeg + (size_t)i * p.N;
+  const uint32_t* drow = p.cw_delta + (size_t)i * p.S;
+  uint32_t l[kU], m[kU];
+#pragma unroll
+  for (uint32_t u = 0; u < kU; ++u) {
+    const uint32_t k = c.y + u * 256 + threadIdx.x;
+    l[u] = 0;
+    m[u] = 0;
+    if (k < e) {
+      l[u] = __ldg(topo_at(p.cw_src, p.cw_src_h, p.splitQ, k));
+      m[u] = p.mapper ? __ldg(topo_at(p.mapper, p.mapper_h, p.splitQ, k)) : __ldg(topo_at(p.cw_win, p.cw_win_h, p.splitQ, k));
+    }
+  }
+  uint32_t val[kU];
+#pragma unroll
+  for (uint32_t u = 0; u < kU; ++u) {
+    const uint32_t k = c.y + u * 256 + threadIdx.x;
+    if (k < e) {
+      if (!p.mapper) m[u] = __ldg(drow + m[u]) + k;
+      val[u] = A::wb_value(vv[l[u]], A::kOutDeg ? __ldg(od + l[u]) : 0u);
+    }
+  }
+#pragma unroll
+  for (uint32_t u = 0; u < kU; ++u)
+    if (c.y + u * 256 + threadIdx.x < e) p.srcvalue[m[u]] = val[u];
+}
+
 __global__ void reset_ctl(Ctl* ctl, uint32_t max_iters) {
   ctl->iter = 0;
   ctl->changed = 0;
@@ -1244,6 +1308,21 @@ KParams make_params(const Graph& g, uint32_t source) {
   return p;
 }
 
+// cudaFuncSetAttribute once per (kernel, device, size): the per-run launch
+// path then makes no attribute calls
+static cudaError_t smem_attr(const void* fn, size_t bytes) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, size_t> done;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lock(mu);
+  size_t& have = done[{fn, dev}];
+  if (have >= bytes) return cudaSuccess;
+  const cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  if (e == cudaSuccess) have = bytes;
+  return e;
+}
+
 template <class A>
 static cudaError_t launch_init_t(const Graph& g, uint32_t source, cudaStream_t s) {
   KParams p = make_params(g, source);
@@ -1252,10 +1331,15 @@ static cudaError_t launch_init_t(const Graph& g, uint32_t source, cudaStream_t s
   if (g.Sl) {
     const size_t sm = 4ull * g.N;  // the shard's write-back values (|N| <= 65534: at most 256 KB)
     const void* fn = g.repr == CUSHA_REPR_CW ? (const void*)&init_srcvalue_cw<A> : (const void*)&init_srcvalue_gs<A>;
-    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaError_t e = smem_attr(fn, sm);
     if (e != cudaSuccess) return e;  // |N| beyond the shared-memory limit cannot run the pass either
-    if (g.repr == CUSHA_REPR_CW) init_srcvalue_cw<A><<<g.Sl, 512, sm, s>>>(p);
-    else init_srcvalue_gs<A><<<g.Sl, 512, sm, s>>>(p);
+    if (g.repr == CUSHA_REPR_CW && g.G == 1 && g.d_init_chunks) {
+      if (g.init_nchunks) init_srcvalue_cw_flat<A><<<g.init_nchunks, 256, 0, s>>>(p, g.d_init_chunks);
+    } else if (g.repr == CUSHA_REPR_CW) {
+      init_srcvalue_cw<A><<<g.Sl, 512, sm, s>>>(p);
+    } else {
+      init_srcvalue_gs<A><<<g.Sl, 512, sm, s>>>(p);
+    }
   }
   return cudaGetLastError();
 }

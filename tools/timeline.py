@@ -37,11 +37,12 @@ with cusha.build_graph(wl.V, src, dst, edge_values=ev, repr=repr_, vertices_per_
     buf = np.zeros((1 << 18) * 10, dtype=np.uint32)
     n = cusha.lib().cusha_diag_timeline(buf.ctypes.data, buf.nbytes)
     assert n > 0, cusha.lib().cusha_last_error()
+    shard_cnt, cw_cnt = cusha.get_layout(g, "shard_sizes"), cusha.get_layout(g, "cw_sizes")
 iters = st["iterations"]
 T = buf.reshape(-1, 10)[: min(n, (iters + 1) * S)].astype(np.int64)
 if out_path:  # raw stamps (row = ticket pass * S + shard) for per-shard analysis
     np.savez_compressed(out_path.rsplit(".", 1)[0] + "_raw.npz", T=T, S=S, iters=iters,
-                        shard_cnt=cusha.get_layout(g, "shard_sizes"), cw_cnt=cusha.get_layout(g, "cw_sizes"))
+                        shard_cnt=shard_cnt, cw_cnt=cw_cnt)
 # steady state: skip the first 2 and the last 2 passes
 lo, hi = 2 * S, max(2 * S, (iters - 2) * S)
 T = T[lo:hi]
