@@ -95,7 +95,7 @@ constexpr bool kBk = CUSHA_BK != 0;
 #define CUSHA_AHEAD_WAIT 1  // the read-ahead starts before the producer's ticket_wait
 #endif
 #ifndef CUSHA_EARLY_SEQ
-#define CUSHA_EARLY_SEQ 1  // a shard's next pass is released by the consumers at the end of its ticket, not by the bookkeeper
+#define CUSHA_EARLY_SEQ 1  // a shard's next pass is released at the end of its ticket: 1 by the consumers, 2 by the bookkeeper warp before its bookkeeping (0: after it)
 #endif
 #ifndef CUSHA_DROW_ASYNC
 #define CUSHA_DROW_ASYNC 1  // the stage-4 delta row arrives by cp.async during stage 2 (0: loads in stage 1)
@@ -349,11 +349,19 @@ __device__ __forceinline__ void proc8(uint32_t* sm, uint32_t st, const uint4& s0
 }
 
 // stage-4 value of local vertex l and whether it must be stored
+// wbs (integer algorithms with the stage-1 stash): after stage 3 the stash
+// holds each vertex's new value, or A::kNoWb when it did not change - one
+// shared load per entry instead of the changed bit and the value
 template <class A>
-__device__ __forceinline__ bool wb_get(const uint32_t* sm, const uint32_t* aux, uint32_t l, uint32_t& val) {
-  if (A::kMonotone) {
+__device__ __forceinline__ bool wb_get(const uint32_t* sm, const uint32_t* aux, const uint32_t* wbs, uint32_t l,
+                                       uint32_t& val) {
+  if constexpr (A::kMonotone) {
     // integer algorithms: local == committed value whenever not updated, so
     // copies of unchanged vertices already hold it (R19) — store only changed
+    if (wbs) {
+      val = wbs[l];
+      return val != A::kNoWb;
+    }
     if (!((aux[l >> 5] >> (l & 31)) & 1u)) return false;
     val = sm[l];
     return true;
@@ -699,6 +707,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
   uint32_t* const drow = tail + (A::kMonotone ? (N + 31) / 32 : 0);
   // stage 1's VertexValues of the shard, for stage 3 (integer algorithms, p.stash)
   uint32_t* const stash = drow + (p.mapj ? p.S : 0u);
+  const uint32_t* const wbs = (A::kMonotone && p.stash) ? stash : nullptr;
   const uint32_t it0 = *reinterpret_cast<volatile uint32_t*>(&p.ctl->iter);
   // a pass launched after the run converged / hit max_iters is a no-op (host-loop mode)
   if (*reinterpret_cast<volatile uint32_t*>(&p.ctl->converged) || it0 >= p.ctl->max_iters) return;
@@ -815,7 +824,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
       if (CUSHA_TIMELINE && ct == 0) tl_mark(tk, 4);
 
       // ---- stage 3: update_condition, commit to VertexValues, values_updated (lines 15-20, L271)
-      uint32_t my_upd = 0;
+      uint32_t my_upd = 0, my_cnt = 0;
       for (uint32_t base = 0; base < nv; base += kVB * kConsumers) {
         V_t x[kVB];
         uint32_t od[kVB];
@@ -838,15 +847,20 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
             uint32_t wbv = 0;
             up = A::update(sm, st, v, x[u], &out, &wbv, od[u]);
             if (up) vv[v] = out;
-            if (!A::kMonotone) aux[v] = wbv;
+            if constexpr (A::kMonotone) {
+              if (p.stash) stash[v] = up ? out : A::kNoWb;  // stage 4's write-back array (wbs)
+            } else {
+              aux[v] = wbv;
+            }
           }
           const uint32_t m = __ballot_sync(kFull, up);
-          if (lane == 0 && m) atomicAdd(&s_upd, (uint32_t)__popc(m));
+          my_cnt += __popc(m);  // (lane 0's count is the warp's; one shared atomic per warp below)
           const uint32_t w0 = base + u * kConsumers + cwarp * 32;
           if (A::kMonotone && lane == 0 && w0 < nv) aux[w0 >> 5] = m;
           my_upd |= up ? 1u : 0u;
         }
       }
+      if (lane == 0 && my_cnt) atomicAdd(&s_upd, my_cnt);
       // this thread's delta-row copies (issued in stage 1) land before the
       // barrier, so after it every thread sees the whole row (stage 4)
       if (CUSHA_DROW_ASYNC && p.mapj) cp_async_wait_all();
@@ -902,7 +916,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
                   const int ri = r + __popc(word & below);
                   const uint32_t k = sp + lane;
                   uint32_t val;
-                  if (k >= alo && k < ahi && wb_get<A>(sm, aux, L[k - d.base], val)) {
+                  if (k >= alo && k < ahi && wb_get<A>(sm, aux, wbs, L[k - d.base], val)) {
                     st_u32(svq + (k + D[ri]), val);
                     ++stores;
                   }
@@ -925,17 +939,16 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
                     // loads (SrcIndexCW, its bit), not five (padding entries carry
                     // SrcIndexCW 0, a valid index, and window 0xFFFF)
                     const uint32_t l = i < d.hi ? (uint32_t)L[i] : 0u;
-                    ok[u] = i < d.hi && ((aux[l >> 5] >> (l & 31)) & 1u);
+                    ok[u] = i < d.hi && wb_get<A>(sm, aux, wbs, l, val[u]);
                     tg[u] = 0u;
                     if (ok[u]) {
                       const uint32_t j = J[i];
                       ok[u] = j != 0xFFFFu;
-                      val[u] = sm[l];
                       tg[u] = (ok[u] ? drow[j] : 0u) + d.base + i;
                     }
                   } else {
                     const uint32_t j = i < d.hi ? (uint32_t)J[i] : 0xFFFFu;
-                    ok[u] = j != 0xFFFFu && wb_get<A>(sm, aux, L[i], val[u]);
+                    ok[u] = j != 0xFFFFu && wb_get<A>(sm, aux, wbs, L[i], val[u]);
                     tg[u] = (ok[u] ? drow[j] : 0u) + d.base + i;
                   }
                 }
@@ -954,12 +967,11 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
                   const uint32_t i = i0 + u * kConsumers;
                   if constexpr (A::kMonotone) {  // the changed bit first (as above)
                     const uint32_t l = i < d.hi ? (uint32_t)L[i] : 0u;
-                    ok[u] = i < d.hi && ((aux[l >> 5] >> (l & 31)) & 1u);
+                    ok[u] = i < d.hi && wb_get<A>(sm, aux, wbs, l, val[u]);
                     tg[u] = ok[u] ? M[i] : 0u;
-                    if (ok[u]) val[u] = sm[l];
                   } else {
                     tg[u] = i < d.hi ? M[i] : 0u;
-                    ok[u] = i < d.hi && wb_get<A>(sm, aux, L[i], val[u]);
+                    ok[u] = i < d.hi && wb_get<A>(sm, aux, wbs, L[i], val[u]);
                   }
                 }
 #pragma unroll
@@ -985,7 +997,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
         // batch of 32 windows per warp with one entry per lane (gs_walk)
         gs_walk(p, s, lane, cwarp, kConsumerWarps, [&](uint32_t e, uint32_t l) {
           uint32_t val;
-          if (wb_get<A>(sm, aux, l, val)) { st_u32(p.sv_write + e, val); ++stores; }
+          if (wb_get<A>(sm, aux, wbs, l, val)) { st_u32(p.sv_write + e, val); ++stores; }
         });
       }
 #pragma unroll
@@ -1017,7 +1029,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
       // ---- per-shard bookkeeping: convergence flag (line 26), predictor, trace
       if (ct == 0) {
         if (kBk) {
-          if (CUSHA_EARLY_SEQ && p.multi) {
+          if (CUSHA_EARLY_SEQ == 1 && p.multi) {
             // the shard's next pass may start now: every consumer's stores of this
             // ticket precede this fence (barrier above; the fence is cumulative).
             // The trace / done bookkeeping follows in the bookkeeper warp; the
@@ -1052,6 +1064,13 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
         mbar_wait(&bk_full[b], (n >> 1) & 1u);
         const BkRec r = bk[b];
         if (r.s == 0xFFFFFFFFu) break;
+        if (CUSHA_EARLY_SEQ == 2 && p.multi) {
+          // release the shard's next pass first (the consumers' stores precede the
+          // hand-over: barrier, then the mbarrier; this fence is cumulative), so
+          // the fence's latency is off the consumers' path
+          __threadfence();
+          st_vol(&p.shard_seq[r.s], r.it + 1);
+        }
         ticket_bookkeeping(p, r.s, r.it, r.any != 0, r.upd, r.stores, Sloc);
         if (CUSHA_TIMELINE) tl_mark(r.it * Sloc + r.s, 7);
         mbar_arrive(&bk_empty[b]);
