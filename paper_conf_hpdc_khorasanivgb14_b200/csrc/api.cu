@@ -62,6 +62,7 @@ struct PassCfg {
   size_t smem = 0;
   int mapj = 0, stash = 0;
   uint32_t nst = 0;
+  uint32_t grid = 0;  // persistent grid (resident CTAs)
   bool one_cta = false;
 };
 
@@ -698,6 +699,7 @@ static int pass_config(const Graph& g, const PassKernel& pk, PassCfg* c) {
       ++c->nst;
     }
   }
+  c->grid = pass_grid(g, pk, c->smem);
   return CUSHA_OK;
 }
 
@@ -779,7 +781,7 @@ static int ensure_exec(cusha_graph* h, int alg, const PassKernel& pk, const Pass
   void* args[] = {&kp};
   cudaKernelNodeParams knp = {};
   knp.func = const_cast<void*>(pk.func);
-  knp.gridDim = dim3(pass_grid(g, pk, c.smem));
+  knp.gridDim = dim3(c.grid);
   knp.blockDim = dim3(pk.threads);
   knp.sharedMemBytes = (unsigned)c.smem;
   knp.kernelParams = args;
@@ -947,7 +949,7 @@ int cusha_run(cusha_algorithm alg, cusha_graph* h, uint32_t source, uint32_t max
     // DESIGN.md "Overlapped passes")
     kp.window = g.E < (uint64_t)kLowDegree * g.V ? kWideWindow : 2u;
     void* args[] = {&kp};
-    CKA(cudaLaunchKernel(pk.func, dim3(pass_grid(g, pk, cfg.smem)), dim3(pk.threads), args, cfg.smem, st));
+    CKA(cudaLaunchKernel(pk.func, dim3(cfg.grid), dim3(pk.threads), args, cfg.smem, st));
   } else if (max_iters > 0) {
     // passes in chunks; a pass that finds the run converged (or at max_iters)
     // exits at once, so over-launching is exact.  Partitioned: every
