@@ -120,7 +120,7 @@ constexpr uint32_t tile_of() {
 }
 constexpr uint32_t kStages = CUSHA_STAGES;          // ring depth (the default)
 #ifndef CUSHA_MAX_STAGES
-#define CUSHA_MAX_STAGES 6
+#define CUSHA_MAX_STAGES 8
 #endif
 // ring depth of a run (KParams::nst): kStages, or more when shared memory has
 // room for another slot at the same CTAs per SM (chosen by the host)
