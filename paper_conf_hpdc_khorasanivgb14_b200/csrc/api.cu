@@ -118,7 +118,7 @@ static void free_handle(cusha_graph* h) {
   for (Graph* g : h->parts) {
     free_device_arrays(*g);
     nccl_destroy(*g);
-    if (g->h_ctl) cudaFreeHost(g->h_ctl);
+    g->free_mirror();
     for (cudaEvent_t e : {g->ev0, g->evm, g->ev1})
       if (e) cudaEventDestroy(e);
     delete g;
@@ -164,11 +164,20 @@ static int alloc_run_state(Graph& g, bool ipc) {
   }
   CKA(dev_alloc((void**)&g.d_ctl, sizeof(Ctl), g.stream));
   CKA(cudaMemsetAsync(g.d_ctl, 0, sizeof(Ctl), g.stream));
-  // pinned, so the end-of-run read-back is one asynchronous copy
-  void* hb = nullptr;
-  CKA(cudaMallocHost(&hb, sizeof(Ctl) + sizeof(TraceRec) * kHostTrace));
-  g.h_ctl = new (hb) Ctl();
-  g.h_trace = reinterpret_cast<TraceRec*>(static_cast<uint8_t*>(hb) + sizeof(Ctl));
+  // host mirror of the Ctl block and the trace head, read back together at the
+  // end of a run.  Pageable on purpose: pinning (cudaMallocHost / cudaFreeHost)
+  // per graph costs more than the copy it would save (e2e builds and frees a
+  // graph per step)
+  struct HostMirror {
+    Ctl ctl;
+    TraceRec tr[kHostTrace];
+  };
+  HostMirror* hm = new (std::nothrow) HostMirror();
+  if (!hm) return fail(CUSHA_ENOMEM, "host allocation");
+  g.h_ctl = &hm->ctl;
+  g.h_trace = hm->tr;
+  g.h_mirror = hm;
+  g.mirror_deleter = [](void* q) { delete static_cast<HostMirror*>(q); };
   CKA(cudaEventCreate(&g.ev0));
   CKA(cudaEventCreate(&g.evm));
   CKA(cudaEventCreate(&g.ev1));

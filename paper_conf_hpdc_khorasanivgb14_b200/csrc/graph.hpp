@@ -206,10 +206,18 @@ struct Graph {
   TraceRec* d_trace = nullptr;
   uint32_t trace_cap = 0;
   uint32_t trace_dirty = 0;         // leading trace records a previous run may have written
-  // pinned host mirror: the Ctl block, then the first kHostTrace trace records,
-  // read back in one copy at the end of a run
+  // host mirror (api.cu): the Ctl block, then the first kHostTrace trace
+  // records, read back together at the end of a run
   Ctl* h_ctl = nullptr;
   TraceRec* h_trace = nullptr;
+  void* h_mirror = nullptr;
+  void (*mirror_deleter)(void*) = nullptr;
+  void free_mirror() {
+    if (h_mirror && mirror_deleter) mirror_deleter(h_mirror);
+    h_mirror = nullptr;
+    h_ctl = nullptr;
+    h_trace = nullptr;
+  }
   cudaEvent_t ev0 = nullptr, ev1 = nullptr, evm = nullptr;  // run timing (created once per graph)
   // destination-range partition (row e)
   int world_size = 1, rank = 0;

@@ -100,9 +100,6 @@ constexpr bool kBk = CUSHA_BK != 0;
 #ifndef CUSHA_DROW_ASYNC
 #define CUSHA_DROW_ASYNC 1  // the stage-4 delta row arrives by cp.async during stage 2 (0: loads in stage 1)
 #endif
-#ifndef CUSHA_EARLY_DRAW
-#define CUSHA_EARLY_DRAW 0  // 1: draw the next ticket while waiting for a non-predicted shard's stage-3 decision (measured slower)
-#endif
 #ifndef CUSHA_AHEAD4
 #define CUSHA_AHEAD4 1  // the L2 read-ahead also covers CW stage-4 tiles
 #endif
@@ -234,12 +231,11 @@ __device__ __forceinline__ void fence_sc_gpu() { asm volatile("fence.sc.gpu;" ::
 // run stopped meanwhile (the ticket is abandoned - every waiting ticket polls
 // stop, so an abandoned ticket never leaves another one waiting for it)
 // known: every pass below it is known (to this producer) to have completed
-// seq0 / done0: the first reads of both conditions, issued by the caller
-// together with the shard's scalars (one round trip for all of them)
-__device__ __forceinline__ bool ticket_wait(const KParams& p, uint32_t s, uint32_t pass, uint32_t Sloc, uint32_t& known,
-                                            uint32_t seq0, uint32_t done0) {
+__device__ __forceinline__ bool ticket_wait(const KParams& p, uint32_t s, uint32_t pass, uint32_t Sloc, uint32_t& known) {
+  // both conditions' first reads in flight together (the common case: both hold)
   const bool need_w = pass >= p.window && pass - p.window >= known;
-  if (!need_w) done0 = Sloc;
+  const uint32_t seq0 = ld_vol(&p.shard_seq[s]);
+  const uint32_t done0 = need_w ? ld_vol(&p.trace[pass - p.window].done) : Sloc;
   if (seq0 >= pass && done0 >= Sloc) {
     if (need_w) known = pass - p.window + 1;
     __threadfence();                                      // acquire the completed passes' stores ...
@@ -505,45 +501,6 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
   const uint32_t ahead = p.ahead ? CUSHA_AHEAD : 0u;
   const uint32_t max_iters = p.ctl->max_iters;  // constant during the launch
   uint32_t known_done = 0;                      // passes below it have completed (ticket_wait)
-  // a ticket drawn early (overlapped passes, CUSHA_EARLY_DRAW): while the
-  // producer waits for a non-predicted shard's stage-3 decision it already
-  // draws the next ticket, reads its scalars and L2-prefetches its first tiles;
-  // its ticket_wait still follows the current ticket's last push, so it never
-  // waits on a ticket this CTA has not finished pushing
-  struct Drawn {
-    uint32_t s, pass, sb, se, ca, cb, seq0, done0;
-    uint8_t act;
-    bool over;
-  };
-  auto draw = [&](Drawn& n, bool early) {
-    const unsigned long long t = atomicAdd(&p.ctl->ticket, 1ull);
-    n.pass = (uint32_t)(t / Sloc);
-    n.s = (uint32_t)(t - (unsigned long long)n.pass * Sloc);
-    if (p.order && n.pass < max_iters) n.s = p.order[n.s];
-    n.over = n.pass >= max_iters || ld_vol(&p.ctl->stop) != 0;
-    if (CUSHA_TIMELINE && !n.over) tl_mark((uint32_t)t, 0);
-    if (!n.over) {
-      // the shard's scalars and first stage-2 tiles start towards the SM / L2
-      // while the producer waits (a prefetch reads nothing into the CTA, so it
-      // needs no ordering; the offsets are read-only)
-      // the ticket waits' first reads go out with the scalars (ticket_wait)
-      n.seq0 = ld_vol(&p.shard_seq[n.s]);
-      n.done0 = (n.pass >= p.window && n.pass - p.window >= known_done) ? ld_vol(&p.trace[n.pass - p.window].done) : 0u;
-      n.sb = p.shard_off[n.s];
-      n.se = p.shard_off[n.s + 1];
-      n.act = p.active[n.s];
-      if (REPR == CUSHA_REPR_CW && p.G == 1) {
-        n.ca = p.cw_off[n.s];
-        n.cb = n.ca + p.cw_cnt[n.s];
-      }
-      if (CUSHA_AHEAD_WAIT && ahead)
-        for (uint32_t j = 0; j <= ahead; ++j) pf2(n.sb + j * kTile, n.se);
-      else if (early)
-        pf2(n.sb, n.se);  // drawn during the decision wait: its first tile towards L2 meanwhile
-    }
-  };
-  Drawn nxt{};
-  bool have_next = false;
   for (uint32_t round = 0;; ++round) {
     uint32_t s;  // local shard index
     uint32_t sb = 0, se = 0;  // the shard's entry range (read before the waits in overlapped mode)
@@ -551,17 +508,27 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     uint8_t act = 0;          // stage-4 predictor (a hint: a stale read costs bandwidth, not correctness)
     if (p.multi) {
       // overlapped passes: the next ticket, whatever pass it belongs to
-      if (!have_next) draw(nxt, false);
-      have_next = false;
-      s = nxt.s;
-      cur_pass = nxt.pass;
-      sb = nxt.sb;
-      se = nxt.se;
-      ca = nxt.ca;
-      cb = nxt.cb;
-      act = nxt.act;
-      bool over = nxt.over || ld_vol(&p.ctl->stop) != 0;
-      if (!over) over = !ticket_wait(p, s, cur_pass, Sloc, known_done, nxt.seq0, nxt.done0);
+      const unsigned long long t = atomicAdd(&p.ctl->ticket, 1ull);
+      cur_pass = (uint32_t)(t / Sloc);
+      s = (uint32_t)(t - (unsigned long long)cur_pass * Sloc);
+      if (p.order && cur_pass < max_iters) s = p.order[s];
+      bool over = cur_pass >= max_iters || ld_vol(&p.ctl->stop) != 0;
+      if (CUSHA_TIMELINE && !over) tl_mark((uint32_t)t, 0);
+      if (!over) {
+        // the shard's scalars and first stage-2 tiles start towards the SM / L2
+        // while the producer waits (a prefetch reads nothing into the CTA, so it
+        // needs no ordering; the offsets are read-only)
+        sb = p.shard_off[s];
+        se = p.shard_off[s + 1];
+        act = p.active[s];
+        if (REPR == CUSHA_REPR_CW && p.G == 1) {
+          ca = p.cw_off[s];
+          cb = ca + p.cw_cnt[s];
+        }
+        if (CUSHA_AHEAD_WAIT && ahead)
+          for (uint32_t j = 0; j <= ahead; ++j) pf2(sb + j * kTile, se);
+        over = !ticket_wait(p, s, cur_pass, Sloc, known_done);
+      }
       if (over) {
         push(0, kDescDone, 0, 0, nullptr, 0, nullptr, 0, 0, nullptr, 0, 0);
         return;
@@ -638,10 +605,6 @@ __device__ __forceinline__ void producer(const KParams& p, uint8_t* ring, TileDe
     }
     bool send4 = spec;
     if (REPR == CUSHA_REPR_CW && !spec) {
-      if (CUSHA_EARLY_DRAW && p.multi) {
-        draw(nxt, true);
-        have_next = true;
-      }
       mbar_wait(decide_bar, dph);  // consumers finished stage 3 of shard s
       dph ^= 1;
       send4 = *s_any != 0;

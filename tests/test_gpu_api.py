@@ -96,3 +96,36 @@ def test_per_pass_mode_uses_fixed_graph_chunks(c1):
         got, st = gpu_run("bfs", V, s, d, repr="gs", N=128, pass_barrier=True, max_iters=k,
                           expect_converged=False)
         assert st["iterations"] == min(k, st["iterations"]) and st["iterations"] <= k
+
+
+def test_run_host_path_reuse_and_long_trace(c1):
+    """cusha_run's host path: the pass
+    configuration is cached per graph and algorithm, so one handle running
+    different algorithms in turn must give each one's own result; a run of
+    more than 256 passes reads its trace beyond the head copied with the Ctl
+    block, and the trace must account for every committed update."""
+    V, s, d, _ = c1
+    with cusha.build_graph(V, s, d, repr="cw", vertices_per_shard=128) as g:
+        want_bfs = oracle.bfs(V, s, d, 0)
+        want_cc = oracle.cc(V, s, d)
+        for alg in ("bfs", "cc", "bfs", "pr", "cc"):
+            assert cusha.run(alg, g) == cusha.OK
+            got = cusha.get_values(g)
+            if alg == "bfs":
+                np.testing.assert_array_equal(got, want_bfs)
+            elif alg == "cc":
+                np.testing.assert_array_equal(got, want_cc)
+    # a path against the shard order: edges (i+1 -> i), source V-1, |N| = 8.
+    # Shards run in id order, so each pass carries the wave about one shard
+    # further: several hundred passes
+    n = 4000
+    ps = np.arange(1, n, dtype=np.uint32)
+    pd = ps - 1
+    with cusha.build_graph(n, ps, pd, repr="cw", vertices_per_shard=8) as g:
+        assert cusha.run("bfs", g, source=n - 1, max_iters=1 << 16) == cusha.OK
+        np.testing.assert_array_equal(cusha.get_values(g), oracle.bfs(n, ps, pd, n - 1))
+        st = cusha.get_stats(g)
+        assert st["iterations"] > 256
+        upd, act = cusha.get_trace(g)
+        assert len(upd) == st["iterations"]
+        assert int(upd.sum()) == n - 1 == st["updated_total"]  # every vertex but the source commits once
