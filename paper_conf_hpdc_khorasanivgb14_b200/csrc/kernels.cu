@@ -1235,6 +1235,40 @@ __global__ void __launch_bounds__(256) init_srcvalue_cw_flat(const KParams p, co
     if (c.y + u * 256 + threadIdx.x < e) p.srcvalue[m[u]] = val[u];
 }
 
+// Start states uniform except at the source (A::kUniformStart, one partition):
+// SrcValue at t = 0 is wb_value(start(v)) = U for every source v but the BFS /
+// SSSP / SSWP source, so the R20 write-back is a fill of every entry (filler
+// entries included: they reduce into the trash slot) followed by a patch of the
+// source's out-edges - a write-only stream instead of a gather per entry.
+__global__ void fill_u32(uint32_t* a, uint64_t n, uint32_t v) {
+  const uint64_t n4 = n / 4;
+  uint4* a4 = reinterpret_cast<uint4*>(a);  // SrcValue is 256-B aligned (pool allocation)
+  const uint4 q = make_uint4(v, v, v, v);
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n4; i += (uint64_t)gridDim.x * blockDim.x)
+    a4[i] = q;
+  for (uint64_t i = n4 * 4 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    a[i] = v;
+}
+// the source's out-edges: its shard i's CW_i entries with SrcIndexCW == the
+// source's local index (CW), or its windows W_ij (G-Shards)
+template <class A>
+__global__ void patch_source_cw(const KParams p, uint32_t i, uint32_t lsrc, uint32_t val) {
+  const uint32_t a = p.cw_off[i], b = a + p.cw_cnt[i];
+  const uint32_t* drow = p.cw_delta + (size_t)i * p.S;
+  for (uint32_t k = a + blockIdx.x * blockDim.x + threadIdx.x; k < b; k += gridDim.x * blockDim.x)
+    if (__ldg(topo_at(p.cw_src, p.cw_src_h, p.splitQ, k)) == lsrc) {
+      const uint32_t m = p.mapper ? __ldg(topo_at(p.mapper, p.mapper_h, p.splitQ, k))
+                                  : __ldg(drow + __ldg(topo_at(p.cw_win, p.cw_win_h, p.splitQ, k))) + k;
+      p.srcvalue[m] = val;
+    }
+}
+__global__ void __launch_bounds__(512) patch_source_gs(const KParams p, uint32_t i, uint32_t lsrc, uint32_t val) {
+  const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+  gs_walk(p, i, lane, warp, blockDim.x / 32, [&](uint32_t e, uint32_t l) {
+    if (l == lsrc) p.srcvalue[e] = val;
+  });
+}
+
 __global__ void reset_ctl(Ctl* ctl, uint32_t max_iters) {
   ctl->iter = 0;
   ctl->changed = 0;
@@ -1347,6 +1381,18 @@ static cudaError_t launch_init_t(const Graph& g, uint32_t source, cudaStream_t s
   KParams p = make_params(g, source);
   const uint32_t vb = (uint32_t)((g.nvl + 255) / 256);
   init_vertex_values<A><<<vb < 148 * 16 ? (vb ? vb : 1) : 148 * 16, 256, 0, s>>>(p, g.d_init[A::kId], g.v0, g.nvl);
+  if (g.Sl && A::kUniformStart && g.G == 1 && !g.d_init[A::kId] && source < g.V) {
+    // host copies of start(): U for every vertex but the source, the source's own
+    uint32_t U = 0, Vs = 0;
+    if (A::kId == kSSWP) { U = 0u; Vs = kInf; } else { U = kInf; Vs = 0u; }
+    const uint64_t n = g.P + 1;
+    const uint64_t blocks = std::min<uint64_t>((n / 4 + 255) / 256 + 1, 148ull * 16);
+    fill_u32<<<(uint32_t)blocks, 256, 0, s>>>(g.d_srcvalue, n, U);
+    const uint32_t i = source / g.N, lsrc = source - i * g.N;
+    if (g.repr == CUSHA_REPR_CW) patch_source_cw<A><<<148, 256, 0, s>>>(p, i, lsrc, Vs);
+    else patch_source_gs<<<1, 512, 0, s>>>(p, i, lsrc, Vs);
+    return cudaGetLastError();
+  }
   if (g.Sl) {
     const size_t sm = 4ull * g.N;  // the shard's write-back values (|N| <= 65534: at most 256 KB)
     const void* fn = g.repr == CUSHA_REPR_CW ? (const void*)&init_srcvalue_cw<A> : (const void*)&init_srcvalue_gs<A>;
