@@ -246,7 +246,7 @@ struct Graph {
 // kernels.cu
 const PassKernel& pass_kernel(int alg, int repr);
 // CW entries per block of the SrcValue initialisation (one partition, G = 1)
-constexpr uint32_t kInitChunk = 2048;
+constexpr uint32_t kInitChunk = 1024;
 cudaError_t launch_init(const Graph& g, int alg, uint32_t source, cudaStream_t s);
 cudaError_t launch_reset_ctl(Ctl* ctl, uint32_t max_iters, cudaStream_t s);
 cudaError_t launch_close_parts(Ctl* const* ctls, uint32_t G, cudaStream_t s);  // partitioned: global convergence

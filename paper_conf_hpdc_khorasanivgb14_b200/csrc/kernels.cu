@@ -1202,7 +1202,7 @@ __global__ void __launch_bounds__(512) init_srcvalue_cw(const KParams p) {
 // load issued before the stores: the entries are independent, so the stream
 // runs at bandwidth instead of one dependent chain per thread and shard.
 template <class A>
-__global__ void __launch_bounds__(256) init_srcvalue_cw_flat(const KParams p, const uint2* chunks) {
+__global__ void __launch_bounds__(256, 8) init_srcvalue_cw_flat(const KParams p, const uint2* chunks) {
   using V_t = typename A::Value;
   constexpr uint32_t kU = kInitChunk / 256;
   const uint2 c = chunks[blockIdx.x];
