@@ -400,7 +400,9 @@ def bench_cusha(args):
         barrier()
         t0 = time.perf_counter()
         for _ in range(n_e2e):
+            ts = time.perf_counter()
             e2e_edges += e2e_step()
+            log(f"[bench] e2e step {1e3 * (time.perf_counter() - ts):.1f} ms")
         torch.cuda.synchronize()
         el = max_over_ranks(time.perf_counter() - t0)
         e2e_edges = sum_over_ranks(e2e_edges)

@@ -72,6 +72,21 @@ def test_sswp(c1, repr):
     np.testing.assert_array_equal(got, want)
 
 
+@pytest.mark.parametrize("repr", REPRS)
+def test_sources_on_one_graph(c1, repr):
+    """SSSP and SSWP from several sources on one graph, alternating with BFS.
+    Their start state is uniform except at the source, so a run initialises
+    SrcValue by a fill of every entry and a patch of the source's out-edges
+    (DESIGN.md "Host path of a run"); nothing of the previous run may survive."""
+    V, s, d, w = c1
+    with cusha.build_graph(V, s, d, edge_values=w, repr=repr, vertices_per_shard=128) as g:
+        for src in (0, 777, V - 1, 129):
+            for alg, want in (("sssp", oracle.sssp(V, s, d, w, src)), ("sswp", oracle.sswp(V, s, d, w, src)),
+                              ("bfs", oracle.bfs(V, s, d, src))):
+                assert cusha.run(alg, g, source=src) == cusha.OK
+                np.testing.assert_array_equal(cusha.get_values(g), want)
+
+
 # ------------------------------------------------------------------- CC
 @pytest.mark.parametrize("repr", REPRS)
 def test_cc_symmetric(repr):
