@@ -78,7 +78,16 @@ constexpr uint32_t kEPT = CUSHA_EPT;  // stage-2 entries per consumer thread per
 #ifndef CUSHA_S4U
 #define CUSHA_S4U 1
 #endif
-constexpr uint32_t kS4U = CUSHA_S4U;  // stage-4 entries per consumer thread per step (loads before stores)
+#ifndef CUSHA_S4U_INT
+#define CUSHA_S4U_INT 1
+#endif
+// stage-4 entries per consumer thread per step (loads before stores), per
+// kind of algorithm: 2 for the integer ones gained 4% on C4 SSWP but lost up
+// to 7% on C3 depending on the box, 2 for PR lost 2.5% (DESIGN.md tuning log)
+template <class A>
+constexpr uint32_t s4u_of() {
+  return A::kMonotone ? CUSHA_S4U_INT : CUSHA_S4U;
+}
 constexpr uint32_t kConsumerWarps = CUSHA_CONSUMER_WARPS;
 constexpr uint32_t kConsumers = kConsumerWarps * 32;
 #ifndef CUSHA_BK
@@ -174,8 +183,10 @@ constexpr uint32_t kDiag = CUSHA_DIAG;
 // stamps of each ticket's steps, kTlSlots words per ticket, ticket = pass * |S|
 // + shard.  0 producer drew it, 1 producer passed ticket_wait, 2 consumers got
 // its first tile, 3 stage 1 done, 4 stage 2 done, 5 stage 3 done, 6 stage 4
-// done, 7 ticket completed, 8 CTA index, 9 stage-4 tiles were prefetched.
-constexpr uint32_t kTlSlots = 10, kTlCap = 1u << 18;
+// done, 7 ticket completed, 8 CTA index, 9 stage-4 tiles were prefetched,
+// 10 first stage-4 tile acquired, 11 last stage-4 tile processed (thread 0),
+// 12 thread 0 finished its stage-3 vertices (before the stage-3 barrier).
+constexpr uint32_t kTlSlots = 13, kTlCap = 1u << 18;
 #if CUSHA_TIMELINE
 __device__ uint32_t g_timeline[kTlCap * kTlSlots];
 __device__ __forceinline__ void tl_mark(uint32_t ticket, uint32_t k, uint32_t v = 0xFFFFFFFFu) {
@@ -708,6 +719,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
   // stage 1's VertexValues of the shard, for stage 3 (integer algorithms, p.stash)
   uint32_t* const stash = drow + (p.mapj ? p.S : 0u);
   const uint32_t* const wbs = (A::kMonotone && p.stash) ? stash : nullptr;
+  constexpr uint32_t kS4U = s4u_of<A>();
   const uint32_t it0 = *reinterpret_cast<volatile uint32_t*>(&p.ctl->iter);
   // a pass launched after the run converged / hit max_iters is a no-op (host-loop mode)
   if (*reinterpret_cast<volatile uint32_t*>(&p.ctl->converged) || it0 >= p.ctl->max_iters) return;
@@ -861,6 +873,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
         }
       }
       if (lane == 0 && my_cnt) atomicAdd(&s_upd, my_cnt);
+      if (CUSHA_TIMELINE && ct == 0) tl_mark(tk, 12);
       // this thread's delta-row copies (issued in stage 1) land before the
       // barrier, so after it every thread sees the whole row (stage 4)
       if (CUSHA_DROW_ASYNC && p.mapj) cp_async_wait_all();
@@ -879,8 +892,9 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
           mbar_arrive(&decide_bar);
         }
         if (spec4 || any) {
-          for (;;) {
+          for (bool first4 = true;; first4 = false) {
             mbar_wait(&full_bar[slot], ph);
+            if (CUSHA_TIMELINE && ct == 0 && first4) tl_mark(tk, 10);
             d = desc[slot];
             // the partition owning this tile's windows (this one on a single GPU):
             // in the multi-GPU mode the stores below go over NVLink to its SrcValue
@@ -989,7 +1003,10 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty_bar[slot]);
             if (++slot == nst) { slot = 0; ph ^= 1; }
-            if (d.flags & kFlagLast) break;
+            if (d.flags & kFlagLast) {
+              if (CUSHA_TIMELINE && ct == 0) tl_mark(tk, 11);
+              break;
+            }
           }
         }
       } else if (any) {

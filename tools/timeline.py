@@ -34,12 +34,12 @@ with cusha.build_graph(wl.V, src, dst, edge_values=ev, repr=repr_, vertices_per_
     cusha.run(alg, g, source=source)
     st = cusha.get_stats(g)
     S = st["num_shards"]
-    buf = np.zeros((1 << 18) * 10, dtype=np.uint32)
+    buf = np.zeros((1 << 18) * 13, dtype=np.uint32)
     n = cusha.lib().cusha_diag_timeline(buf.ctypes.data, buf.nbytes)
     assert n > 0, cusha.lib().cusha_last_error()
     shard_cnt, cw_cnt = cusha.get_layout(g, "shard_sizes"), cusha.get_layout(g, "cw_sizes")
 iters = st["iterations"]
-T = buf.reshape(-1, 10)[: min(n, (iters + 1) * S)].astype(np.int64)
+T = buf.reshape(-1, 13)[: min(n, (iters + 1) * S)].astype(np.int64)
 if out_path:  # raw stamps (row = ticket pass * S + shard) for per-shard analysis
     np.savez_compressed(out_path.rsplit(".", 1)[0] + "_raw.npz", T=T, S=S, iters=iters,
                         shard_cnt=shard_cnt, cw_cnt=cw_cnt)
