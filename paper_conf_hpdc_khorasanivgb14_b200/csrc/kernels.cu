@@ -1219,7 +1219,9 @@ __global__ void __launch_bounds__(512) init_srcvalue_cw(const KParams p) {
 // load issued before the stores: the entries are independent, so the stream
 // runs at bandwidth instead of one dependent chain per thread and shard.
 template <class A>
-__global__ void __launch_bounds__(256, 8) init_srcvalue_cw_flat(const KParams p, const uint2* chunks) {
+// from_start: VertexValues hold A::start (no user initial values), so the
+// value is computed from the vertex id instead of loaded (PR: Rank 1, CC: the id)
+__global__ void __launch_bounds__(256, 8) init_srcvalue_cw_flat(const KParams p, const uint2* chunks, int from_start) {
   using V_t = typename A::Value;
   constexpr uint32_t kU = kInitChunk / 256;
   const uint2 c = chunks[blockIdx.x];
@@ -1244,7 +1246,8 @@ __global__ void __launch_bounds__(256, 8) init_srcvalue_cw_flat(const KParams p,
     const uint32_t k = c.y + u * 256 + threadIdx.x;
     if (k < e) {
       if (!p.mapper) m[u] = __ldg(drow + m[u]) + k;
-      val[u] = A::wb_value(vv[l[u]], A::kOutDeg ? __ldg(od + l[u]) : 0u);
+      const V_t x = from_start ? A::start((p.s0 + i) * p.N + l[u], p.source) : vv[l[u]];
+      val[u] = A::wb_value(x, A::kOutDeg ? __ldg(od + l[u]) : 0u);
     }
   }
 #pragma unroll
@@ -1416,7 +1419,8 @@ static cudaError_t launch_init_t(const Graph& g, uint32_t source, cudaStream_t s
     cudaError_t e = smem_attr(fn, sm);
     if (e != cudaSuccess) return e;  // |N| beyond the shared-memory limit cannot run the pass either
     if (g.repr == CUSHA_REPR_CW && g.G == 1 && g.d_init_chunks) {
-      if (g.init_nchunks) init_srcvalue_cw_flat<A><<<g.init_nchunks, 256, 0, s>>>(p, g.d_init_chunks);
+      if (g.init_nchunks)
+        init_srcvalue_cw_flat<A><<<g.init_nchunks, 256, 0, s>>>(p, g.d_init_chunks, g.d_init[A::kId] ? 0 : 1);
     } else if (g.repr == CUSHA_REPR_CW) {
       init_srcvalue_cw<A><<<g.Sl, 512, sm, s>>>(p);
     } else {
