@@ -773,6 +773,11 @@ static KParams pass_params(const Graph& g, uint32_t source, const PassCfg& c, in
   kp.mapj = c.mapj;
   kp.stash = c.stash;
   kp.nst = c.nst;
+  {  // one CTA per SM (the few-tickets mode, or shared memory for one only)
+    int sms = 148;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g.device);
+    kp.s4two = c.grid <= (uint32_t)sms ? 1u : 0u;
+  }
   kp.ahead = pass_ahead(g, alg);
   if (CUSHA_BIG_FIRST && !kp.ahead) kp.order = g.d_order;
   return kp;

@@ -84,6 +84,7 @@ struct KParams {
   int stash;                   // 1: integer algorithms keep stage 1's VertexValues in smem for stage 3
   int ahead;                   // 1: the producer prefetches stage-2 tiles into L2 beyond the ring (HBM-resident passes)
   uint32_t nst;                // ring slots of this run (kStages, or more when shared memory has room)
+  uint32_t s4two;              // integer algorithms: two stage-4 entries per thread per step (one CTA per SM)
   uint32_t* shard_seq;         // Sl: passes of shard s completed (overlapped passes)
   const uint32_t* order;       // Sl: shard processed by the q-th ticket of a pass (nullptr: shard order)
   // destination-range partition (row e); G = 1: single partition

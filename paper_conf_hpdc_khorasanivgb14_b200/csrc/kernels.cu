@@ -23,6 +23,7 @@
 // previous pass (a misprediction only costs bandwidth: an unpredicted active
 // shard reads its index arrays directly, a predicted inactive one drops them).
 #include <cstdio>
+#include <type_traits>
 #include <map>
 #include <mutex>
 
@@ -942,11 +943,13 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
               // kS4U entries per thread: every shared load of a step before its stores
               const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
               const uint16_t* J = reinterpret_cast<const uint16_t*>(ring + slot * SLOT + 2 * tile4j_of<A>());
-              for (uint32_t i0 = d.lo + ct; i0 < d.hi; i0 += kS4U * kConsumers) {
-                uint32_t tg[kS4U], val[kS4U];
-                bool ok[kS4U];
+              auto walk = [&](auto u_tag) {
+              constexpr uint32_t kU = decltype(u_tag)::value;
+              for (uint32_t i0 = d.lo + ct; i0 < d.hi; i0 += kU * kConsumers) {
+                uint32_t tg[kU], val[kU];
+                bool ok[kU];
 #pragma unroll
-                for (uint32_t u = 0; u < kS4U; ++u) {
+                for (uint32_t u = 0; u < kU; ++u) {
                   const uint32_t i = i0 + u * kConsumers;
                   if constexpr (A::kMonotone) {
                     // the changed bit first: an unchanged source costs two shared
@@ -967,9 +970,14 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
                   }
                 }
 #pragma unroll
-                for (uint32_t u = 0; u < kS4U; ++u)
+                for (uint32_t u = 0; u < kU; ++u)
                   if (ok[u]) { st_u32(svq + tg[u], val[u]); ++stores; }
               }
+              };
+              // integer algorithms at one CTA per SM (fewer warps to hide the
+              // shared-load chain of each entry): two entries per thread per step
+              if (A::kMonotone && p.s4two) walk(std::integral_constant<uint32_t, 2>{});
+              else walk(std::integral_constant<uint32_t, kS4U>{});
             } else if (any) {
               const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
               const uint32_t* M = reinterpret_cast<const uint32_t*>(ring + slot * SLOT + 2 * tile4m_of<A>());
@@ -1378,6 +1386,7 @@ KParams make_params(const Graph& g, uint32_t source) {
   p.stash = 0;
   p.ahead = 0;
   p.nst = kStages;
+  p.s4two = 0;
   return p;
 }
 
