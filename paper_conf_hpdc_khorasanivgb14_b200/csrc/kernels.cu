@@ -79,6 +79,9 @@ constexpr uint32_t kEPT = CUSHA_EPT;  // stage-2 entries per consumer thread per
 #ifndef CUSHA_S4U
 #define CUSHA_S4U 1
 #endif
+#ifndef CUSHA_S4TWO_ALL
+#define CUSHA_S4TWO_ALL 0  // 1: the float algorithms also take 2 stage-4 entries per step at one CTA per SM
+#endif
 #ifndef CUSHA_S4U_INT
 #define CUSHA_S4U_INT 1
 #endif
@@ -976,7 +979,7 @@ __global__ void __launch_bounds__(kPassThreads, CUSHA_MIN_BLOCKS) shard_pass(con
               };
               // integer algorithms at one CTA per SM (fewer warps to hide the
               // shared-load chain of each entry): two entries per thread per step
-              if (A::kMonotone && p.s4two) walk(std::integral_constant<uint32_t, 2>{});
+              if ((A::kMonotone || CUSHA_S4TWO_ALL) && p.s4two) walk(std::integral_constant<uint32_t, 2>{});
               else walk(std::integral_constant<uint32_t, kS4U>{});
             } else if (any) {
               const uint16_t* L = reinterpret_cast<const uint16_t*>(ring + slot * SLOT);
